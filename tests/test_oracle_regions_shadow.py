@@ -1,0 +1,170 @@
+"""Pins of the oracle's brute-force regions, grid split and shadow tracker (no GPU).
+
+Checked against hand derivations from the kernel definitions,
+closed-form stale-byte minima (oracle/closed_forms.py) and the
+paper's qualitative statements (Fig. 3 text P:L561-566; fragmentation P:L860-870;
+redundant transfers without shared copies P:L929-931).
+"""
+import numpy as np
+import pytest
+
+from oracle import closed_forms as cf
+from oracle import grid, regions, shadow
+
+
+def _rng(a, b):
+    return list(range(a, b))
+
+
+# ------------------------------ grid split (Q1) ------------------------------
+def test_partition_rule():
+    assert grid.split_dim((16, 64, 1)) == grid.Y
+    assert grid.split_dim((8, 128, 16)) == grid.Z
+    assert grid.split_dim((4096, 1, 1)) == grid.X
+    assert grid.split_dim((1, 1, 1)) == grid.X
+    boxes = [grid.partition_box((16, 64, 1), 2, p) for p in range(2)]
+    assert boxes == [(0, 1, 0, 32, 0, 16), (0, 1, 32, 64, 0, 16)]
+    # balanced floor split, empty partitions when P > G
+    assert [grid.partition_box((1, 3, 1), 5, p)[2:4] for p in range(5)] == \
+        [(0, 0), (0, 1), (1, 1), (1, 2), (2, 3)]
+    covered = []
+    for p in range(7):
+        b = grid.partition_box((5, 100, 1), 7, p)
+        covered += _rng(b[2], b[3])
+    assert covered == _rng(0, 100)
+
+
+# ----------------------- C1 worked example (hand derived) -----------------------
+def test_c1_partition0_read_and_write_sets():
+    n = 512
+    acc = regions.jacobi2d(grid.partition_box((16, 64, 1), 2, 0), (32, 8), n, n)
+    # Partition 0 = rows [0, 256).  Threads on rows 1..255, cols 1..510 (Dirichlet).
+    # Row 0: only the 'up' tap of row 1 -> interior cols 1..510.
+    # Rows 1..255: left tap of col 1 reaches col 0, right tap of col 510 reaches 511.
+    # Row 256: only the 'down' tap of row 255 -> interior.
+    r = regions.to_byte_ranges(acc[(0, "r")], 1)
+    assert r == [(1, 511), (512, 131072), (131073, 131583)]
+    w = regions.to_byte_ranges(acc[(1, "w")], 1)
+    assert len(w) == 255 and w[0] == (513, 1023) and w[-1] == (255 * 512 + 1, 255 * 512 + 511)
+    assert sum(e - s for s, e in w) == 130050
+    acc1 = regions.jacobi2d(grid.partition_box((16, 64, 1), 2, 1), (32, 8), n, n)
+    assert regions.to_byte_ranges(acc1[(0, "r")], 1) == [(130561, 131071), (131072, 261632), (261633, 262143)]
+
+
+def test_hotspot_heat_nbody_gemm_sets_shape():
+    # hotspot: clamped 5-point -> one contiguous range rows [r0-1, r1+1) clamped
+    acc = regions.hotspot2d((0, 1, 2, 5, 0, 1), (16,), 40, 64, 4)   # rows 8..19
+    assert regions.to_byte_ranges(acc[(0, "r")], 1) == [(7 * 64, 21 * 64)]
+    assert regions.to_byte_ranges(acc[(1, "r")], 1) == [(8 * 64, 20 * 64)]
+    assert regions.to_byte_ranges(acc[(2, "w")], 1) == [(8 * 64, 20 * 64)]
+    # ragged tail: last block row clipped to H; the top partition clamps at row 0
+    acc = regions.hotspot2d((0, 1, 0, 1, 0, 1), (16,), 3, 64, 4)
+    assert regions.to_byte_ranges(acc[(0, "r")], 1) == [(0, 3 * 64)]
+    # heat: planes
+    acc = regions.heat3d((1, 2, 0, 2, 0, 1), (8, 4), 10, 8, 32, 3)   # planes 3..5
+    assert regions.to_byte_ranges(acc[(0, "r")], 1) == [(2 * 256, 7 * 256)]
+    assert regions.to_byte_ranges(acc[(1, "w")], 1) == [(3 * 256, 6 * 256)]
+    # nbody: everything read, own slab written
+    acc = regions.nbody((0, 1, 0, 1, 2, 3), (64,), 300)
+    assert regions.to_byte_ranges(acc[(0, "r")], 16) == [(0, 300 * 16)]
+    assert regions.to_byte_ranges(acc[(2, "w")], 16) == [(128 * 16, 192 * 16)]
+    # gemm: A row band, B whole, C tile rows
+    acc = regions.gemm((0, 1, 1, 2, 0, 2), 10, 12, 5, 4, 8)
+    assert regions.to_byte_ranges(acc[(0, "r")], 1) == [(20, 40)]
+    assert regions.to_byte_ranges(acc[(1, "r")], 1) == [(0, 60)]
+    assert regions.to_byte_ranges(acc[(2, "w")], 1) == [(48, 96)]
+
+
+# ------------------------------ shadow tracker ------------------------------
+def _jacobi_run(n, nparts, iters, single=False, block=(32, 8)):
+    sh = shadow.Shadow(nparts, single)
+    sh.register("u0", n * n, 4, True)
+    sh.register("u1", n * n, 4, True)
+    g = ((n + block[0] - 1) // block[0], (n + block[1] - 1) // block[1], 1)
+    per_iter = []
+    for t in range(iters):
+        a, b = ("u0", "u1") if t % 2 == 0 else ("u1", "u0")
+        per = []
+        for p in range(nparts):
+            box = grid.partition_box(g, nparts, p)
+            if grid.box_empty(box):
+                per.append(None)
+                continue
+            acc = regions.jacobi2d(box, block, n, n)
+            per.append({a: (acc[(0, "r")], None), b: (None, acc[(1, "w")])})
+        per_iter.append(sum(sh.launch(per)["stale"]))
+    return sh, per_iter
+
+
+def test_c1_stale_bytes_40800():
+    sh, per = _jacobi_run(512, 2, 10)
+    assert per == [cf.jacobi2d_stale_per_iter(512, 2)] * 10
+    assert sh.stale_bytes == 40800
+
+
+def test_misaligned_h2d_redistribution_and_paper_mode_redundancy():
+    # Q2: linear H2D misaligned with P=3 row partitions -> extra first-launch traffic.
+    _, per = _jacobi_run(64, 3, 6)
+    assert per[0] > per[2] and per[2:] == [per[2]] * 4
+    # without shared copies the same halo is re-fetched -> never fewer bytes.
+    _, per_so = _jacobi_run(64, 3, 6, single=True)
+    assert all(a >= b for a, b in zip(per_so, per)) and sum(per_so) > sum(per)
+
+
+@pytest.mark.parametrize("nparts", [2, 3, 4, 8])
+def test_hotspot_steady_state_matches_closed_form(nparts):
+    h = w = 64
+    ty, bdx = 4, 8                                      # block = 32 columns x 4 rows
+    g = ((w + 4 * bdx - 1) // (4 * bdx), (h + ty - 1) // ty, 1)
+    sh = shadow.Shadow(nparts)
+    sh.register("t0", h * w, 4, True)
+    sh.register("t1", h * w, 4, False)
+    sh.register("pw", h * w, 4, True)
+    stale = []
+    for it in range(5):
+        a, b = ("t0", "t1") if it % 2 == 0 else ("t1", "t0")
+        per = []
+        for p in range(nparts):
+            box = grid.partition_box(g, nparts, p)
+            acc = regions.hotspot2d(box, (bdx,), h, w, ty)
+            per.append({a: (acc[(0, "r")], None), "pw": (acc[(1, "r")], None), b: (None, acc[(2, "w")])})
+        stale.append(sum(sh.launch(per)["stale"]))
+    assert stale[1:] == [cf.hotspot2d_stale_per_iter(w, nparts)] * 4
+    # fragmentation: bounded segment count per buffer
+    for name in ("t0", "t1"):
+        assert len(sh.buffers[name].rle()) <= 2 * nparts - 1
+
+
+def test_nbody_allgather_and_validity_vs_single_owner():
+    n, P = 1024, 8
+    sh = shadow.Shadow(P)
+    sh.register("p0", n, 16, True)
+    sh.register("p1", n, 16, False)
+    sh.register("v", n, 16, True)
+    g = (n // 64, 1, 1)
+    tot = 0
+    for s in range(3):
+        a, b = ("p0", "p1") if s % 2 == 0 else ("p1", "p0")
+        per = []
+        for p in range(P):
+            acc = regions.nbody(grid.partition_box(g, P, p), (64,), n)
+            per.append({a: (acc[(0, "r")], None), "v": (acc[(1, "r")], acc[(1, "w")]),
+                        b: (None, acc[(2, "w")])})
+        tot += sum(sh.launch(per)["stale"])
+    assert tot == 3 * cf.nbody_stale_per_step(n, P)
+
+
+def test_write_overlap_is_rejected():
+    sh = shadow.Shadow(2)
+    sh.register("x", 10, 4, False)
+    with pytest.raises(shadow.WriteOverlap):
+        sh.launch([{"x": (None, np.arange(0, 6))}, {"x": (None, np.arange(5, 10))}])
+
+
+def test_rle_and_source_choice():
+    b = shadow.ShadowBuffer(10, 4, 3)
+    b.h2d_linear()
+    assert b.rle() == [(0, 12, 1), (12, 24, 2), (24, 40, 4)]
+    assert shadow.choose_source(0b101, 1, 3) == 0          # tie -> lower
+    assert shadow.choose_source(0b110, 0, 3) == 1
+    assert shadow.choose_source(0b1001, 2, 4) == 3
