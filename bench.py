@@ -1,0 +1,449 @@
+#!/usr/bin/env python
+"""Benchmark of the partitioned hot path (BASELINE.json metric: GLUP/s and roofline
+fraction; stale bytes moved).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload hotspot2d|heat3d|jacobi2d|nbody]
+                    [--parts P] [--impl pk|reference]
+
+A "step" is one pass of the whole hot path over one batch: for the default
+workload (C2, BASELINE.json configs[1]) that is 100 Hotspot iterations on a
+16384 x 16384 fp32 grid, each iteration one pk_launch_partitioned (grid
+partition -> regions -> stale plan -> transfers -> partitioned kernels ->
+tracker update).  ``value`` is device-timed (CUDA events on the library's
+streams via pk_timer_begin/end) with the inputs resident in HBM; ``e2e`` adds
+the H2D upload (pk_copy_from_host from pinned memory) and the D2H gather
+(pk_sync_to_host) of every step and is wall-clock timed.
+
+Process model: one host process drives every GPU of the box, as
+in the paper.  Under torchrun with N ranks, rank 0 drives N
+partitions on devices 0..N-1 and the other ranks only join the barriers; the
+reported time is the max over ranks.  ``--parts P`` runs P partitions as
+virtual devices on the visible GPUs (transfers then are D2D copies).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+WORKLOADS = {
+    # name: (config text, default iterations/steps per bench step)
+    "hotspot2d": ("C2 Hotspot-style 2D stencil 16384x16384 fp32 (temp+power), 100 iterations/step", 100),
+    "heat3d": ("C3 3D 7-point heat stencil 1024^3 fp32, 50 iterations/step", 50),
+    "jacobi2d": ("C1 2D 5-point Jacobi 512x512 fp32, 10 iterations/step", 10),
+    "nbody": ("C5 all-pairs N-body 2^20 bodies fp32, 10 steps/step", 10),
+}
+
+
+def env_int(name, default):
+    try:
+        return int(os.environ.get(name, default))
+    except ValueError:
+        return default
+
+
+def load_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return None
+
+
+def ncu_traffic(kernel):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch from a committed ncu capture."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        v = d.get(kernel)
+        return None if v is None else v.get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled DURING the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpus):
+        self.gpus = set(gpus)
+        self.lines = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL,
+                                         text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                idx = int(f[0])
+            except ValueError:
+                continue
+            if idx not in self.gpus:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+                power.append(float(f[3]))
+            except ValueError:
+                pass
+            for n, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm),
+                "power_w_max": max(power) if power else None}
+
+
+# ------------------------------------------------------------------ workloads
+class Workload:
+    """Inputs, setup and per-step loop of one config, driven through the C-ABI."""
+
+    def __init__(self, name, iters):
+        self.name, self.iters = name, iters
+        import synth
+        from paper_conf_icppw_matzdf20_b200 import kernels as K
+        self.K = K
+        if name == "hotspot2d":
+            self.shape = (16384, 16384)
+            self.host = synth.hotspot_grids(*self.shape)
+            self.units_per_iter = self.shape[0] * self.shape[1]
+            self.bytes_per_unit = 12          # temp read + power read + temp write
+            self.unit, self.metric = "GLUP/s", "hotspot2d_glups"
+        elif name == "heat3d":
+            self.shape = (1024, 1024, 1024)
+            self.host = (synth.heat_grid(*self.shape),)
+            self.units_per_iter = int(np.prod(self.shape))
+            self.bytes_per_unit = 8
+            self.unit, self.metric = "GLUP/s", "heat3d_glups"
+        elif name == "jacobi2d":
+            self.shape = (512, 512)
+            self.host = (synth.jacobi_grid(*self.shape),)
+            self.units_per_iter = (self.shape[0] - 2) * (self.shape[1] - 2)
+            self.bytes_per_unit = 8
+            self.unit, self.metric = "GLUP/s", "jacobi2d_glups"
+        elif name == "nbody":
+            n = 1 << 20
+            self.shape = (n,)
+            self.host = synth.nbody_bodies(n)
+            self.units_per_iter = n * n
+            self.bytes_per_unit = 0
+            self.unit, self.metric = "Ginteractions/s", "nbody_ginteractions"
+        else:
+            raise SystemExit(f"unknown workload {name}")
+
+    def setup(self, ctx):
+        K = self.K
+        if self.name == "hotspot2d":
+            self.pr = K.hotspot2d_setup(ctx, *self.host)
+            self.upload_bufs = [(self.pr.tb[0], self.host[0]), (self.pr.tb[2], self.host[1])]
+        elif self.name == "heat3d":
+            self.pr = K.heat3d_setup(ctx, self.host[0])
+            self.upload_bufs = [(self.pr.ub[0], self.host[0])]
+        elif self.name == "jacobi2d":
+            self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0)
+            self.upload_bufs = [(b, self.host[0]) for b in self.pr.bufs]
+        elif self.name == "nbody":
+            self.pr = K.nbody_setup(ctx, *self.host)
+            self.upload_bufs = [(self.pr.nb[0], self.host[0]), (self.pr.nb[2], self.host[1])]
+        self.t = 0
+
+    def step(self):
+        K, pr = self.K, self.pr
+        if self.name == "hotspot2d":
+            out = K.hotspot2d_iterate(pr, self.iters, self.t)
+        elif self.name == "heat3d":
+            out = K.heat3d_iterate(pr, self.iters, self.t)
+        elif self.name == "jacobi2d":
+            h, w = self.shape
+            grid, blk, sc = K.jacobi2d_launch(h, w)
+            b0, b1 = pr.bufs
+            for t in range(self.t, self.t + self.iters):
+                a, b = (b0, b1) if t % 2 == 0 else (b1, b0)
+                pr.launch(grid, blk, [a, b, h, w], sc)
+            out = b1 if (self.t + self.iters) % 2 == 1 else b0
+        else:
+            out, _ = K.nbody_iterate(pr, self.iters, self.t)
+        self.t += self.iters
+        return out
+
+    def out_shape(self):
+        return (self.shape[0], 4) if self.name == "nbody" else self.shape
+
+    def stale_min(self, P):
+        from_cf = {
+            "hotspot2d": lambda: 2 * self.shape[1] * 4 * (P - 1),
+            "heat3d": lambda: 2 * self.shape[1] * self.shape[2] * 4 * (P - 1),
+            "jacobi2d": lambda: 2 * (self.shape[1] - 2) * 4 * (P - 1),
+            "nbody": lambda: self.shape[0] * 16 * (P - 1),
+        }
+        return from_cf[self.name]() * self.iters
+
+
+def cpu_oracle_rate(w: Workload, budget_s=10.0, max_iters=50):
+    """Time the oracle as it stands on a bounded sample of the same workload."""
+    import ctypes
+    from oracle import kernels as ok
+    L = ok.lib()
+    D = ctypes.POINTER(ctypes.c_double)
+    t0 = time.perf_counter()
+    if w.name in ("hotspot2d", "jacobi2d", "heat3d"):
+        if w.name == "hotspot2d":
+            rows = min(4096, w.shape[0])
+            a = np.ascontiguousarray(w.host[0][:rows], dtype=np.float64)
+            p = np.ascontiguousarray(w.host[1][:rows], dtype=np.float64)
+            b = np.empty_like(a)
+            cells = a.size
+            sample = f"{rows}x{w.shape[1]} band of the 16384^2 grid"
+
+            def one(src, dst):
+                L.oracle_hotspot2d_sweep(src.ctypes.data_as(D), p.ctypes.data_as(D), dst.ctypes.data_as(D),
+                                         ctypes.c_int64(rows), ctypes.c_int64(w.shape[1]),
+                                         ctypes.c_double(ok.HOTSPOT_CAP), ctypes.c_double(ok.HOTSPOT_RX1),
+                                         ctypes.c_double(ok.HOTSPOT_RY1), ctypes.c_double(ok.HOTSPOT_RZ1),
+                                         ctypes.c_double(ok.HOTSPOT_AMB))
+        elif w.name == "heat3d":
+            planes = min(128, w.shape[0])
+            a = np.ascontiguousarray(w.host[0][:planes], dtype=np.float64)
+            b = np.empty_like(a)
+            cells = a.size
+            sample = f"{planes} planes of the 1024^3 grid"
+
+            def one(src, dst):
+                L.oracle_heat3d_sweep(src.ctypes.data_as(D), dst.ctypes.data_as(D), ctypes.c_int64(planes),
+                                      ctypes.c_int64(w.shape[1]), ctypes.c_int64(w.shape[2]),
+                                      ctypes.c_double(ok.HEAT_ALPHA))
+        else:
+            a = np.ascontiguousarray(w.host[0], dtype=np.float64)
+            b = a.copy()
+            cells = (w.shape[0] - 2) * (w.shape[1] - 2)
+            sample = "full 512^2 grid"
+
+            def one(src, dst):
+                L.oracle_jacobi2d_sweep(src.ctypes.data_as(D), dst.ctypes.data_as(D), ctypes.c_int64(w.shape[0]),
+                                        ctypes.c_int64(w.shape[1]))
+        for fn in ("oracle_hotspot2d_sweep", "oracle_heat3d_sweep", "oracle_jacobi2d_sweep"):
+            getattr(L, fn).restype = None
+        its, el = 0, 0.0
+        ts = time.perf_counter()
+        while its < max_iters and el < budget_s:
+            if its % 2 == 0:
+                one(a, b)
+            else:
+                one(b, a)
+            its += 1
+            el = time.perf_counter() - ts
+        rate = cells * its / el / 1e9
+        sample += f", {its} iterations"
+    else:
+        nt = 256
+        pos = np.ascontiguousarray(w.host[0], dtype=np.float64)
+        tg = np.arange(0, w.shape[0], w.shape[0] // nt, dtype=np.int64)[:nt]
+        ts = time.perf_counter()
+        ok.nbody_accel(pos, tg)
+        el = time.perf_counter() - ts
+        rate = nt * w.shape[0] / el / 1e9
+        sample = f"{nt} sampled targets x {w.shape[0]} sources, 1 step (fp64)"
+    return {"value": rate, "unit": w.unit, "cores": ok.num_threads(), "kind": "oracle", "sample": sample,
+            "seconds": round(time.perf_counter() - t0, 2)}
+
+
+def run_reference(args, w: Workload, rank):
+    """--impl reference: the oracle as it stands, on the host cores, same metric."""
+    if rank != 0:
+        return None
+    # each step is a bounded sample; warmup steps are run untimed
+    for _ in range(args.warmup):
+        cpu_oracle_rate(w, budget_s=1.0, max_iters=1)
+    vals = [cpu_oracle_rate(w, budget_s=5.0, max_iters=4) for _ in range(args.steps)]
+    v = statistics.median(x["value"] for x in vals)
+    line = {"impl": "reference", "metric": w.metric, "value": v, "unit": w.unit, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": WORKLOADS[w.name][0]},
+            "cpu_baseline": {"value": v, "unit": w.unit, "cores": vals[0]["cores"], "kind": "oracle",
+                             "sample": vals[0]["sample"] + " per step"},
+            "e2e": {"value": v, "unit": w.unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "vs_baseline": None}
+    return line
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="hotspot2d", choices=sorted(WORKLOADS))
+    ap.add_argument("--parts", type=int, default=0, help="partitions (default: one per GPU)")
+    ap.add_argument("--iters", type=int, default=0, help="iterations per step (default: the config's)")
+    ap.add_argument("--impl", default="pk", choices=["pk", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "pk":
+        print("warning: fewer than 3 warm-up steps", file=sys.stderr)
+
+    rank, world = env_int("RANK", 0), env_int("WORLD_SIZE", 1)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo")
+    w = Workload(args.workload, args.iters or WORKLOADS[args.workload][1])
+
+    if args.impl == "reference":
+        line = run_reference(args, w, rank)
+        if dist:
+            dist.barrier()
+        if rank == 0:
+            print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    from paper_conf_icppw_matzdf20_b200 import abi
+
+    ngpu = max(1, args.gpus)
+    P = args.parts or ngpu
+    elapsed_ms = 0.0
+    result = {}
+    if rank == 0:
+        ndev = torch.cuda.device_count()
+        if ndev < ngpu:
+            raise SystemExit(f"--gpus {ngpu} but only {ndev} visible")
+        part_device = [p % ngpu for p in range(P)]
+        ctx = abi.pk_init(P, part_device=part_device)
+        w.setup(ctx)
+        for _ in range(args.warmup):
+            w.step()
+        abi.pk_synchronize(ctx)
+        abi.pk_reset_stats(ctx)
+        abi.pk_set_mode(ctx, abi.PK_MODE_TIME_KERNELS)
+    if dist:
+        dist.barrier()
+    sampler = ClockSampler(range(ngpu)) if rank == 0 else None
+    if rank == 0:
+        sampler.start()
+        time.sleep(0.3)
+        abi.pk_synchronize(ctx)
+        abi.pk_timer_begin(ctx)
+        for _ in range(args.steps):
+            w.step()
+        elapsed_ms = abi.pk_timer_end(ctx)
+        clocks = sampler.stop()
+        st = abi.pk_get_stats(ctx)
+        abi.pk_set_mode(ctx, 0)
+    if dist:
+        import torch as _t
+        tt = _t.tensor([elapsed_ms], dtype=_t.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(tt.item())
+    if rank != 0:
+        if dist:
+            dist.barrier()
+        return
+
+    units = w.units_per_iter * w.iters * args.steps
+    value = units / (elapsed_ms / 1e3) / 1e9
+    peaks = load_peaks()
+    kname = w.name
+    avg_kernel_ms = st["kernel_ms"] / max(1, st["timed_kernels"])
+    per_launch_units = w.units_per_iter / P
+    if w.name == "nbody":
+        # FP32-ALU bound: 12 FP32-pipe instructions per interaction on 128 lanes/SM
+        sm_mhz = clocks.get("sm_mhz") or (peaks or {}).get("sm_max_mhz", 1965.0)
+        peak = 148 * 128 / 12 * (sm_mhz * 1e6) / 1e9
+        achieved = per_launch_units / (avg_kernel_ms / 1e3) / 1e9
+        roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Ginteractions/s",
+                    "frac": achieved / peak, "traffic": None,
+                    "peak_source": f"148 SMs x 128 FP32 lanes / 12 ops per interaction at {sm_mhz:.0f} MHz"}
+    else:
+        bytes_per_launch = w.bytes_per_unit * per_launch_units
+        achieved = bytes_per_launch / (avg_kernel_ms / 1e3) / 1e9
+        peak = (peaks or {}).get("hbm_gbs", 6650.0)
+        roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                    "frac": achieved / peak, "traffic": ncu_traffic(kname),
+                    "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if peaks else "fallback 6.65 TB/s"}
+    result.update({
+        "metric": w.metric, "value": value, "unit": w.unit, "n_gpus": ngpu, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": WORKLOADS[w.name][0], "iterations_per_step": w.iters, "partitions": P,
+                   "partition_devices": sorted(set(p % ngpu for p in range(P))),
+                   "l2": "inputs larger than the 126 MB L2 (no flush)" if w.name != "jacobi2d"
+                   else "1 MB working set stays in L2 (latency-bound C1)",
+                   "process_model": "one host process drives all partitions (rank 0)"},
+        "gpu_launches": int(st["kernel_launches"]),
+        "clocks": clocks,
+        "roofline": roofline,
+        "kernel_ms_avg": avg_kernel_ms,
+        "transfers": {"stale_bytes": int(st["stale_bytes"]), "moved_bytes": int(st["moved_bytes"]),
+                      "analytic_min_bytes": w.stale_min(P) * args.steps, "copies": int(st["copies"])},
+        "host_us_per_launch": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"]
+                               + st["host_ns_issue"] + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
+    })
+
+    # ---- e2e: same metric with the H2D upload and D2H gather inside every step ----
+    if not args.no_e2e:
+        pinned = [(b, torch.from_numpy(h).pin_memory()) for b, h in w.upload_bufs]
+        out_host = torch.empty(w.out_shape(), dtype=torch.float32).pin_memory()
+        abi.pk_synchronize(ctx)
+        t0 = time.perf_counter()
+        h2d = d2h = 0
+        for _ in range(args.e2e_steps):
+            for b, hbuf in pinned:
+                abi.pk_copy_from_host(ctx, b, hbuf)
+                h2d += hbuf.numel() * hbuf.element_size()
+            w.t = 0
+            out = w.step()
+            abi.pk_sync_to_host(ctx, out, out_host)
+            d2h += out_host.numel() * out_host.element_size()
+        el = time.perf_counter() - t0
+        result["e2e"] = {"value": w.units_per_iter * w.iters * args.e2e_steps / el / 1e9, "unit": w.unit,
+                         "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
+                         "steps": args.e2e_steps, "timing": "wall clock around pk_copy_from_host + launches + "
+                                                           "pk_sync_to_host (pinned host buffers)"}
+    abi.pk_finalize(ctx)
+    if not args.no_cpu_baseline and ngpu == 1:
+        result["cpu_baseline"] = cpu_oracle_rate(w)
+    if dist:
+        dist.barrier()
+    print(json.dumps(result), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,275 @@
+/*
+ * pk_api.h -- C-ABI of the B200-native partitioned-kernel runtime ("pk").
+ *
+ * Hot path of Matz, Doerfert, Fröning, "Automated Partitioning of Data-Parallel
+ * Kernels using Polyhedral Compilation" (ICPP Workshops 2020).  Citations
+ * "P:Lnnn" are lines of /root/reference/PAPER.md (the paper's text) plus the
+ * section / equation / figure they fall in.
+ *
+ * One regular, affine-access CUDA kernel has its grid split along thread-block
+ * boundaries into P partitions (§5 task (1), §7 Eq. 8-10).
+ * Before each launch the read/write regions of every partition are computed
+ * from declared affine access descriptors (replacing the paper's polyhedral
+ * analysis, §4, and its generated enumerators, §6), a
+ * per-buffer validity map finds the stale ranges (§8.1,
+ * P:L914-936 §8.3) and only those move between device instances before the
+ * sub-grids launch (Fig. 4).
+ *
+ * Conventions
+ *  - Every entry point returns an int status: PK_OK (0) or a negative PK_ERR_*.
+ *    No C++ exception crosses the ABI.  A thread-local message describing the
+ *    last failure is returned by pk_last_error().
+ *  - Plain pointers and sizes only; no torch or CUDA types in the signatures.
+ *    "device pointer" = a CUDA global-memory address valid on the partition's
+ *    device; "host pointer" = ordinary process memory (pinned or pageable).
+ *  - A context is used from one host thread at a time, like the paper's single
+ *    rewritten host program (§8.4).
+ *  - Integer parameters of descriptors and enumerators are int64 arrays, as in
+ *    the paper's enumerator interface (§6.2).
+ *  - Grid/block triples are ordered (x, y, z) like CUDA's dim3; partition
+ *    6-tuples are ordered (zmin, zmax, ymin, ymax, xmin, xmax) like the paper's
+ *    (§7, §6.2), half-open, in thread blocks.
+ */
+#ifndef PK_API_H
+#define PK_API_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ------------------------------------------------------------------ status */
+enum {
+    PK_OK = 0,
+    PK_ERR_INVALID = -1,        /* bad argument / handle / descriptor */
+    PK_ERR_CUDA = -2,           /* a CUDA runtime call failed (message has the cudaError name) */
+    PK_ERR_NCCL = -3,           /* reserved: NCCL transport */
+    PK_ERR_OOM = -4,            /* device or host allocation failed */
+    PK_ERR_OUT_OF_BOUNDS = -5,  /* an unclamped access leaves [0, shape) */
+    PK_ERR_WRITE_OVERLAP = -6,  /* two partitions write the same byte: WAW, §4.1 */
+    PK_ERR_OVERFLOW = -7,       /* int64 overflow in region arithmetic (P:L405-407 ignores it; we check) */
+    PK_ERR_STATE = -8           /* call not valid in the context's current state/mode */
+};
+
+/* ------------------------------------------------------------------ handles */
+typedef struct pk_ctx_s* pk_ctx;
+typedef int64_t pk_buf;     /* virtual buffer id (§8.1) */
+typedef int64_t pk_kernel;  /* kernel model record id (§4.1) */
+
+#define PK_MAX_PARTS 64     /* validity masks are 64-bit */
+#define PK_MAX_DIMS 4       /* array dimensions per descriptor */
+#define PK_MAX_SCALARS 8    /* int64 scalar arguments visible to descriptors */
+#define PK_MAX_ARGS 16      /* kernel arguments */
+
+/* ---------------------------------------------------------------- init */
+enum {
+    PK_INIT_HOST_ONLY = 1u << 0  /* no CUDA call at all: partitioning, regions, tracker and
+                                    transfer planning run, nothing is allocated, copied or
+                                    launched.  For host-side tests and planning. */
+};
+
+typedef struct {
+    int32_t nparts;              /* P, 1..PK_MAX_PARTS: partitions = virtual devices (§8.3:
+                                    "each partition corresponds to exactly one GPU", P:L919-920;
+                                    here several partitions may share one physical GPU) */
+    int32_t my_rank;             /* SPMD process rank (0 for the single-process model) */
+    int32_t world_size;          /* number of processes (1 = one host process drives every GPU) */
+    uint32_t flags;              /* PK_INIT_* */
+    const int32_t* part_device;  /* [nparts] CUDA ordinal of each partition's device on its rank;
+                                    NULL = partition p on device p % cudaGetDeviceCount() */
+    const int32_t* part_rank;    /* [nparts] owning rank; NULL = all partitions on rank 0 */
+} pk_init_params;
+
+/* Create a context: per-partition streams and events, peer access between every
+ * pair of distinct devices (P:L927-929 copies "from its most recently written to
+ * GPU").  Ownership: the context owns its streams/events; *out is released by
+ * pk_finalize.  Errors: PK_ERR_INVALID (bad params), PK_ERR_CUDA. */
+int pk_init(const pk_init_params* params, pk_ctx* out);
+int pk_finalize(pk_ctx ctx);
+
+/* ---------------------------------------------------------------- buffers */
+/* Virtual buffer = one full-size device instance per partition + a tracker
+ * (§8.1; full-size instances keep the kernels' global indices, reading
+ * Q13).  Row-major array of `ndim` (1..4) dims `shape[0..ndim)` (slowest first) of
+ * `elem_bytes`-byte elements.
+ *   dev_ptrs  == NULL: the library cudaMallocs and owns every instance.
+ *   dev_ptrs  != NULL: [nparts] caller-owned device pointers (e.g. torch tensors),
+ *                      16-byte aligned, which must outlive the registration.
+ *   host_init == NULL: contents undefined -> valid on every partition (reading Q3).
+ *   host_init != NULL: H2D 1:n linear distribution of the host array (P:L881-895
+ *                      §8.2, reading Q2); blocking with respect to host memory.
+ * Errors: PK_ERR_INVALID, PK_ERR_OOM, PK_ERR_CUDA. */
+int pk_register_buffer(pk_ctx ctx, int ndim, const int64_t* shape, int elem_bytes,
+                       void* const* dev_ptrs, const void* host_init, pk_buf* out);
+/* cudaMemcpy(HostToDevice) replacement: 1:n linear distribution.
+ * `bytes` must equal the buffer size.  Returns after the copies completed. */
+int pk_copy_from_host(pk_ctx ctx, pk_buf buf, const void* host, size_t bytes);
+/* cudaMemcpy(DeviceToHost) replacement: n:1 gather, one copy per tracker segment
+ * from a partition holding it (§8.2).  Blocking. */
+int pk_sync_to_host(pk_ctx ctx, pk_buf buf, void* host, size_t bytes);
+/* cudaFree replacement.  Library-owned instances are freed after pending work. */
+int pk_unregister_buffer(pk_ctx ctx, pk_buf buf);
+/* Device pointer of partition `part`'s instance (tests / caller-side kernels). */
+int pk_buffer_instance(pk_ctx ctx, pk_buf buf, int part, void** dev_ptr);
+
+/* ---------------------------------------------------------------- descriptors */
+/* Affine expression in the kernel's int64 scalar arguments and the launch's
+ * blockDim (the paper's blockOff = blockIdx * blockDim trick, §4.1
+ * Eq. 5-7, keeps descriptors affine in blockIdx):
+ *   value = c0 + sum_s c_scalar[s] * scalars[s] + sum_w c_blockdim[w] * blockDim[w] */
+typedef struct {
+    int64_t c0;
+    int64_t c_scalar[PK_MAX_SCALARS];
+    int64_t c_blockdim[3];
+} pk_expr;
+
+enum { PK_DIM_CLAMP = 1u << 0, PK_DIM_GUARD = 1u << 1 };
+
+/* One array dimension of one access "tap".  For a partition whose block range
+ * along grid dimension `grid_dim` (0=x 1=y 2=z) is [m, M):
+ *   Pos = U_{b in [m,M)} [b*scale, b*scale + extent)      (grid_dim >= 0)
+ *   Pos = [0, extent)                                      (grid_dim == -1: all blocks
+ *                                                           touch the same positions)
+ *   if PK_DIM_GUARD: Pos = Pos n [guard_lo, guard_hi)      (the kernel's bounds test)
+ *   Idx = { p + offset : p in Pos }, then
+ *   if PK_DIM_CLAMP: each index clamped to [0, shape-1]    (replicate borders)
+ *   else: every index must lie in [0, shape) or the call fails PK_ERR_OUT_OF_BOUNDS.
+ * This is the paper's block-granular access map (threadId projected out under
+ * 0 <= threadId < blockDim, §4.1) restricted to separable boxes. */
+typedef struct {
+    int32_t grid_dim;
+    uint32_t flags;              /* PK_DIM_* */
+    pk_expr scale, extent, guard_lo, guard_hi, offset;
+} pk_dim_map;
+
+/* One tap = the product of its per-dimension index sets (exact because a grid
+ * dimension may drive at most one array dimension of a tap; otherwise
+ * PK_ERR_INVALID).  Several taps of one (arg, mode) are unioned exactly, which is
+ * the per-convex-piece enumeration of P:L773-775 §6.1 (no union over-approximation). */
+typedef struct {
+    int32_t ndim;                /* must equal the bound buffer's ndim */
+    int32_t reserved;
+    pk_dim_map dim[PK_MAX_DIMS]; /* dim[0] = slowest (row-major) */
+} pk_affine_access;
+
+enum { PK_READ = 1, PK_WRITE = 2, PK_MAY_WRITE = 3 };   /* PK_MAY_WRITE = read + write (reading Q6) */
+
+/* ---------------------------------------------------------------- kernels */
+enum { PK_ARG_BUFFER = 1, PK_ARG_SCALAR = 2 };
+
+/* Passed BY VALUE as the kernel's last argument (§7): the kernel
+ * computes blockIdx' = min + blockIdx (Eq. 8) and must read the full grid from
+ * `grid` instead of gridDim (Eq. 9, reading Q10).  Index 0=x, 1=y, 2=z. */
+typedef struct {
+    int32_t min[3];
+    int32_t max[3];
+    int32_t grid[3];
+} pk_partition;
+
+/* Kernel model record (name, suggested partitioning strategy,
+ * per-argument maps).  `fn` is a __global__ function of this library's CUDA
+ * runtime (see pk_builtin_fn) launched with cudaLaunchKernel; arguments are the
+ * kernel's own followed by a pk_partition.  arg_kind[nargs] = PK_ARG_*.
+ * partition_dim: 0/1/2 forces x/y/z, -1 = slowest grid dim > 1 (reading Q1). */
+int pk_register_kernel(pk_ctx ctx, const char* name, const void* fn, int nargs,
+                       const int32_t* arg_kind, int32_t partition_dim, pk_kernel* out);
+/* Add one access tap for argument `arg_index` with `mode` (PK_READ / PK_WRITE /
+ * PK_MAY_WRITE).  Taps accumulate (union).  Write taps must be exact and
+ * injective; read taps may over-approximate. */
+int pk_declare_affine_access(pk_ctx ctx, pk_kernel k, int arg_index, int mode,
+                             const pk_affine_access* tap);
+/* Register one of the library's sm_100a kernels ("jacobi2d", "hotspot2d",
+ * "heat3d", "nbody", "sgemm_tf32x3") with its descriptors already declared. */
+int pk_builtin_kernel(pk_ctx ctx, const char* name, pk_kernel* out);
+/* __global__ entry of a builtin kernel, for pk_register_kernel + user-declared
+ * descriptors.  NULL if unknown. */
+const void* pk_builtin_fn(const char* name);
+
+/* The kernel-launch replacement of Fig. 4:
+ *   (1) partition the grid,  (2) synchronise every read buffer: stale
+ *   ranges of each partition's read set are copied from a holder,
+ *   (3) launch every partition with grid' = max - min (Eq. 10) on its device,
+ *   (4) update the trackers with the write sets, on the host while
+ *   the kernels run.
+ * grid/block: the ORIGINAL single-device launch (x, y, z).  args[nargs]: for a
+ * buffer argument a pointer to its pk_buf, for a scalar a pointer to its value
+ * (copied at launch).  scalars[nscalars]: int64 scalar values the descriptors
+ * use.  Asynchronous like <<<>>>: faults surface at pk_synchronize.
+ * Errors: PK_ERR_INVALID, PK_ERR_OUT_OF_BOUNDS, PK_ERR_WRITE_OVERLAP (nothing is
+ * launched), PK_ERR_OVERFLOW, PK_ERR_CUDA. */
+int pk_launch_partitioned(pk_ctx ctx, pk_kernel k, const int32_t grid[3],
+                          const int32_t block[3], size_t smem_bytes,
+                          const void* const* args, const int64_t* scalars, int nscalars);
+/* cudaDeviceSynchronize replacement: all partitions' streams (§8.4). */
+int pk_synchronize(pk_ctx ctx);
+/* Device-side timer over everything the context enqueues between the two calls:
+ * begin records an event on partition 0's stream and makes every other stream
+ * wait for it; end makes partition 0's stream wait for every stream's tail and
+ * records the stop event there, then blocks and returns the elapsed ms (CUDA
+ * events, both on partition 0's device).  Not nestable.  PK_ERR_STATE in a
+ * host-only context or when end is called without begin. */
+int pk_timer_begin(pk_ctx ctx);
+int pk_timer_end(pk_ctx ctx, double* elapsed_ms);
+
+/* ---------------------------------------------------------------- introspection */
+/* Grid partition p of the kernel's launch (a1), as (zmin,zmax,ymin,ymax,xmin,xmax). */
+int pk_partition_grid(pk_ctx ctx, pk_kernel k, const int32_t grid[3], int part,
+                      int64_t part_out[6]);
+typedef void (*pk_range_cb)(void* user, uint64_t begin_byte, uint64_t end_byte);
+/* Enumerator of §6.2: canonical (sorted, disjoint, coalesced) byte
+ * ranges of the image of (arg, mode) over the 6-tuple block box `part`, for
+ * buffer `buf`'s shape; one callback per range, no allocation visible to the
+ * caller.  mode PK_READ includes PK_MAY_WRITE taps, PK_WRITE includes them too. */
+int pk_enumerate(pk_ctx ctx, pk_kernel k, int arg_index, int mode, pk_buf buf,
+                 const int64_t part[6], const int32_t block[3],
+                 const int64_t* scalars, int nscalars, pk_range_cb cb, void* user);
+typedef void (*pk_segment_cb)(void* user, uint64_t begin_byte, uint64_t end_byte,
+                              uint64_t valid_mask);
+/* Tracker state: canonical segments covering the buffer, each with the mask of
+ * partitions holding its latest value (paper: owner). */
+int pk_tracker_dump(pk_ctx ctx, pk_buf buf, pk_segment_cb cb, void* user);
+typedef void (*pk_copy_cb)(void* user, pk_buf buf, int src_part, int dst_part,
+                           uint64_t begin_byte, uint64_t end_byte);
+/* Copies planned by the most recent pk_launch_partitioned (coalesced, in issue order). */
+int pk_last_plan(pk_ctx ctx, pk_copy_cb cb, void* user);
+
+typedef struct {
+    uint64_t launches;           /* pk_launch_partitioned calls */
+    uint64_t kernel_launches;    /* partition kernels actually launched */
+    uint64_t copies;             /* device-to-device copy operations issued */
+    uint64_t stale_bytes;        /* bytes of read sets not valid on the reader */
+    uint64_t moved_bytes;        /* bytes actually copied between instances */
+    uint64_t h2d_bytes, d2h_bytes;
+    uint64_t pair_bytes[16][16]; /* [src][dst] moved bytes, partitions < 16 */
+    uint64_t host_ns_partition;  /* host time per phase (a1, a2, a3, issue, a7) */
+    uint64_t host_ns_regions;
+    uint64_t host_ns_plan;
+    uint64_t host_ns_issue;
+    uint64_t host_ns_update;
+    double kernel_ms;            /* sum over partition kernels (PK_MODE_TIME_KERNELS) */
+    double kernel_ms_max_launch; /* per launch: max over partitions, summed */
+    uint64_t timed_kernels;      /* kernels included in kernel_ms */
+} pk_stats;
+int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
+int pk_reset_stats(pk_ctx ctx);
+
+/* ---------------------------------------------------------------- modes */
+enum {
+    PK_MODE_SINGLE_OWNER = 1u << 0,  /* paper tracker: one owner, no shared copies */
+    PK_MODE_NO_TRANSFERS = 1u << 1,  /* beta of §9.2: resolve + track, do not copy */
+    PK_MODE_NO_TRACKING = 1u << 2,   /* gamma of §9.2: no resolution, no tracker, no copies */
+    PK_MODE_GLOBAL_BARRIER = 1u << 3,/* literal all_devs_synchronize() between sync and launch (Fig. 4 l. 8) */
+    PK_MODE_TIME_KERNELS = 1u << 4   /* CUDA events around every partition kernel -> pk_stats.kernel_ms */
+};
+int pk_set_mode(pk_ctx ctx, uint32_t flags);
+uint32_t pk_get_mode(pk_ctx ctx);
+
+const char* pk_last_error(void);
+const char* pk_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PK_API_H */

@@ -104,14 +104,15 @@ def heat3d(box, block, d, h, w, zc, vec=4):
 
 
 # ---------------------------------------------------------------------------
-# C5 nbody(pos_in, vel, pos_out; N): block (bdx); thread i = bx*bdx + tx,
-#   guard i < N.  Reads every body of pos_in (all-pairs), reads and writes
-#   vel[i] (in place), writes pos_out[i].  Elements are float4 bodies.
+# C5 nbody(pos_in, vel, pos_out; N): block (bdx); thread tx of block bx owns
+#   the `per_thread` bodies i = bx*per_thread*bdx + tx + u*bdx, guard i < N.
+#   Reads every body of pos_in (all-pairs), reads and writes vel[i] (in place),
+#   writes pos_out[i].  Elements are float4 bodies.
 # ---------------------------------------------------------------------------
-def nbody(box, block, n):
+def nbody(box, block, n, per_thread=2):
     bdx = block[0]
     _, _, bxs = _block_ranges(box)
-    i = (bxs[:, None] * bdx + np.arange(bdx)[None, :]).ravel()
+    i = (bxs[:, None] * (per_thread * bdx) + np.arange(per_thread * bdx)[None, :]).ravel()
     i = i[i < n]
     allpos = np.arange(n, dtype=np.int64) if i.size else np.zeros(0, dtype=np.int64)
     return {(0, READ): allpos, (1, READ): _uniq([i]), (1, WRITE): _uniq([i]),

@@ -1,0 +1,340 @@
+"""Thin ctypes binding of include/pk_api.h -- same names, argument marshalling only.
+
+Every step of the hot path runs inside libpk.so (host C++ + sm_100a kernels).
+If the library is missing this module raises at import of ``lib()``: there is no
+Python or CPU fallback.  Build it with ``python -m paper_conf_icppw_matzdf20_b200.build``.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libpk.so")
+
+PK_OK = 0
+PK_ERR = {-1: "PK_ERR_INVALID", -2: "PK_ERR_CUDA", -3: "PK_ERR_NCCL", -4: "PK_ERR_OOM",
+          -5: "PK_ERR_OUT_OF_BOUNDS", -6: "PK_ERR_WRITE_OVERLAP", -7: "PK_ERR_OVERFLOW",
+          -8: "PK_ERR_STATE"}
+PK_INIT_HOST_ONLY = 1
+PK_MAX_PARTS, PK_MAX_DIMS, PK_MAX_SCALARS, PK_MAX_ARGS = 64, 4, 8, 16
+PK_DIM_CLAMP, PK_DIM_GUARD = 1, 2
+PK_READ, PK_WRITE, PK_MAY_WRITE = 1, 2, 3
+PK_ARG_BUFFER, PK_ARG_SCALAR = 1, 2
+PK_MODE_SINGLE_OWNER = 1 << 0
+PK_MODE_NO_TRANSFERS = 1 << 1
+PK_MODE_NO_TRACKING = 1 << 2
+PK_MODE_GLOBAL_BARRIER = 1 << 3
+PK_MODE_TIME_KERNELS = 1 << 4
+
+
+class PkError(RuntimeError):
+    def __init__(self, code, where, msg):
+        self.code = code
+        self.name = PK_ERR.get(code, str(code))
+        super().__init__(f"{where}: {self.name}: {msg}")
+
+
+# ------------------------------------------------------------------ structs
+class pk_init_params(C.Structure):
+    _fields_ = [("nparts", C.c_int32), ("my_rank", C.c_int32), ("world_size", C.c_int32),
+                ("flags", C.c_uint32), ("part_device", C.POINTER(C.c_int32)),
+                ("part_rank", C.POINTER(C.c_int32))]
+
+
+class pk_expr(C.Structure):
+    _fields_ = [("c0", C.c_int64), ("c_scalar", C.c_int64 * PK_MAX_SCALARS),
+                ("c_blockdim", C.c_int64 * 3)]
+
+
+class pk_dim_map(C.Structure):
+    _fields_ = [("grid_dim", C.c_int32), ("flags", C.c_uint32), ("scale", pk_expr),
+                ("extent", pk_expr), ("guard_lo", pk_expr), ("guard_hi", pk_expr),
+                ("offset", pk_expr)]
+
+
+class pk_affine_access(C.Structure):
+    _fields_ = [("ndim", C.c_int32), ("reserved", C.c_int32), ("dim", pk_dim_map * PK_MAX_DIMS)]
+
+
+class pk_partition(C.Structure):
+    _fields_ = [("min", C.c_int32 * 3), ("max", C.c_int32 * 3), ("grid", C.c_int32 * 3)]
+
+
+class pk_stats(C.Structure):
+    _fields_ = [("launches", C.c_uint64), ("kernel_launches", C.c_uint64), ("copies", C.c_uint64),
+                ("stale_bytes", C.c_uint64), ("moved_bytes", C.c_uint64), ("h2d_bytes", C.c_uint64),
+                ("d2h_bytes", C.c_uint64), ("pair_bytes", (C.c_uint64 * 16) * 16),
+                ("host_ns_partition", C.c_uint64), ("host_ns_regions", C.c_uint64),
+                ("host_ns_plan", C.c_uint64), ("host_ns_issue", C.c_uint64),
+                ("host_ns_update", C.c_uint64), ("kernel_ms", C.c_double),
+                ("kernel_ms_max_launch", C.c_double), ("timed_kernels", C.c_uint64)]
+
+
+RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)
+SEGMENT_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64, C.c_uint64)
+COPY_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_int64, C.c_int, C.c_int, C.c_uint64, C.c_uint64)
+
+_lib = None
+_I64P = C.POINTER(C.c_int64)
+_I32P = C.POINTER(C.c_int32)
+
+
+def lib():
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} is missing: build the CUDA extension first "
+                           "(python -m paper_conf_icppw_matzdf20_b200.build); there is no fallback")
+    L = C.CDLL(LIB_PATH)
+    sig = {
+        "pk_init": [C.POINTER(pk_init_params), C.POINTER(C.c_void_p)],
+        "pk_finalize": [C.c_void_p],
+        "pk_register_buffer": [C.c_void_p, C.c_int, _I64P, C.c_int, C.POINTER(C.c_void_p), C.c_void_p, _I64P],
+        "pk_copy_from_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
+        "pk_sync_to_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
+        "pk_unregister_buffer": [C.c_void_p, C.c_int64],
+        "pk_buffer_instance": [C.c_void_p, C.c_int64, C.c_int, C.POINTER(C.c_void_p)],
+        "pk_register_kernel": [C.c_void_p, C.c_char_p, C.c_void_p, C.c_int, _I32P, C.c_int32, _I64P],
+        "pk_declare_affine_access": [C.c_void_p, C.c_int64, C.c_int, C.c_int, C.POINTER(pk_affine_access)],
+        "pk_builtin_kernel": [C.c_void_p, C.c_char_p, _I64P],
+        "pk_launch_partitioned": [C.c_void_p, C.c_int64, _I32P, _I32P, C.c_size_t,
+                                  C.POINTER(C.c_void_p), _I64P, C.c_int],
+        "pk_synchronize": [C.c_void_p],
+        "pk_timer_begin": [C.c_void_p],
+        "pk_timer_end": [C.c_void_p, C.POINTER(C.c_double)],
+        "pk_partition_grid": [C.c_void_p, C.c_int64, _I32P, C.c_int, _I64P],
+        "pk_enumerate": [C.c_void_p, C.c_int64, C.c_int, C.c_int, C.c_int64, _I64P, _I32P, _I64P,
+                         C.c_int, RANGE_CB, C.c_void_p],
+        "pk_tracker_dump": [C.c_void_p, C.c_int64, SEGMENT_CB, C.c_void_p],
+        "pk_last_plan": [C.c_void_p, COPY_CB, C.c_void_p],
+        "pk_get_stats": [C.c_void_p, C.POINTER(pk_stats)],
+        "pk_reset_stats": [C.c_void_p],
+        "pk_set_mode": [C.c_void_p, C.c_uint32],
+    }
+    for name, args in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = C.c_int
+    L.pk_builtin_fn.argtypes = [C.c_char_p]
+    L.pk_builtin_fn.restype = C.c_void_p
+    L.pk_get_mode.argtypes = [C.c_void_p]
+    L.pk_get_mode.restype = C.c_uint32
+    L.pk_last_error.restype = C.c_char_p
+    L.pk_version.restype = C.c_char_p
+    _lib = L
+    return L
+
+
+def _check(rc, where):
+    if rc != PK_OK:
+        raise PkError(rc, where, lib().pk_last_error().decode())
+
+
+def _addr(x):
+    """Host or device address of a numpy array, torch tensor or int."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if hasattr(x, "ctypes"):
+        return x.ctypes.data
+    raise TypeError(f"cannot take the address of {type(x)}")
+
+
+def _nbytes(x):
+    if hasattr(x, "nbytes"):
+        return int(x.nbytes)
+    return int(x.numel() * x.element_size())
+
+
+def _i32(v):
+    return (C.c_int32 * len(v))(*v)
+
+
+def _i64(v):
+    return (C.c_int64 * max(1, len(v)))(*v)
+
+
+# ------------------------------------------------------------------ same names as the C-ABI
+def pk_version() -> str:
+    return lib().pk_version().decode()
+
+
+def pk_last_error() -> str:
+    return lib().pk_last_error().decode()
+
+
+def pk_init(nparts, part_device=None, part_rank=None, my_rank=0, world_size=1, flags=0):
+    p = pk_init_params(nparts, my_rank, world_size, flags,
+                       _i32(part_device) if part_device is not None else None,
+                       _i32(part_rank) if part_rank is not None else None)
+    ctx = C.c_void_p()
+    _check(lib().pk_init(C.byref(p), C.byref(ctx)), "pk_init")
+    return ctx
+
+
+def pk_finalize(ctx):
+    _check(lib().pk_finalize(ctx), "pk_finalize")
+
+
+def pk_register_buffer(ctx, shape, elem_bytes, dev_ptrs=None, host_init=None, nparts=None):
+    shape = list(shape)
+    out = C.c_int64()
+    dp = None
+    if dev_ptrs is not None:
+        dp = (C.c_void_p * len(dev_ptrs))(*[_addr(d) for d in dev_ptrs])
+    _check(lib().pk_register_buffer(ctx, len(shape), _i64(shape), elem_bytes, dp, _addr(host_init),
+                                    C.byref(out)), "pk_register_buffer")
+    return out.value
+
+
+def pk_copy_from_host(ctx, buf, host, nbytes=None):
+    _check(lib().pk_copy_from_host(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
+           "pk_copy_from_host")
+
+
+def pk_sync_to_host(ctx, buf, host, nbytes=None):
+    _check(lib().pk_sync_to_host(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
+           "pk_sync_to_host")
+
+
+def pk_unregister_buffer(ctx, buf):
+    _check(lib().pk_unregister_buffer(ctx, buf), "pk_unregister_buffer")
+
+
+def pk_buffer_instance(ctx, buf, part) -> int:
+    p = C.c_void_p()
+    _check(lib().pk_buffer_instance(ctx, buf, part, C.byref(p)), "pk_buffer_instance")
+    return p.value or 0
+
+
+def pk_builtin_fn(name) -> int:
+    return lib().pk_builtin_fn(name.encode()) or 0
+
+
+def pk_register_kernel(ctx, name, fn, arg_kinds, partition_dim=-1) -> int:
+    out = C.c_int64()
+    _check(lib().pk_register_kernel(ctx, name.encode(), fn, len(arg_kinds), _i32(arg_kinds), partition_dim,
+                                    C.byref(out)), "pk_register_kernel")
+    return out.value
+
+
+def pk_declare_affine_access(ctx, kernel, arg_index, mode, tap: pk_affine_access):
+    _check(lib().pk_declare_affine_access(ctx, kernel, arg_index, mode, C.byref(tap)),
+           "pk_declare_affine_access")
+
+
+def pk_builtin_kernel(ctx, name) -> int:
+    out = C.c_int64()
+    _check(lib().pk_builtin_kernel(ctx, name.encode(), C.byref(out)), "pk_builtin_kernel")
+    return out.value
+
+
+def pk_launch_partitioned(ctx, kernel, grid, block, args, scalars=(), smem=0):
+    """args: one int per kernel argument -- the pk_buf id for a buffer, the
+    (int64) value for a scalar; None passes a NULL pointer."""
+    vals = [C.c_int64(a) if a is not None else None for a in args]
+    argv = (C.c_void_p * max(1, len(vals)))(*[C.addressof(v) if v is not None else None for v in vals])
+    sc = list(scalars)
+    _check(lib().pk_launch_partitioned(ctx, kernel, _i32(grid), _i32(block), smem, argv, _i64(sc), len(sc)),
+           "pk_launch_partitioned")
+
+
+def pk_synchronize(ctx):
+    _check(lib().pk_synchronize(ctx), "pk_synchronize")
+
+
+def pk_timer_begin(ctx):
+    _check(lib().pk_timer_begin(ctx), "pk_timer_begin")
+
+
+def pk_timer_end(ctx) -> float:
+    ms = C.c_double()
+    _check(lib().pk_timer_end(ctx, C.byref(ms)), "pk_timer_end")
+    return ms.value
+
+
+def pk_partition_grid(ctx, kernel, grid, part):
+    out = (C.c_int64 * 6)()
+    _check(lib().pk_partition_grid(ctx, kernel, _i32(grid), part, out), "pk_partition_grid")
+    return tuple(out)
+
+
+def pk_enumerate(ctx, kernel, arg_index, mode, buf, part6, block, scalars=()):
+    ranges = []
+    cb = RANGE_CB(lambda _u, b, e: ranges.append((b, e)))
+    sc = list(scalars)
+    _check(lib().pk_enumerate(ctx, kernel, arg_index, mode, buf, _i64(list(part6)), _i32(block), _i64(sc),
+                              len(sc), cb, None), "pk_enumerate")
+    return ranges
+
+
+def pk_tracker_dump(ctx, buf):
+    segs = []
+    cb = SEGMENT_CB(lambda _u, b, e, m: segs.append((b, e, m)))
+    _check(lib().pk_tracker_dump(ctx, buf, cb, None), "pk_tracker_dump")
+    return segs
+
+
+def pk_last_plan(ctx):
+    ops = []
+    cb = COPY_CB(lambda _u, buf, s, d, b, e: ops.append((buf, s, d, b, e)))
+    _check(lib().pk_last_plan(ctx, cb, None), "pk_last_plan")
+    return ops
+
+
+def pk_get_stats(ctx) -> dict:
+    s = pk_stats()
+    _check(lib().pk_get_stats(ctx, C.byref(s)), "pk_get_stats")
+    d = {name: getattr(s, name) for name, _ in pk_stats._fields_ if name != "pair_bytes"}
+    d["pair_bytes"] = [[s.pair_bytes[i][j] for j in range(16)] for i in range(16)]
+    return d
+
+
+def pk_reset_stats(ctx):
+    _check(lib().pk_reset_stats(ctx), "pk_reset_stats")
+
+
+def pk_set_mode(ctx, flags):
+    _check(lib().pk_set_mode(ctx, flags), "pk_set_mode")
+
+
+def pk_get_mode(ctx) -> int:
+    return int(lib().pk_get_mode(ctx))
+
+
+# ------------------------------------------------------------------ descriptor builders
+def expr(c0=0, scalars=None, blockdim=None) -> pk_expr:
+    """c0 + sum scalars[s] * coef + sum blockdim[w] * coef (dicts index -> coef)."""
+    e = pk_expr()
+    e.c0 = c0
+    for s, v in (scalars or {}).items():
+        e.c_scalar[s] = v
+    for w, v in (blockdim or {}).items():
+        e.c_blockdim[w] = v
+    return e
+
+
+def dim_map(grid_dim, scale, extent, offset=0, clamp=False, guard=None) -> pk_dim_map:
+    """scale/extent/offset: int or pk_expr; guard: (lo, hi) of ints/pk_expr or None."""
+    def ex(v):
+        return v if isinstance(v, pk_expr) else expr(int(v))
+    d = pk_dim_map()
+    d.grid_dim = grid_dim
+    d.flags = (PK_DIM_CLAMP if clamp else 0) | (PK_DIM_GUARD if guard is not None else 0)
+    d.scale, d.extent, d.offset = ex(scale), ex(extent), ex(offset)
+    if guard is not None:
+        d.guard_lo, d.guard_hi = ex(guard[0]), ex(guard[1])
+    return d
+
+
+def affine_access(dims) -> pk_affine_access:
+    a = pk_affine_access()
+    a.ndim = len(dims)
+    for i, d in enumerate(dims):
+        a.dim[i] = d
+    return a

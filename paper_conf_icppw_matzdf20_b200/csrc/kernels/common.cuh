@@ -1,0 +1,39 @@
+// common.cuh -- small device helpers shared by the sm_100a kernels.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "pk_api.h"
+
+namespace pk {
+namespace dev {
+
+// Streaming read-only 16-byte load: the stencils read every input byte once, so
+// keep it out of L1 (L2 still catches the neighbour-block halo re-reads).
+__device__ __forceinline__ float4 ld_stream4(const float* p) {
+    float4 r;
+    asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                 : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+                 : "l"(p));
+    return r;
+}
+__device__ __forceinline__ float ld_nc(const float* p) {
+    float r;
+    asm("ld.global.nc.f32 %0, [%1];" : "=f"(r) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ float4 ld_l1(const float* p) {  // expect an L1 hit (re-read by a neighbour warp)
+    float4 r;
+    asm("ld.global.nc.v4.f32 {%0,%1,%2,%3}, [%4];"
+                 : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+                 : "l"(p));
+    return r;
+}
+__device__ __forceinline__ void st4(float* p, float4 v) {
+    asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+                 : "memory");
+}
+
+}  // namespace dev
+}  // namespace pk

@@ -1,0 +1,75 @@
+// builtins.h -- registry of the library's hand-written sm_100a kernels.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "pk_api.h"
+
+namespace pk {
+
+// Everything a launcher needs for one partition (Fig. 4 lines 10-19).
+struct LaunchInfo {
+    const void* fn;
+    dim3 grid;                 // partition grid: max - min (Eq. 10)
+    dim3 block;
+    size_t smem;
+    cudaStream_t stream;
+    int device;
+    void* const* inst;         // [nargs] instance pointers (nullptr for scalars)
+    const void* const* args;   // [nargs] user arg pointers (scalar values)
+    const int64_t* scalars;
+    int nscalars;
+    pk_partition part;
+};
+using LauncherFn = cudaError_t (*)(const LaunchInfo&);
+
+struct Builtin {
+    const char* name;
+    const void* fn;
+    int nargs;
+    int32_t kinds[PK_MAX_ARGS];
+    int32_t partition_dim;
+    // declares the kernel's access taps through pk_declare_affine_access
+    int (*describe)(pk_ctx, pk_kernel);
+    LauncherFn launcher;       // nullptr = generic cudaLaunchKernel
+};
+
+const Builtin* find_builtin(const char* name);
+
+// Per-kernel-file registration (defined in kernels/*.cu)
+extern const Builtin kBuiltinJacobi2d;
+extern const Builtin kBuiltinHotspot2d;
+extern const Builtin kBuiltinHeat3d;
+extern const Builtin kBuiltinNbody;
+
+// Descriptor helpers used by the kernel files' describe() functions.
+inline pk_expr E(int64_t c0) {
+    pk_expr e{};
+    e.c0 = c0;
+    return e;
+}
+inline pk_expr S(int s, int64_t coef = 1, int64_t c0 = 0) {  // coef * scalars[s] + c0
+    pk_expr e{};
+    e.c0 = c0;
+    e.c_scalar[s] = coef;
+    return e;
+}
+inline pk_expr BD(int w, int64_t coef = 1) {  // coef * blockDim[w]
+    pk_expr e{};
+    e.c_blockdim[w] = coef;
+    return e;
+}
+inline pk_dim_map DimMap(int grid_dim, pk_expr scale, pk_expr extent, pk_expr offset,
+                         uint32_t flags, pk_expr glo = E(0), pk_expr ghi = E(0)) {
+    pk_dim_map d{};
+    d.grid_dim = grid_dim;
+    d.flags = flags;
+    d.scale = scale;
+    d.extent = extent;
+    d.offset = offset;
+    d.guard_lo = glo;
+    d.guard_hi = ghi;
+    return d;
+}
+
+}  // namespace pk

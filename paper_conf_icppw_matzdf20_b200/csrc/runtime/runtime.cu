@@ -1,0 +1,908 @@
+// runtime.cu -- the C-ABI of include/pk_api.h: virtual buffers, kernel model
+// records, the Fig. 4 launch replacement (partition -> regions -> stale plan ->
+// transfers -> partitioned launches -> tracker update), D2H/H2D translation.
+//
+// Process model: one host process drives every partition (the paper's single
+// rewritten host program, §8.4).  A partition is a virtual device:
+// several may share one physical GPU (each with its own full-size instance), so
+// P-way partitioning and its transfers are exercised on any GPU count.
+//
+// Ordering replaces the global barrier of Fig. 4 line 8 by a
+// cross-stream event DAG per (buffer, partition) instance:
+//   RAW  a copy out of (b,q) waits for the last writer of (b,q);
+//   WAR  any write into (b,p) -- kernel or incoming copy -- waits for the copies
+//        that read (b,p) since its last write ("readers").
+// PK_MODE_GLOBAL_BARRIER restores the literal host-side barrier.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "../core/host_core.h"
+#include "builtins.h"
+#include "pk_api.h"
+
+using namespace pk;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+int fail(const Status& s) { return fail(s.code, s.msg); }
+
+#define PK_CUDA(call)                                                                   \
+    do {                                                                                \
+        cudaError_t e_ = (call);                                                        \
+        if (e_ != cudaSuccess)                                                          \
+            return fail(PK_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorName(e_) + \
+                                         " (" + cudaGetErrorString(e_) + ")");          \
+    } while (0)
+
+uint64_t now_ns() {
+    return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+               std::chrono::steady_clock::now().time_since_epoch())
+        .count();
+}
+
+enum : uint8_t { W_NONE = 0, W_KERNEL = 1, W_COPY = 2 };
+
+struct Buffer {
+    bool alive = false;
+    int ndim = 0;
+    int64_t shape[PK_MAX_DIMS] = {0, 0, 0, 0};
+    int eb = 0;
+    uint64_t bytes = 0;
+    bool owned = false;
+    std::vector<void*> inst;
+    Tracker tracker;
+    std::vector<uint8_t> last_writer;  // per partition
+    std::vector<uint64_t> readers;     // per partition: mask of partitions whose ev_copy must precede a write
+};
+
+struct Tap {
+    int arg;
+    int mode;
+    pk_affine_access acc;
+};
+
+struct Kernel {
+    std::string name;
+    const void* fn = nullptr;
+    int nargs = 0;
+    int32_t kinds[PK_MAX_ARGS] = {};
+    int32_t partition_dim = -1;
+    std::vector<Tap> taps;
+    LauncherFn launcher = nullptr;
+    uint64_t version = 0;  // bumps when taps change (region cache key)
+};
+
+struct ArgRegions {
+    RangeList r, w;
+};
+struct Regions {
+    bool empty;
+    int64_t box[6];
+    std::vector<ArgRegions> args;  // [nargs]
+};
+
+struct CopyOp {
+    int64_t buf;
+    int src, dst;
+    uint64_t b, e;
+};
+
+struct TimedLaunch {
+    cudaEvent_t start, stop;
+    int part;
+    uint64_t launch_id;
+};
+
+}  // namespace
+
+struct pk_ctx_s {
+    int P = 0;
+    int rank = 0, world = 1;
+    uint32_t init_flags = 0;
+    uint32_t mode = 0;
+    bool host_only = false;
+    std::vector<int> dev, prank;
+    std::vector<cudaStream_t> stream;
+    std::vector<cudaEvent_t> ev_kernel, ev_copy;
+    std::vector<Buffer> bufs;
+    std::vector<Kernel> kernels;
+    pk_stats stats{};
+    std::vector<CopyOp> last_plan;
+    std::unordered_map<std::string, std::shared_ptr<std::vector<Regions>>> region_cache;
+    std::vector<TimedLaunch> pending_timing;
+    std::vector<std::vector<cudaEvent_t>> event_pool;  // per partition (device-bound)
+    uint64_t launch_counter = 0;
+    int cur_device = -1;
+    cudaEvent_t timer_start = nullptr, timer_stop = nullptr;
+    bool timer_running = false;
+
+    bool local(int p) const { return prank[p] == rank; }
+    int set_device(int d) {
+        if (d != cur_device) {
+            cudaError_t e = cudaSetDevice(d);
+            if (e != cudaSuccess)
+                return fail(PK_ERR_CUDA, std::string("cudaSetDevice: ") + cudaGetErrorName(e));
+            cur_device = d;
+        }
+        return PK_OK;
+    }
+};
+
+namespace {
+
+bool valid_buf(pk_ctx c, pk_buf b) { return c && b >= 0 && b < (int64_t)c->bufs.size() && c->bufs[b].alive; }
+bool valid_kernel(pk_ctx c, pk_kernel k) { return c && k >= 0 && k < (int64_t)c->kernels.size(); }
+
+int choose_source(uint64_t mask, int p, int P) {
+    // reading Q5: nearest holder, ties to the lower index
+    int best = -1, bestd = 1 << 30;
+    for (int q = 0; q < P; ++q) {
+        if (!((mask >> q) & 1)) continue;
+        int d = q > p ? q - p : p - q;
+        if (d < bestd) { bestd = d; best = q; }
+    }
+    return best;
+}
+
+int split_dim(const int32_t grid[3], int forced) {
+    if (forced >= 0 && forced <= 2) return forced;
+    for (int w = 2; w >= 0; --w)
+        if (grid[w] > 1) return w;
+    return 0;
+}
+
+// a1: partition p of the grid, box6 = (zmin,zmax,ymin,ymax,xmin,xmax)
+void partition_box(const int32_t grid[3], int P, int p, int w, int64_t box[6]) {
+    int64_t lo[3] = {0, 0, 0}, hi[3] = {grid[0], grid[1], grid[2]};
+    int64_t g = hi[w];
+    lo[w] = (p * g) / P;
+    hi[w] = ((p + 1) * g) / P;
+    box[0] = lo[2]; box[1] = hi[2];
+    box[2] = lo[1]; box[3] = hi[1];
+    box[4] = lo[0]; box[5] = hi[0];
+}
+
+bool box_empty(const int64_t box[6]) { return box[0] >= box[1] || box[2] >= box[3] || box[4] >= box[5]; }
+
+Status arg_ranges(const Kernel& k, int arg, int want_mode, const int64_t box[6], const Buffer& buf,
+                  const EvalEnv& env, RangeList* out) {
+    out->clear();
+    RangeList tmp;
+    for (const Tap& t : k.taps) {
+        if (t.arg != arg) continue;
+        bool is_read = t.mode == PK_READ || t.mode == PK_MAY_WRITE;
+        bool is_write = t.mode == PK_WRITE || t.mode == PK_MAY_WRITE;
+        if ((want_mode == PK_READ && !is_read) || (want_mode == PK_WRITE && !is_write)) continue;
+        Status st = tap_ranges(t.acc, box, buf.ndim, buf.shape, buf.eb, env, &tmp);
+        if (!st.ok()) return st;
+        out->insert(out->end(), tmp.begin(), tmp.end());
+    }
+    canonicalize(out);
+    return Status::Ok();
+}
+
+std::string region_key(const Kernel& k, int64_t kid, const int32_t grid[3], const int32_t block[3],
+                       const int64_t* scalars, int ns, int P, const std::vector<const Buffer*>& bound) {
+    std::string key;
+    key.reserve(256);
+    auto put = [&key](const void* p, size_t n) { key.append((const char*)p, n); };
+    put(&kid, sizeof kid);
+    put(&k.version, sizeof k.version);
+    put(grid, 12);
+    put(block, 12);
+    put(&P, sizeof P);
+    put(&ns, sizeof ns);
+    if (ns) put(scalars, sizeof(int64_t) * ns);
+    for (const Buffer* b : bound) {
+        int64_t z = 0;
+        if (!b) { put(&z, sizeof z); continue; }
+        put(&b->ndim, sizeof b->ndim);
+        put(b->shape, sizeof(int64_t) * b->ndim);
+        put(&b->eb, sizeof b->eb);
+    }
+    return key;
+}
+
+}  // namespace
+
+// ====================================================================== ABI
+extern "C" {
+
+const char* pk_last_error(void) { return g_err.c_str(); }
+const char* pk_version(void) { return "pk 0.1 (sm_100a)"; }
+
+int pk_init(const pk_init_params* prm, pk_ctx* out) {
+    if (!prm || !out) return fail(PK_ERR_INVALID, "null argument");
+    if (prm->nparts < 1 || prm->nparts > PK_MAX_PARTS)
+        return fail(PK_ERR_INVALID, "nparts must be in [1, 64]");
+    if (prm->world_size < 1 || prm->my_rank < 0 || prm->my_rank >= prm->world_size)
+        return fail(PK_ERR_INVALID, "bad rank/world_size");
+    std::unique_ptr<pk_ctx_s> c(new pk_ctx_s());
+    c->P = prm->nparts;
+    c->rank = prm->my_rank;
+    c->world = prm->world_size;
+    c->init_flags = prm->flags;
+    c->host_only = prm->flags & PK_INIT_HOST_ONLY;
+    c->dev.assign(c->P, 0);
+    c->prank.assign(c->P, 0);
+    for (int p = 0; p < c->P; ++p) {
+        if (prm->part_rank) {
+            if (prm->part_rank[p] < 0 || prm->part_rank[p] >= c->world)
+                return fail(PK_ERR_INVALID, "part_rank out of range");
+            c->prank[p] = prm->part_rank[p];
+        }
+    }
+    if (!c->host_only) {
+        if (c->world != 1)
+            return fail(PK_ERR_STATE, "multi-process execution is not implemented (host-only planning only)");
+        int ndev = 0;
+        PK_CUDA(cudaGetDeviceCount(&ndev));
+        if (ndev < 1) return fail(PK_ERR_CUDA, "no CUDA device");
+        for (int p = 0; p < c->P; ++p) {
+            c->dev[p] = prm->part_device ? prm->part_device[p] : p % ndev;
+            if (c->dev[p] < 0 || c->dev[p] >= ndev) return fail(PK_ERR_INVALID, "part_device out of range");
+        }
+        // peer access between every pair of distinct devices in use
+        std::vector<int> used(c->dev);
+        std::sort(used.begin(), used.end());
+        used.erase(std::unique(used.begin(), used.end()), used.end());
+        for (int a : used)
+            for (int b : used) {
+                if (a == b) continue;
+                int can = 0;
+                PK_CUDA(cudaDeviceCanAccessPeer(&can, a, b));
+                if (!can) continue;
+                PK_CUDA(cudaSetDevice(a));
+                cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+                if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+                else if (e != cudaSuccess)
+                    return fail(PK_ERR_CUDA, std::string("cudaDeviceEnablePeerAccess: ") + cudaGetErrorName(e));
+            }
+        c->stream.resize(c->P);
+        c->ev_kernel.resize(c->P);
+        c->ev_copy.resize(c->P);
+        c->event_pool.resize(c->P);
+        for (int p = 0; p < c->P; ++p) {
+            PK_CUDA(cudaSetDevice(c->dev[p]));
+            PK_CUDA(cudaStreamCreateWithFlags(&c->stream[p], cudaStreamNonBlocking));
+            PK_CUDA(cudaEventCreateWithFlags(&c->ev_kernel[p], cudaEventDisableTiming));
+            PK_CUDA(cudaEventCreateWithFlags(&c->ev_copy[p], cudaEventDisableTiming));
+        }
+        c->cur_device = c->dev[c->P - 1];
+    }
+    *out = c.release();
+    return PK_OK;
+}
+
+int pk_synchronize(pk_ctx c) {
+    if (!c) return fail(PK_ERR_INVALID, "null ctx");
+    if (c->host_only) return PK_OK;
+    for (int p = 0; p < c->P; ++p) {
+        if (!c->local(p)) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        PK_CUDA(cudaStreamSynchronize(c->stream[p]));
+    }
+    return PK_OK;
+}
+
+int pk_timer_begin(pk_ctx c) {
+    if (!c) return fail(PK_ERR_INVALID, "null ctx");
+    if (c->host_only) return fail(PK_ERR_STATE, "host-only context has no device timer");
+    if (!c->timer_start) {
+        for (cudaEvent_t* e : {&c->timer_start, &c->timer_stop}) {
+            if (int r = c->set_device(c->dev[0])) return r;
+            PK_CUDA(cudaEventCreate(e));
+        }
+    }
+    if (int r = c->set_device(c->dev[0])) return r;
+    PK_CUDA(cudaEventRecord(c->timer_start, c->stream[0]));
+    for (int p = 1; p < c->P; ++p) {
+        if (!c->local(p)) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->timer_start, 0));
+    }
+    c->timer_running = true;
+    return PK_OK;
+}
+
+int pk_timer_end(pk_ctx c, double* ms) {
+    if (!c || !ms) return fail(PK_ERR_INVALID, "null argument");
+    if (c->host_only || !c->timer_running) return fail(PK_ERR_STATE, "timer not running");
+    for (int p = 1; p < c->P; ++p) {
+        if (!c->local(p)) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        PK_CUDA(cudaEventRecord(c->ev_kernel[p], c->stream[p]));
+        if (int r = c->set_device(c->dev[0])) return r;
+        PK_CUDA(cudaStreamWaitEvent(c->stream[0], c->ev_kernel[p], 0));
+    }
+    if (int r = c->set_device(c->dev[0])) return r;
+    PK_CUDA(cudaEventRecord(c->timer_stop, c->stream[0]));
+    PK_CUDA(cudaEventSynchronize(c->timer_stop));
+    float f = 0.f;
+    PK_CUDA(cudaEventElapsedTime(&f, c->timer_start, c->timer_stop));
+    *ms = f;
+    c->timer_running = false;
+    return PK_OK;
+}
+
+static int drain_timing(pk_ctx c) {
+    for (TimedLaunch& t : c->pending_timing) {
+        if (int r = c->set_device(c->dev[t.part])) return r;
+        PK_CUDA(cudaEventSynchronize(t.stop));
+        float ms = 0.f;
+        PK_CUDA(cudaEventElapsedTime(&ms, t.start, t.stop));
+        c->stats.kernel_ms += ms;
+        c->stats.timed_kernels += 1;
+        c->event_pool[t.part].push_back(t.start);
+        c->event_pool[t.part].push_back(t.stop);
+    }
+    // per launch: max over partitions
+    std::unordered_map<uint64_t, double> mx;
+    for (TimedLaunch& t : c->pending_timing) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, t.start, t.stop);
+        double& v = mx[t.launch_id];
+        v = std::max(v, (double)ms);
+    }
+    for (auto& kv : mx) c->stats.kernel_ms_max_launch += kv.second;
+    c->pending_timing.clear();
+    return PK_OK;
+}
+
+int pk_finalize(pk_ctx c) {
+    if (!c) return PK_OK;
+    if (!c->host_only) {
+        pk_synchronize(c);
+        drain_timing(c);
+        for (size_t b = 0; b < c->bufs.size(); ++b) {
+            Buffer& B = c->bufs[b];
+            if (B.alive && B.owned)
+                for (int p = 0; p < c->P; ++p)
+                    if (B.inst[p]) { cudaSetDevice(c->dev[p]); cudaFree(B.inst[p]); }
+        }
+        for (int p = 0; p < c->P; ++p) {
+            cudaSetDevice(c->dev[p]);
+            cudaStreamDestroy(c->stream[p]);
+            cudaEventDestroy(c->ev_kernel[p]);
+            cudaEventDestroy(c->ev_copy[p]);
+            for (cudaEvent_t e : c->event_pool[p]) cudaEventDestroy(e);
+        }
+        if (c->timer_start) {
+            cudaSetDevice(c->dev[0]);
+            cudaEventDestroy(c->timer_start);
+            cudaEventDestroy(c->timer_stop);
+        }
+    }
+    delete c;
+    return PK_OK;
+}
+
+// ------------------------------------------------------------------ buffers
+int pk_register_buffer(pk_ctx c, int ndim, const int64_t* shape, int elem_bytes, void* const* dev_ptrs,
+                       const void* host_init, pk_buf* out) {
+    if (!c || !shape || !out) return fail(PK_ERR_INVALID, "null argument");
+    if (ndim < 1 || ndim > PK_MAX_DIMS) return fail(PK_ERR_INVALID, "ndim must be 1..4");
+    if (elem_bytes < 1) return fail(PK_ERR_INVALID, "elem_bytes must be >= 1");
+    Buffer B;
+    B.ndim = ndim;
+    B.eb = elem_bytes;
+    int64_t n = elem_bytes;
+    for (int k = 0; k < ndim; ++k) {
+        if (shape[k] < 0) return fail(PK_ERR_INVALID, "negative shape");
+        B.shape[k] = shape[k];
+        if (!mul_ok(n, shape[k], &n)) return fail(PK_ERR_OVERFLOW, "buffer size overflows int64");
+    }
+    B.bytes = (uint64_t)n;
+    B.inst.assign(c->P, nullptr);
+    B.last_writer.assign(c->P, W_NONE);
+    B.readers.assign(c->P, 0);
+    const uint64_t all = c->P == 64 ? ~0ull : ((1ull << c->P) - 1);
+    B.tracker.init(B.bytes, all);  // reading Q3: undefined contents are valid everywhere
+    if (!c->host_only) {
+        if (dev_ptrs) {
+            for (int p = 0; p < c->P; ++p) {
+                if (!c->local(p)) continue;
+                if (!dev_ptrs[p] && B.bytes) return fail(PK_ERR_INVALID, "null instance pointer");
+                if (((uintptr_t)dev_ptrs[p]) % 16) return fail(PK_ERR_INVALID, "instance not 16-byte aligned");
+                B.inst[p] = dev_ptrs[p];
+            }
+        } else {
+            B.owned = true;
+            for (int p = 0; p < c->P; ++p) {
+                if (!c->local(p) || !B.bytes) continue;
+                if (int r = c->set_device(c->dev[p])) return r;
+                cudaError_t e = cudaMalloc(&B.inst[p], B.bytes);
+                if (e != cudaSuccess) {
+                    cudaGetLastError();
+                    for (int q = 0; q < p; ++q)
+                        if (B.inst[q]) { cudaSetDevice(c->dev[q]); cudaFree(B.inst[q]); }
+                    c->cur_device = -1;
+                    return fail(PK_ERR_OOM, "cudaMalloc of a buffer instance failed");
+                }
+            }
+        }
+    }
+    B.alive = true;
+    c->bufs.push_back(std::move(B));
+    *out = (pk_buf)(c->bufs.size() - 1);
+    if (host_init) {
+        int r = pk_copy_from_host(c, *out, host_init, c->bufs[*out].bytes);
+        if (r) return r;
+    }
+    return PK_OK;
+}
+
+int pk_buffer_instance(pk_ctx c, pk_buf b, int part, void** dev_ptr) {
+    if (!valid_buf(c, b) || part < 0 || part >= c->P || !dev_ptr) return fail(PK_ERR_INVALID, "bad argument");
+    *dev_ptr = c->bufs[b].inst[part];
+    return PK_OK;
+}
+
+int pk_unregister_buffer(pk_ctx c, pk_buf b) {
+    if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "bad buffer");
+    Buffer& B = c->bufs[b];
+    if (!c->host_only && B.owned) {
+        if (int r = pk_synchronize(c)) return r;
+        for (int p = 0; p < c->P; ++p)
+            if (B.inst[p]) {
+                if (int r = c->set_device(c->dev[p])) return r;
+                PK_CUDA(cudaFree(B.inst[p]));
+            }
+    }
+    B = Buffer();
+    return PK_OK;
+}
+
+// Wait, on partition p's stream, for every copy that read (b,p) since its last write.
+static int wait_readers(pk_ctx c, Buffer& B, int p) {
+    uint64_t m = B.readers[p];
+    for (int q = 0; m; ++q, m >>= 1) {
+        if (!(m & 1) || q == p) continue;
+        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_copy[q], 0));
+    }
+    B.readers[p] = 0;
+    return PK_OK;
+}
+
+int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
+    if (!valid_buf(c, b) || !host) return fail(PK_ERR_INVALID, "bad argument");
+    Buffer& B = c->bufs[b];
+    if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (H2D copies the whole virtual buffer)");
+    const uint64_t n = B.bytes / B.eb;
+    uint64_t t0 = now_ns();
+    if (!c->host_only) {
+        if (int r = pk_synchronize(c)) return r;  // WAR against everything in flight
+        for (int p = 0; p < c->P; ++p) {
+            if (!c->local(p)) continue;
+            uint64_t lo = (uint64_t)p * n / c->P * B.eb, hi = (uint64_t)(p + 1) * n / c->P * B.eb;
+            if (hi <= lo) continue;
+            if (int r = c->set_device(c->dev[p])) return r;
+            PK_CUDA(cudaMemcpyAsync((char*)B.inst[p] + lo, (const char*)host + lo, hi - lo,
+                                    cudaMemcpyHostToDevice, c->stream[p]));
+        }
+        if (int r = pk_synchronize(c)) return r;
+        for (int p = 0; p < c->P; ++p) { B.last_writer[p] = W_NONE; B.readers[p] = 0; }
+    }
+    // linear distribution; tracker says slab p lives on p (reading Q2)
+    for (int p = 0; p < c->P; ++p) {
+        uint64_t lo = (uint64_t)p * n / c->P * B.eb, hi = (uint64_t)(p + 1) * n / c->P * B.eb;
+        if (hi > lo) B.tracker.assign(RangeList{Range{lo, hi}}, 1ull << p);
+    }
+    c->stats.h2d_bytes += B.bytes;
+    (void)t0;
+    return PK_OK;
+}
+
+int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
+    if (!valid_buf(c, b) || !host) return fail(PK_ERR_INVALID, "bad argument");
+    Buffer& B = c->bufs[b];
+    if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (D2H gathers the whole virtual buffer)");
+    if (c->host_only) return fail(PK_ERR_STATE, "host-only context holds no data");
+    // query all segments, copy each from a partition that holds it.
+    struct Piece { uint64_t b, e; int src; };
+    std::vector<Piece> pieces;
+    for (const Seg& s : B.tracker.segments()) {
+        int src = -1;
+        for (int q = 0; q < c->P; ++q)
+            if (((s.mask >> q) & 1) && c->local(q)) { src = q; break; }
+        if (src < 0) return fail(PK_ERR_STATE, "segment held by no local partition");
+        if (!pieces.empty() && pieces.back().src == src && pieces.back().e == s.b) pieces.back().e = s.e;
+        else pieces.push_back({s.b, s.e, src});
+    }
+    for (const Piece& pc : pieces) {
+        if (int r = c->set_device(c->dev[pc.src])) return r;
+        PK_CUDA(cudaMemcpyAsync((char*)host + pc.b, (const char*)B.inst[pc.src] + pc.b, pc.e - pc.b,
+                                cudaMemcpyDeviceToHost, c->stream[pc.src]));
+    }
+    if (int r = pk_synchronize(c)) return r;
+    c->stats.d2h_bytes += B.bytes;
+    return PK_OK;
+}
+
+// ------------------------------------------------------------------ kernels
+int pk_register_kernel(pk_ctx c, const char* name, const void* fn, int nargs, const int32_t* arg_kind,
+                       int32_t partition_dim, pk_kernel* out) {
+    if (!c || !out || !arg_kind) return fail(PK_ERR_INVALID, "null argument");
+    if (nargs < 0 || nargs > PK_MAX_ARGS) return fail(PK_ERR_INVALID, "nargs must be 0..16");
+    if (partition_dim < -1 || partition_dim > 2) return fail(PK_ERR_INVALID, "partition_dim must be -1..2");
+    Kernel k;
+    k.name = name ? name : "";
+    k.fn = fn;
+    k.nargs = nargs;
+    k.partition_dim = partition_dim;
+    for (int i = 0; i < nargs; ++i) {
+        if (arg_kind[i] != PK_ARG_BUFFER && arg_kind[i] != PK_ARG_SCALAR)
+            return fail(PK_ERR_INVALID, "arg_kind must be PK_ARG_BUFFER or PK_ARG_SCALAR");
+        k.kinds[i] = arg_kind[i];
+    }
+    c->kernels.push_back(std::move(k));
+    *out = (pk_kernel)(c->kernels.size() - 1);
+    return PK_OK;
+}
+
+int pk_declare_affine_access(pk_ctx c, pk_kernel k, int arg, int mode, const pk_affine_access* tap) {
+    if (!valid_kernel(c, k) || !tap) return fail(PK_ERR_INVALID, "bad kernel or null tap");
+    Kernel& K = c->kernels[k];
+    if (arg < 0 || arg >= K.nargs || K.kinds[arg] != PK_ARG_BUFFER)
+        return fail(PK_ERR_INVALID, "arg_index is not a buffer argument");
+    if (mode != PK_READ && mode != PK_WRITE && mode != PK_MAY_WRITE) return fail(PK_ERR_INVALID, "bad mode");
+    if (tap->ndim < 1 || tap->ndim > PK_MAX_DIMS) return fail(PK_ERR_INVALID, "tap ndim must be 1..4");
+    int used[3] = {0, 0, 0};
+    for (int d = 0; d < tap->ndim; ++d) {
+        int g = tap->dim[d].grid_dim;
+        if (g < -1 || g > 2) return fail(PK_ERR_INVALID, "grid_dim must be -1..2");
+        if (g >= 0 && used[g]++) return fail(PK_ERR_INVALID, "a grid dimension drives two array dimensions");
+    }
+    K.taps.push_back(Tap{arg, mode, *tap});
+    K.version++;
+    return PK_OK;
+}
+
+const void* pk_builtin_fn(const char* name) {
+    const Builtin* b = find_builtin(name);
+    return b ? b->fn : nullptr;
+}
+
+int pk_builtin_kernel(pk_ctx c, const char* name, pk_kernel* out) {
+    const Builtin* b = find_builtin(name);
+    if (!b) return fail(PK_ERR_INVALID, std::string("unknown builtin kernel '") + (name ? name : "") + "'");
+    int r = pk_register_kernel(c, b->name, b->fn, b->nargs, b->kinds, b->partition_dim, out);
+    if (r) return r;
+    c->kernels[*out].launcher = b->launcher;
+    return b->describe(c, *out);
+}
+
+int pk_partition_grid(pk_ctx c, pk_kernel k, const int32_t grid[3], int part, int64_t part_out[6]) {
+    if (!valid_kernel(c, k) || !grid || !part_out || part < 0 || part >= c->P)
+        return fail(PK_ERR_INVALID, "bad argument");
+    partition_box(grid, c->P, part, split_dim(grid, c->kernels[k].partition_dim), part_out);
+    return PK_OK;
+}
+
+int pk_enumerate(pk_ctx c, pk_kernel k, int arg, int mode, pk_buf b, const int64_t part[6],
+                 const int32_t block[3], const int64_t* scalars, int ns, pk_range_cb cb, void* user) {
+    if (!valid_kernel(c, k) || !valid_buf(c, b) || !part || !block || !cb) return fail(PK_ERR_INVALID, "bad argument");
+    if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
+    const Kernel& K = c->kernels[k];
+    if (arg < 0 || arg >= K.nargs) return fail(PK_ERR_INVALID, "bad arg index");
+    EvalEnv env{scalars, ns, {block[0], block[1], block[2]}};
+    RangeList r;
+    Status st = arg_ranges(K, arg, mode == PK_WRITE ? PK_WRITE : PK_READ, part, c->bufs[b], env, &r);
+    if (!st.ok()) return fail(st);
+    for (const Range& x : r) cb(user, x.b, x.e);
+    return PK_OK;
+}
+
+int pk_tracker_dump(pk_ctx c, pk_buf b, pk_segment_cb cb, void* user) {
+    if (!valid_buf(c, b) || !cb) return fail(PK_ERR_INVALID, "bad argument");
+    for (const Seg& s : c->bufs[b].tracker.segments()) cb(user, s.b, s.e, s.mask);
+    return PK_OK;
+}
+
+int pk_last_plan(pk_ctx c, pk_copy_cb cb, void* user) {
+    if (!c || !cb) return fail(PK_ERR_INVALID, "bad argument");
+    for (const CopyOp& o : c->last_plan) cb(user, o.buf, o.src, o.dst, o.b, o.e);
+    return PK_OK;
+}
+
+int pk_get_stats(pk_ctx c, pk_stats* out) {
+    if (!c || !out) return fail(PK_ERR_INVALID, "bad argument");
+    if (!c->host_only && !c->pending_timing.empty())
+        if (int r = drain_timing(c)) return r;
+    *out = c->stats;
+    return PK_OK;
+}
+
+int pk_reset_stats(pk_ctx c) {
+    if (!c) return fail(PK_ERR_INVALID, "bad argument");
+    if (!c->host_only && !c->pending_timing.empty())
+        if (int r = drain_timing(c)) return r;
+    c->stats = pk_stats{};
+    return PK_OK;
+}
+
+int pk_set_mode(pk_ctx c, uint32_t flags) {
+    if (!c) return fail(PK_ERR_INVALID, "bad argument");
+    if (flags & ~0x1Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
+    c->mode = flags;
+    return PK_OK;
+}
+uint32_t pk_get_mode(pk_ctx c) { return c ? c->mode : 0; }
+
+// ------------------------------------------------------------------ Fig. 4
+int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
+                          const void* const* args, const int64_t* scalars, int ns) {
+    if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
+    if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
+    const Kernel& K = c->kernels[k];
+    if (K.nargs && !args) return fail(PK_ERR_INVALID, "null args");
+    for (int w = 0; w < 3; ++w)
+        if (grid[w] < 0 || block[w] < 1) return fail(PK_ERR_INVALID, "bad grid/block");
+    const int P = c->P;
+    // resolve buffer arguments
+    std::vector<const Buffer*> bound(K.nargs, nullptr);
+    std::vector<int64_t> bid(K.nargs, -1);
+    for (int a = 0; a < K.nargs; ++a) {
+        if (K.kinds[a] != PK_ARG_BUFFER) continue;
+        if (!args[a]) return fail(PK_ERR_INVALID, "null buffer argument");
+        pk_buf b = *(const pk_buf*)args[a];
+        if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "argument " + std::to_string(a) + " is not a live buffer");
+        bound[a] = &c->bufs[b];
+        bid[a] = b;
+    }
+    const uint32_t mode = c->mode;
+    const bool track = !(mode & PK_MODE_NO_TRACKING);
+    const bool transfer = track && !(mode & PK_MODE_NO_TRANSFERS);
+    const bool single_owner = mode & PK_MODE_SINGLE_OWNER;
+    uint64_t t0 = now_ns();
+
+    // ---- a1 + a2: partition boxes and regions (cached) ----
+    const int w = split_dim(grid, K.partition_dim);
+    std::shared_ptr<std::vector<Regions>> regs;
+    std::string key = region_key(K, k, grid, block, scalars, ns, P, bound);
+    auto it = c->region_cache.find(key);
+    uint64_t t1 = now_ns();
+    if (it != c->region_cache.end()) {
+        regs = it->second;
+    } else {
+        regs = std::make_shared<std::vector<Regions>>(P);
+        EvalEnv env{scalars, ns, {block[0], block[1], block[2]}};
+        for (int p = 0; p < P; ++p) {
+            Regions& R = (*regs)[p];
+            partition_box(grid, P, p, w, R.box);
+            R.empty = box_empty(R.box);
+            R.args.resize(K.nargs);
+            if (R.empty) continue;
+            for (int a = 0; a < K.nargs; ++a) {
+                if (!bound[a]) continue;
+                Status st = arg_ranges(K, a, PK_READ, R.box, *bound[a], env, &R.args[a].r);
+                if (st.ok()) st = arg_ranges(K, a, PK_WRITE, R.box, *bound[a], env, &R.args[a].w);
+                if (!st.ok()) return fail(st);
+            }
+        }
+        if (c->region_cache.size() > 4096) c->region_cache.clear();
+        c->region_cache.emplace(key, regs);
+    }
+    c->stats.host_ns_partition += t1 - t0;
+    uint64_t t2 = now_ns();
+    c->stats.host_ns_regions += t2 - t1;
+
+    // per (partition, distinct buffer): merged read / write sets
+    struct BufSets { int64_t b; RangeList r, w; };
+    std::vector<std::vector<BufSets>> sets(P);
+    if (track) {
+        for (int p = 0; p < P; ++p) {
+            const Regions& R = (*regs)[p];
+            if (R.empty) continue;
+            for (int a = 0; a < K.nargs; ++a) {
+                if (!bound[a]) continue;
+                BufSets* bs = nullptr;
+                for (auto& x : sets[p]) if (x.b == bid[a]) bs = &x;
+                if (!bs) { sets[p].push_back(BufSets{bid[a], {}, {}}); bs = &sets[p].back(); }
+                if (!R.args[a].r.empty()) bs->r = bs->r.empty() ? R.args[a].r : union_ranges(bs->r, R.args[a].r);
+                if (!R.args[a].w.empty()) bs->w = bs->w.empty() ? R.args[a].w : union_ranges(bs->w, R.args[a].w);
+            }
+        }
+        // WAW across partitions: reject before anything happens
+        std::unordered_map<int64_t, std::vector<std::pair<Range, int>>> allw;
+        for (int p = 0; p < P; ++p)
+            for (auto& bs : sets[p])
+                for (const Range& x : bs.w) allw[bs.b].push_back({x, p});
+        for (auto& kv : allw) {
+            auto& v = kv.second;
+            std::sort(v.begin(), v.end(), [](const std::pair<Range, int>& a, const std::pair<Range, int>& b) {
+                return a.first.b < b.first.b;
+            });
+            for (size_t i = 1; i < v.size(); ++i)
+                if (v[i].first.b < v[i - 1].first.e && v[i].second != v[i - 1].second)
+                    return fail(PK_ERR_WRITE_OVERLAP, "partitions " + std::to_string(v[i - 1].second) + " and " +
+                                                          std::to_string(v[i].second) +
+                                                          " write the same bytes of buffer " + std::to_string(kv.first));
+        }
+    }
+
+    // ---- a3: stale detection + transfer plan against the pre-launch state ----
+    c->last_plan.clear();
+    if (track) {
+        for (int p = 0; p < P; ++p) {
+            for (auto& bs : sets[p]) {
+                const Buffer& B = c->bufs[bs.b];
+                for (const Range& x : bs.r) {
+                    B.tracker.query(x.b, x.e, [&](uint64_t lo, uint64_t hi, uint64_t m) {
+                        if ((m >> p) & 1) return;
+                        c->stats.stale_bytes += hi - lo;
+                        int q = choose_source(m, p, P);
+                        if (!c->last_plan.empty()) {
+                            CopyOp& l = c->last_plan.back();
+                            if (l.buf == bs.b && l.src == q && l.dst == p && l.e == lo) { l.e = hi; return; }
+                        }
+                        c->last_plan.push_back(CopyOp{bs.b, q, p, lo, hi});
+                    });
+                }
+            }
+        }
+        if (!single_owner)  // validity map: a reader becomes a co-holder (reading Q4)
+            for (int p = 0; p < P; ++p)
+                for (auto& bs : sets[p])
+                    if (!bs.r.empty()) c->bufs[bs.b].tracker.add_bit(bs.r, p);
+    }
+    uint64_t t3 = now_ns();
+    c->stats.host_ns_plan += t3 - t2;
+    c->stats.launches += 1;
+    const uint64_t launch_id = c->launch_counter++;
+
+    // ---- a4 + a5: transfers, pulled on the destination stream ----
+    if (!c->host_only) {
+        if (transfer && !c->last_plan.empty()) {
+            size_t i = 0;
+            while (i < c->last_plan.size()) {
+                const int p = c->last_plan[i].dst;
+                size_t j = i;
+                while (j < c->last_plan.size() && c->last_plan[j].dst == p) ++j;
+                if (int r = c->set_device(c->dev[p])) return r;
+                // WAR on the destination instances + RAW on each source's last writer
+                uint64_t waited_src = 0;
+                for (size_t t = i; t < j; ++t) {
+                    const CopyOp& o = c->last_plan[t];
+                    Buffer& B = c->bufs[o.buf];
+                    if (B.readers[p]) if (int r = wait_readers(c, B, p)) return r;
+                    const uint8_t lw = B.last_writer[o.src];
+                    uint64_t bit = 1ull << o.src;
+                    if (lw != W_NONE && !(waited_src & bit)) {
+                        PK_CUDA(cudaStreamWaitEvent(c->stream[p], lw == W_KERNEL ? c->ev_kernel[o.src]
+                                                                                 : c->ev_copy[o.src], 0));
+                        waited_src |= bit;
+                    }
+                }
+                for (size_t t = i; t < j; ++t) {
+                    const CopyOp& o = c->last_plan[t];
+                    Buffer& B = c->bufs[o.buf];
+                    char* dst = (char*)B.inst[p] + o.b;
+                    const char* src = (const char*)B.inst[o.src] + o.b;
+                    if (c->dev[o.src] == c->dev[p])
+                        PK_CUDA(cudaMemcpyAsync(dst, src, o.e - o.b, cudaMemcpyDeviceToDevice, c->stream[p]));
+                    else
+                        PK_CUDA(cudaMemcpyPeerAsync(dst, c->dev[p], src, c->dev[o.src], o.e - o.b, c->stream[p]));
+                    c->stats.copies += 1;
+                    c->stats.moved_bytes += o.e - o.b;
+                    if (o.src < 16 && p < 16) c->stats.pair_bytes[o.src][p] += o.e - o.b;
+                }
+                PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
+                for (size_t t = i; t < j; ++t) {
+                    const CopyOp& o = c->last_plan[t];
+                    Buffer& B = c->bufs[o.buf];
+                    B.readers[o.src] |= 1ull << p;
+                    B.last_writer[p] = W_COPY;
+                }
+                i = j;
+            }
+        }
+        if (mode & PK_MODE_GLOBAL_BARRIER)  // Fig. 4 line 8, literally
+            if (int r = pk_synchronize(c)) return r;
+    }
+    uint64_t t4 = now_ns();
+
+    // ---- a6: partitioned launches (Eq. 8-10) ----
+    if (!c->host_only) {
+        void* inst[PK_MAX_ARGS];
+        void* argv[PK_MAX_ARGS + 1];
+        for (int p = 0; p < P; ++p) {
+            const Regions& R = (*regs)[p];
+            if (R.empty || !c->local(p)) continue;
+            if (int r = c->set_device(c->dev[p])) return r;
+            // WAR: writes into (b,p) wait for copies that read (b,p)
+            if (track) {
+                for (auto& bs : sets[p])
+                    if (!bs.w.empty() && c->bufs[bs.b].readers[p])
+                        if (int r = wait_readers(c, c->bufs[bs.b], p)) return r;
+            } else {
+                for (int a = 0; a < K.nargs; ++a)
+                    if (bound[a] && c->bufs[bid[a]].readers[p])
+                        if (int r = wait_readers(c, c->bufs[bid[a]], p)) return r;
+            }
+            pk_partition part;
+            part.min[0] = (int32_t)R.box[4]; part.max[0] = (int32_t)R.box[5];
+            part.min[1] = (int32_t)R.box[2]; part.max[1] = (int32_t)R.box[3];
+            part.min[2] = (int32_t)R.box[0]; part.max[2] = (int32_t)R.box[1];
+            for (int d = 0; d < 3; ++d) part.grid[d] = grid[d];
+            for (int a = 0; a < K.nargs; ++a) {
+                if (bound[a]) { inst[a] = c->bufs[bid[a]].inst[p]; argv[a] = &inst[a]; }
+                else { inst[a] = nullptr; argv[a] = const_cast<void*>(args[a]); }
+            }
+            argv[K.nargs] = &part;
+            dim3 g(part.max[0] - part.min[0], part.max[1] - part.min[1], part.max[2] - part.min[2]);
+            dim3 bl(block[0], block[1], block[2]);
+            cudaEvent_t e0 = nullptr, e1 = nullptr;
+            if (mode & PK_MODE_TIME_KERNELS) {
+                auto& pool = c->event_pool[p];
+                for (cudaEvent_t* e : {&e0, &e1}) {
+                    if (!pool.empty()) { *e = pool.back(); pool.pop_back(); }
+                    else PK_CUDA(cudaEventCreate(e));
+                }
+                PK_CUDA(cudaEventRecord(e0, c->stream[p]));
+            }
+            cudaError_t err;
+            if (K.launcher) {
+                LaunchInfo li{K.fn, g, bl, smem, c->stream[p], c->dev[p], inst, args, scalars, ns, part};
+                err = K.launcher(li);
+            } else {
+                err = cudaLaunchKernel(K.fn, g, bl, argv, smem, c->stream[p]);
+            }
+            if (err != cudaSuccess)
+                return fail(PK_ERR_CUDA, "launch of '" + K.name + "' on partition " + std::to_string(p) + ": " +
+                                             cudaGetErrorName(err) + " (" + cudaGetErrorString(err) + ")");
+            if (mode & PK_MODE_TIME_KERNELS) {
+                PK_CUDA(cudaEventRecord(e1, c->stream[p]));
+                c->pending_timing.push_back(TimedLaunch{e0, e1, p, launch_id});
+            }
+            if (P > 1) PK_CUDA(cudaEventRecord(c->ev_kernel[p], c->stream[p]));
+            c->stats.kernel_launches += 1;
+            for (int a = 0; a < K.nargs; ++a)
+                if (bound[a]) {
+                    bool writes = false;
+                    for (const Tap& t : K.taps)
+                        if (t.arg == a && t.mode != PK_READ) writes = true;
+                    if (writes || !track) c->bufs[bid[a]].last_writer[p] = (P > 1) ? W_KERNEL : W_NONE;
+                }
+        }
+    } else {
+        for (int p = 0; p < P; ++p)
+            if (!(*regs)[p].empty && c->local(p)) c->stats.kernel_launches += 1;
+    }
+    uint64_t t5 = now_ns();
+    c->stats.host_ns_issue += (t4 - t3) + (t5 - t4);
+
+    // ---- a7: tracker update with the write sets, kernels running ----
+    if (track)
+        for (int p = 0; p < P; ++p)
+            for (auto& bs : sets[p])
+                if (!bs.w.empty()) c->bufs[bs.b].tracker.assign(bs.w, 1ull << p);
+    c->stats.host_ns_update += now_ns() - t5;
+    return PK_OK;
+}
+
+}  // extern "C"
+
+namespace pk {
+const Builtin* find_builtin(const char* name) {
+    if (!name) return nullptr;
+    static const Builtin* all[] = {&kBuiltinJacobi2d, &kBuiltinHotspot2d, &kBuiltinHeat3d, &kBuiltinNbody};
+    for (const Builtin* b : all)
+        if (std::strcmp(b->name, name) == 0) return b;
+    return nullptr;
+}
+}  // namespace pk

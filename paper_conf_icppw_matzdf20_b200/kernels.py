@@ -1,0 +1,142 @@
+"""Launch geometry of the builtin sm_100a kernels (their published launch contract,
+DESIGN.md §4) and user-side programs that drive them through the C-ABI.
+
+These are the single-device host programs of the paper's benchmarks (P:L948-954
+Table 1) written against the pk_* calls: register buffers (cudaMalloc +
+cudaMemcpy replacements), launch the kernel repeatedly through the
+launch replacement (Fig. 4), gather the result.  No arithmetic of
+the method happens here.
+"""
+from __future__ import annotations
+
+import math
+
+from . import abi
+
+# ---------------------------------------------------------------- geometry
+JACOBI_BLOCK = (32, 8, 1)
+HOTSPOT_BDX, HOTSPOT_TY = 128, 64
+HEAT_BDY, HEAT_ZC = 8, 64
+NBODY_BDX, NBODY_PER_THREAD = 256, 2
+
+
+def _cdiv(a, b):
+    return -(-a // b)
+
+
+def jacobi2d_launch(h, w, block=JACOBI_BLOCK):
+    return (_cdiv(w, block[0]), _cdiv(h, block[1]), 1), tuple(block), [h, w]
+
+
+def hotspot2d_launch(h, w, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX):
+    return (_cdiv(w, 4 * bdx), _cdiv(h, ty), 1), (bdx, 1, 1), [h, w, ty]
+
+
+def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
+    return (_cdiv(w, 128), _cdiv(h, bdy), _cdiv(d, zc)), (32, bdy, 1), [d, h, w, zc]
+
+
+def nbody_launch(n, bdx=NBODY_BDX):
+    return (_cdiv(n, NBODY_PER_THREAD * bdx), 1, 1), (bdx, 1, 1), [n]
+
+
+# ---------------------------------------------------------------- programs
+class Problem:
+    """A registered builtin kernel plus its ping-pong buffers on one context."""
+
+    def __init__(self, ctx, kernel_name):
+        self.ctx = ctx
+        self.k = abi.pk_builtin_kernel(ctx, kernel_name)
+        self.bufs = []
+
+    def buffer(self, shape, elem_bytes=4, host=None, dev_ptrs=None):
+        b = abi.pk_register_buffer(self.ctx, shape, elem_bytes, dev_ptrs=dev_ptrs, host_init=host)
+        self.bufs.append(b)
+        return b
+
+    def launch(self, grid, block, args, scalars):
+        abi.pk_launch_partitioned(self.ctx, self.k, grid, block, args, scalars)
+
+
+def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK):
+    """C1: both buffers carry the Dirichlet boundary (uploaded); returns the buffer id
+    that holds the result after `iters` sweeps."""
+    h, w = u_host.shape
+    pr = Problem(ctx, "jacobi2d")
+    u0 = pr.buffer((h, w), 4, host=u_host)
+    u1 = pr.buffer((h, w), 4, host=u_host)
+    grid, blk, sc = jacobi2d_launch(h, w, block)
+    for t in range(iters):
+        a, b = (u0, u1) if t % 2 == 0 else (u1, u0)
+        pr.launch(grid, blk, [a, b, h, w], sc)
+    return pr, (u0 if iters % 2 == 0 else u1)
+
+
+def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None):
+    h, w = temp_host.shape
+    pr = Problem(ctx, "hotspot2d")
+    t0 = pr.buffer((h, w), 4, host=temp_host, dev_ptrs=dev_ptrs[0] if dev_ptrs else None)
+    t1 = pr.buffer((h, w), 4, dev_ptrs=dev_ptrs[1] if dev_ptrs else None)   # undefined (reading Q3)
+    pw = pr.buffer((h, w), 4, host=power_host, dev_ptrs=dev_ptrs[2] if dev_ptrs else None)
+    pr.geom = hotspot2d_launch(h, w, ty, bdx)
+    pr.hw = (h, w)
+    pr.tb = (t0, t1, pw)
+    return pr
+
+
+def hotspot2d_iterate(pr, iters, start=0):
+    (t0, t1, pw), (h, w) = pr.tb, pr.hw
+    grid, blk, sc = pr.geom
+    for t in range(start, start + iters):
+        a, b = (t0, t1) if t % 2 == 0 else (t1, t0)
+        pr.launch(grid, blk, [a, pw, b, h, w, sc[2]], sc)
+    return t1 if (start + iters) % 2 == 1 else t0
+
+
+def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY):
+    d, h, w = u_host.shape
+    pr = Problem(ctx, "heat3d")
+    u0 = pr.buffer((d, h, w), 4, host=u_host)
+    u1 = pr.buffer((d, h, w), 4)
+    pr.geom = heat3d_launch(d, h, w, zc, bdy)
+    pr.shape = (d, h, w)
+    pr.ub = (u0, u1)
+    return pr
+
+
+def heat3d_iterate(pr, iters, start=0):
+    (u0, u1), (d, h, w) = pr.ub, pr.shape
+    grid, blk, sc = pr.geom
+    for t in range(start, start + iters):
+        a, b = (u0, u1) if t % 2 == 0 else (u1, u0)
+        pr.launch(grid, blk, [a, b, d, h, w, sc[3]], sc)
+    return u1 if (start + iters) % 2 == 1 else u0
+
+
+def nbody_setup(ctx, pos_host, vel_host, bdx=NBODY_BDX):
+    n = pos_host.shape[0]
+    pr = Problem(ctx, "nbody")
+    p0 = pr.buffer((n,), 16, host=pos_host)
+    p1 = pr.buffer((n,), 16)
+    v = pr.buffer((n,), 16, host=vel_host)
+    pr.geom = nbody_launch(n, bdx)
+    pr.n = n
+    pr.nb = (p0, p1, v)
+    return pr
+
+
+def nbody_iterate(pr, steps, start=0):
+    (p0, p1, v), n = pr.nb, pr.n
+    grid, blk, sc = pr.geom
+    for s in range(start, start + steps):
+        a, b = (p0, p1) if s % 2 == 0 else (p1, p0)
+        pr.launch(grid, blk, [a, v, b, n], sc)
+    return (p1 if (start + steps) % 2 == 1 else p0), v
+
+
+def flops_per_interaction():
+    return 20  # conventional count for the softened all-pairs kernel (SURVEY §8(d) [ext])
+
+
+def isqrt(n):
+    return int(math.isqrt(n))

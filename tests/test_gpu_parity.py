@@ -1,0 +1,234 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the oracle, and P-way vs 1-way.
+
+Bars (BASELINE.json north_star):
+  - partitioned results bit-identical to the 1-partition GPU result;
+  - fp32 kernels within 1e-5 relative of the fp64 oracle (reading Q18 metric);
+  - stale/moved bytes equal to the closed-form minimum; moved == stale;
+  - PK_MODE_NO_TRANSFERS (beta) must change the result (negative control).
+P > 1 runs as virtual partitions on cuda:0 (one full-size instance each).
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import closed_forms as cf
+from oracle import kernels as ok
+from paper_conf_icppw_matzdf20_b200 import abi
+from paper_conf_icppw_matzdf20_b200 import kernels as K
+from tests.gpu_util import fetch, gpu_ctx, rel_ok
+
+pytestmark = pytest.mark.gpu
+
+
+# ------------------------------------------------------------------ C1 Jacobi
+def _jacobi(u, iters, P, mode=0, block=K.JACOBI_BLOCK):
+    ctx = gpu_ctx(P, mode)
+    pr, out = K.jacobi2d_program(ctx, u, iters, block)
+    res = fetch(ctx, out, u.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st
+
+
+def test_c1_jacobi_512_p2_oracle_stale_and_bitwise():
+    u = synth.jacobi_grid(512, 512)
+    g1, s1 = _jacobi(u, 10, 1)
+    g2, s2 = _jacobi(u, 10, 2)
+    assert np.array_equal(g1, g2)
+    ok_, err = rel_ok(g2, ok.jacobi2d(u, 10), 1e-5)
+    assert ok_, err
+    assert s2["stale_bytes"] == 40800 == s2["moved_bytes"]
+    assert s1["stale_bytes"] == 0 and s1["moved_bytes"] == 0
+    assert s2["kernel_launches"] == 20 and s2["pair_bytes"][0][1] == s2["pair_bytes"][1][0] == 20400
+
+
+def test_c1_harmonic_fixed_point_bit_exact_on_gpu():
+    n = 512
+    i = np.arange(n, dtype=np.float32)[:, None]
+    u = (i * i.T).astype(np.float32)
+    g, _ = _jacobi(u, 10, 2)
+    assert np.array_equal(g, u)
+
+
+@pytest.mark.parametrize("h,w", [(37, 50), (64, 64), (130, 257)])
+@pytest.mark.parametrize("P", [3, 5, 8])
+def test_jacobi_ragged_bitwise(h, w, P):
+    u = synth.uniform((h, w), 0, 1, seed=h * w)
+    g1, _ = _jacobi(u, 7, 1)
+    gp, st = _jacobi(u, 7, P)
+    assert np.array_equal(g1, gp)
+    assert st["moved_bytes"] == st["stale_bytes"]
+    assert rel_ok(gp, ok.jacobi2d(u, 7), 1e-5)[0]
+
+
+def test_no_transfers_negative_control_and_barrier_mode():
+    u = synth.jacobi_grid(128, 128)
+    g1, _ = _jacobi(u, 6, 1)
+    gb, _ = _jacobi(u, 6, 2, abi.PK_MODE_NO_TRANSFERS)
+    assert not np.array_equal(g1, gb)
+    gg, _ = _jacobi(u, 6, 4, abi.PK_MODE_GLOBAL_BARRIER)
+    assert np.array_equal(g1, gg)
+    gs, ss = _jacobi(u, 6, 3, abi.PK_MODE_SINGLE_OWNER)
+    assert np.array_equal(g1, gs)
+
+
+# ------------------------------------------------------------------ C2 Hotspot
+def _hotspot(t, p, iters, P, ty=16, bdx=128, mode=0):
+    ctx = gpu_ctx(P, mode)
+    pr = K.hotspot2d_setup(ctx, t, p, ty, bdx)
+    out = K.hotspot2d_iterate(pr, iters)
+    res = fetch(ctx, out, t.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st
+
+
+@pytest.mark.parametrize("h,w,ty,bdx", [(200, 520, 16, 128), (64, 64, 4, 32), (129, 1028, 64, 128)])
+def test_hotspot_oracle_and_bitwise(h, w, ty, bdx):
+    t, p = synth.hotspot_grids(h, w)
+    iters = 20
+    ref = ok.hotspot2d(t, p, iters)
+    g1, _ = _hotspot(t, p, iters, 1, ty, bdx)
+    assert rel_ok(g1, ref, 1e-5)[0]
+    for P in (2, 3, 4, 8):
+        gp, st = _hotspot(t, p, iters, P, ty, bdx)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def test_hotspot_stale_bytes_closed_form():
+    h = w = 1024
+    t, p = synth.hotspot_grids(h, w)
+    for P in (2, 4, 8):
+        _, st = _hotspot(t, p, 10, P, 64, 128)
+        assert st["stale_bytes"] == 10 * cf.hotspot2d_stale_per_iter(w, P) == st["moved_bytes"]
+
+
+def test_hotspot_uniform_closed_form_on_gpu():
+    h, w = 96, 256
+    t = np.full((h, w), 323.0, np.float32)
+    p = np.full((h, w), 0.004, np.float32)
+    g, _ = _hotspot(t, p, 25, 3)
+    exp = cf.hotspot_uniform(323.0, 0.004, 25, ok.HOTSPOT_CAP, ok.HOTSPOT_RZ1, ok.HOTSPOT_AMB)
+    assert np.all(np.abs(g - exp) <= 1e-5 * exp)
+
+
+# ------------------------------------------------------------------ C3 Heat
+def _heat(u, iters, P, zc=8, bdy=8):
+    ctx = gpu_ctx(P)
+    pr = K.heat3d_setup(ctx, u, zc, bdy)
+    out = K.heat3d_iterate(pr, iters)
+    res = fetch(ctx, out, u.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st
+
+
+@pytest.mark.parametrize("d,h,w,zc", [(40, 36, 132, 8), (17, 9, 256, 4), (64, 64, 64, 64)])
+def test_heat_oracle_and_bitwise(d, h, w, zc):
+    u = synth.heat_grid(d, h, w)
+    iters = 10
+    ref = ok.heat3d(u, iters)
+    g1, _ = _heat(u, iters, 1, zc)
+    assert rel_ok(g1, ref, 1e-5)[0]
+    for P in (2, 3, 5):
+        gp, st = _heat(u, iters, P, zc)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def test_heat_conservation_on_gpu():
+    u = synth.heat_grid(32, 32, 64)
+    g, st = _heat(u, 20, 4)
+    assert abs(float(g.astype(np.float64).sum()) - float(u.astype(np.float64).sum())) < 1e-5 * u.size
+    assert st["stale_bytes"] == 20 * cf.heat3d_stale_per_iter(32, 64, 4)
+
+
+# ------------------------------------------------------------------ C5 N-body
+def _nbody(pos, vel, steps, P, bdx=256):
+    ctx = gpu_ctx(P)
+    pr = K.nbody_setup(ctx, pos, vel, bdx)
+    pb, vb = K.nbody_iterate(pr, steps)
+    p_out = fetch(ctx, pb, pos.shape)
+    v_out = fetch(ctx, vb, vel.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return p_out, v_out, st
+
+
+@pytest.mark.parametrize("n", [3000, 1024, 4097])
+def test_nbody_oracle_and_bitwise(n):
+    pos, vel = synth.nbody_bodies(n)
+    steps = 3
+    rp, rv = ok.nbody(pos, vel, steps)
+    p1, v1, _ = _nbody(pos, vel, steps, 1)
+    assert rel_ok(v1[:, :3], rv[:, :3], 1e-5)[0]
+    assert rel_ok(p1[:, :3], rp[:, :3], 1e-5)[0]
+    for P in (2, 3, 8):
+        pp, vp, st = _nbody(pos, vel, steps, P)
+        assert np.array_equal(p1, pp) and np.array_equal(v1, vp)
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def test_nbody_two_bodies_and_momentum():
+    pos = np.array([[0.1, -0.2, 0.3, 0.5], [0.4, 0.2, -0.1, 0.25]], np.float32)
+    vel = np.zeros_like(pos)
+    _, v, _ = _nbody(pos, vel, 1, 1)
+    a0 = cf.nbody_two_body_accel(pos[0, :3], pos[1, :3], 0.25, ok.NBODY_EPS2)
+    assert np.allclose(v[0, :3], a0 * ok.NBODY_DT, rtol=1e-5)
+    rpos, rvel = synth.nbody_bodies(2048)
+    _, v, _ = _nbody(rpos, rvel, 1, 2)
+    mom = (rpos[:, 3:4].astype(np.float64) * v[:, :3]).sum(axis=0)
+    assert np.max(np.abs(mom)) < 1e-5 * np.max(np.abs(v[:, :3]))
+
+
+# ------------------------------------------------------------------ generic path
+def test_generic_register_kernel_with_python_descriptors_matches_builtin():
+    """pk_register_kernel(pk_builtin_fn) + descriptors declared through the binding
+    (the paper's flow: kernel model record + per-argument maps)."""
+    n = 200
+    u = synth.jacobi_grid(n, n)
+    ref, _ = _jacobi(u, 5, 1)
+    ctx = gpu_ctx(3)
+    fn = abi.pk_builtin_fn("jacobi2d")
+    assert fn
+    k = abi.pk_register_kernel(ctx, "jacobi_user", fn, [abi.PK_ARG_BUFFER, abi.PK_ARG_BUFFER,
+                                                        abi.PK_ARG_SCALAR, abi.PK_ARG_SCALAR])
+    H = abi.expr(-1, scalars={0: 1})
+    W = abi.expr(-1, scalars={1: 1})
+    bdx, bdy = abi.expr(0, blockdim={0: 1}), abi.expr(0, blockdim={1: 1})
+    for di, dj in ((-1, 0), (1, 0), (0, -1), (0, 1)):
+        abi.pk_declare_affine_access(ctx, k, 0, abi.PK_READ, abi.affine_access([
+            abi.dim_map(1, bdy, bdy, di, guard=(1, H)), abi.dim_map(0, bdx, bdx, dj, guard=(1, W))]))
+    abi.pk_declare_affine_access(ctx, k, 1, abi.PK_WRITE, abi.affine_access([
+        abi.dim_map(1, bdy, bdy, 0, guard=(1, H)), abi.dim_map(0, bdx, bdx, 0, guard=(1, W))]))
+    b0 = abi.pk_register_buffer(ctx, (n, n), 4, host_init=u)
+    b1 = abi.pk_register_buffer(ctx, (n, n), 4, host_init=u)
+    grid, blk, sc = K.jacobi2d_launch(n, n)
+    for t in range(5):
+        a, b = (b0, b1) if t % 2 == 0 else (b1, b0)
+        abi.pk_launch_partitioned(ctx, k, grid, blk, [a, b, n, n], sc)
+    g = fetch(ctx, b1, (n, n))
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, ref)
+
+
+def test_caller_owned_torch_instances_and_timer():
+    import torch
+    h, w = 256, 512
+    t, p = synth.hotspot_grids(h, w)
+    ref, _ = _hotspot(t, p, 8, 1)
+    P = 2
+    tens = [[torch.empty((h, w), dtype=torch.float32, device="cuda:0") for _ in range(P)] for _ in range(3)]
+    ctx = gpu_ctx(P)
+    pr = K.hotspot2d_setup(ctx, t, p, dev_ptrs=[[x.data_ptr() for x in b] for b in tens])
+    abi.pk_timer_begin(ctx)
+    out = K.hotspot2d_iterate(pr, 8)
+    ms = abi.pk_timer_end(ctx)
+    assert ms > 0
+    g = fetch(ctx, out, (h, w))
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, ref)
+    # partition 0's instance holds its own rows of the result
+    torch.cuda.synchronize()
+    assert np.array_equal(tens[0][0][: h // 2].cpu().numpy(), ref[: h // 2])

@@ -1,0 +1,383 @@
+"""Host core of libpk.so (region analyzer, validity tracker, transfer planner) vs the
+oracle, bit-exact, on CPU (contexts created with PK_INIT_HOST_ONLY: no CUDA call).
+
+  - pk_enumerate == brute-force thread programs (oracle/regions.py) for every
+    builtin kernel, ragged shapes, several block geometries and P
+  - pk_enumerate == brute-force descriptor evaluation (oracle/descriptors.py) for
+    random descriptors (hypothesis)
+  - Eq. 1-4: the library's union of taps is the exact 27-point U,
+    not the 28-point row-wise first/last over-approximation
+  - launch sequences: stale bytes, copy plans and tracker dumps == shadow oracle
+    (c3), and == the closed forms (c5)
+  - error paths: WAW overlap, out of bounds, overflow, non-separable
+"""
+import numpy as np
+import pytest
+from hypothesis import given, settings, strategies as st
+
+from oracle import closed_forms as cf
+from oracle import descriptors as od
+from oracle import grid as og
+from oracle import polyhedral as poly
+from oracle import regions, shadow
+from paper_conf_icppw_matzdf20_b200 import abi
+from paper_conf_icppw_matzdf20_b200 import kernels as K
+
+HO = abi.PK_INIT_HOST_ONLY
+
+
+def host_ctx(P, mode=0):
+    ctx = abi.pk_init(P, flags=HO)
+    if mode:
+        abi.pk_set_mode(ctx, mode)
+    return ctx
+
+
+def _lib_sets(ctx, k, nargs, bufs, box, block, sc):
+    out = {}
+    for a in range(nargs):
+        if bufs[a] is None:
+            continue
+        for mode, tag in ((abi.PK_READ, "r"), (abi.PK_WRITE, "w")):
+            r = abi.pk_enumerate(ctx, k, a, mode, bufs[a], box, block, sc)
+            if r:
+                out[(a, tag)] = r
+    return out
+
+
+def _oracle_sets(acc, ebs):
+    return {key: regions.to_byte_ranges(v, ebs[key[0]]) for key, v in acc.items() if len(v)}
+
+
+# ------------------------------------------------------------ regions vs brute force
+@pytest.mark.parametrize("h,w,block", [(64, 64, (32, 8)), (37, 50, (32, 8)), (9, 70, (16, 4)), (3, 3, (32, 8))])
+@pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
+def test_jacobi_regions(h, w, block, P):
+    ctx = host_ctx(P)
+    k = abi.pk_builtin_kernel(ctx, "jacobi2d")
+    b0 = abi.pk_register_buffer(ctx, (h, w), 4)
+    b1 = abi.pk_register_buffer(ctx, (h, w), 4)
+    grid, blk, sc = K.jacobi2d_launch(h, w, block + (1,))
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, k, grid, p)
+        assert box == og.partition_box(grid, P, p)
+        lib = _lib_sets(ctx, k, 4, [b0, b1, None, None], box, blk, sc)
+        ora = _oracle_sets(regions.jacobi2d(box, blk, h, w), {0: 4, 1: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
+@pytest.mark.parametrize("h,w,ty,bdx", [(64, 64, 4, 32), (100, 36, 16, 32), (33, 520, 4, 128), (5, 4, 64, 128)])
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 7])
+def test_hotspot_regions(h, w, ty, bdx, P):
+    ctx = host_ctx(P)
+    k = abi.pk_builtin_kernel(ctx, "hotspot2d")
+    bufs = [abi.pk_register_buffer(ctx, (h, w), 4) for _ in range(3)]
+    grid, blk, sc = K.hotspot2d_launch(h, w, ty, bdx)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, k, grid, p)
+        lib = _lib_sets(ctx, k, 6, bufs + [None] * 3, box, blk, sc)
+        ora = _oracle_sets(regions.hotspot2d(box, blk, h, w, ty), {0: 4, 1: 4, 2: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
+@pytest.mark.parametrize("d,h,w,zc,bdy", [(16, 8, 32, 3, 4), (10, 9, 132, 8, 8), (1, 1, 4, 64, 8)])
+@pytest.mark.parametrize("P", [1, 2, 3, 6])
+def test_heat_regions(d, h, w, zc, bdy, P):
+    ctx = host_ctx(P)
+    k = abi.pk_builtin_kernel(ctx, "heat3d")
+    bufs = [abi.pk_register_buffer(ctx, (d, h, w), 4) for _ in range(2)]
+    grid, blk, sc = K.heat3d_launch(d, h, w, zc, bdy)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, k, grid, p)
+        lib = _lib_sets(ctx, k, 6, bufs + [None] * 4, box, blk, sc)
+        ora = _oracle_sets(regions.heat3d(box, blk, d, h, w, zc), {0: 4, 1: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
+@pytest.mark.parametrize("n,bdx", [(300, 64), (1024, 256), (1, 32), (5000, 128)])
+@pytest.mark.parametrize("P", [1, 2, 3, 8])
+def test_nbody_regions(n, bdx, P):
+    ctx = host_ctx(P)
+    k = abi.pk_builtin_kernel(ctx, "nbody")
+    bufs = [abi.pk_register_buffer(ctx, (n,), 16) for _ in range(3)]
+    grid, blk, sc = K.nbody_launch(n, bdx)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, k, grid, p)
+        lib = _lib_sets(ctx, k, 4, bufs + [None], box, blk, sc)
+        ora = _oracle_sets(regions.nbody(box, blk, n, K.NBODY_PER_THREAD), {0: 16, 1: 16, 2: 16})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
+# ------------------------------------------------------------ Eq. 1-4 through the library
+def _point_taps():
+    """S1 as one tap per row y: {y} x [y, 4]; S2 = M(S1)."""
+    s1, s2 = [], []
+    for y in range(5):
+        for (dy, dx), out in (((0, 0), s1), ((1, 3), s2)):
+            out.append([{"grid_dim": -1, "scale": 0, "extent": 1, "offset": y + dy, "clamp": False, "guard": None},
+                        {"grid_dim": -1, "scale": 0, "extent": 5 - y, "offset": y + dx, "clamp": False, "guard": None}])
+    return s1, s2
+
+
+def _to_abi(tap):
+    return abi.affine_access([abi.dim_map(d["grid_dim"], d["scale"], d["extent"], d["offset"], d["clamp"],
+                                          d["guard"]) for d in tap])
+
+
+def test_eq1_4_union_is_exact_through_library():
+    ctx = host_ctx(1)
+    k = abi.pk_register_kernel(ctx, "eq1_4", None, [abi.PK_ARG_BUFFER])
+    buf = abi.pk_register_buffer(ctx, (8, 8), 1)
+    s1, s2 = _point_taps()
+    for t in s1 + s2:
+        abi.pk_declare_affine_access(ctx, k, 0, abi.PK_READ, _to_abi(t))
+    rng = abi.pk_enumerate(ctx, k, 0, abi.PK_READ, buf, (0, 1, 0, 1, 0, 1), (1, 1, 1))
+    pts = {(b // 8, b % 8) for (lo, hi) in rng for b in range(lo, hi)}
+    assert pts == poly.U()
+    assert len(pts) == 27                                   # not 28: row y = 4 is [4,4] u [6,7]
+    assert (4, 5) not in pts
+    # the descriptor brute force agrees (pins oracle/descriptors.py by Eq. 1-4)
+    el = od.union_elements(s1 + s2, (0, 1, 0, 1, 0, 1), (8, 8))
+    assert {(e // 8, e % 8) for e in el} == poly.U()
+    abi.pk_finalize(ctx)
+
+
+# ------------------------------------------------------------ random descriptors
+@st.composite
+def _descr(draw):
+    ndim = draw(st.integers(1, 3))
+    shape = tuple(draw(st.integers(1, 9)) for _ in range(ndim))
+    grid_dims = draw(st.permutations([0, 1, 2]))
+    taps = []
+    for _ in range(draw(st.integers(1, 3))):
+        tap = []
+        for k in range(ndim):
+            use = draw(st.booleans())
+            g = grid_dims[k] if use else -1
+            scale = draw(st.integers(0, 4))
+            extent = draw(st.integers(0, 5))
+            clamp = draw(st.booleans())
+            guard = None
+            if draw(st.booleans()):
+                lo = draw(st.integers(-2, 6))
+                guard = (lo, lo + draw(st.integers(0, 8)))
+            off = draw(st.integers(-3, 3)) if clamp else 0
+            tap.append({"grid_dim": g, "scale": scale, "extent": extent, "offset": off, "clamp": clamp,
+                        "guard": guard if clamp else None})
+        taps.append(tap)
+    gridv = tuple(draw(st.integers(1, 4)) for _ in range(3))
+    P = draw(st.integers(1, 4))
+    eb = draw(st.sampled_from([1, 4, 16]))
+    return shape, taps, gridv, P, eb
+
+
+@settings(max_examples=150, deadline=None)
+@given(_descr())
+def test_random_descriptors_match_brute_force(case):
+    shape, taps, gridv, P, eb = case
+    ctx = host_ctx(P)
+    k = abi.pk_register_kernel(ctx, "rand", None, [abi.PK_ARG_BUFFER])
+    buf = abi.pk_register_buffer(ctx, shape, eb)
+    for t in taps:
+        abi.pk_declare_affine_access(ctx, k, 0, abi.PK_READ, _to_abi(t))
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, k, gridv, p)
+        try:
+            exp = regions.to_byte_ranges(od.union_elements(taps, box, shape), eb)
+        except od.OutOfBounds:
+            with pytest.raises(abi.PkError) as ei:
+                abi.pk_enumerate(ctx, k, 0, abi.PK_READ, buf, box, (1, 1, 1))
+            assert ei.value.name == "PK_ERR_OUT_OF_BOUNDS"
+            continue
+        assert abi.pk_enumerate(ctx, k, 0, abi.PK_READ, buf, box, (1, 1, 1)) == exp
+    abi.pk_finalize(ctx)
+
+
+# ------------------------------------------------------------ launch sequences vs shadow
+def _norm_plan(plan, names):
+    out = {}
+    for (b, s, d, lo, hi) in plan:
+        out.setdefault((names[b], s, d), []).append((lo, hi))
+    res = {}
+    for key, rs in out.items():
+        rs.sort()
+        m = []
+        for lo, hi in rs:
+            if m and lo <= m[-1][1]:
+                m[-1] = (m[-1][0], max(hi, m[-1][1]))
+            else:
+                m.append((lo, hi))
+        res[key] = m
+    return res
+
+
+def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0):
+    """specs: {name: (shape, eb, uploaded)}; launches: list of [arg binding names or None];
+    thread_prog(box) -> oracle access dict keyed by (arg, 'r'/'w')."""
+    ctx = host_ctx(P, mode)
+    sh = shadow.Shadow(P, single_owner=bool(mode & abi.PK_MODE_SINGLE_OWNER))
+    k = abi.pk_builtin_kernel(ctx, kernel)
+    ids, names = {}, {}
+    for name, (shape, eb, up) in specs.items():
+        host = np.zeros(int(np.prod(shape)) * eb // 4, dtype=np.float32) if up else None
+        ids[name] = abi.pk_register_buffer(ctx, shape, eb, host_init=host)
+        names[ids[name]] = name
+        sh.register(name, int(np.prod(shape)), eb, up)
+    grid, blk, sc = geom
+    stale_prev = 0
+    for binding in launches:
+        args = [ids[n] if isinstance(n, str) else n for n in binding]
+        abi.pk_launch_partitioned(ctx, k, grid, blk, args, sc)
+        per = []
+        for p in range(P):
+            box = og.partition_box(grid, P, p)
+            if og.box_empty(box):
+                per.append(None)
+                continue
+            acc = thread_prog(box)
+            d = {}
+            for (a, tag), el in acc.items():
+                name = binding[a]
+                r, w = d.get(name, (np.zeros(0, np.int64), np.zeros(0, np.int64)))
+                if tag == "r":
+                    r = np.union1d(r, el)
+                else:
+                    w = np.union1d(w, el)
+                d[name] = (r, w)
+            per.append(d)
+        res = sh.launch(per)
+        st_ = abi.pk_get_stats(ctx)
+        assert st_["stale_bytes"] - stale_prev == sum(res["stale"])
+        stale_prev = st_["stale_bytes"]
+        exp_plan = {key: regions.to_byte_ranges(el, specs[key[0]][1]) for key, el in res["copies"].items()}
+        assert _norm_plan(abi.pk_last_plan(ctx), names) == exp_plan
+        for name, bid in ids.items():
+            assert abi.pk_tracker_dump(ctx, bid) == sh.buffers[name].rle()
+    st_ = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return st_, sh
+
+
+def _jacobi_case(n, P, iters, mode=0):
+    geom = K.jacobi2d_launch(n, n)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), n, n] for t in range(iters)]
+    return _run_pair(P, "jacobi2d", {"u0": ((n, n), 4, True), "u1": ((n, n), 4, True)}, launches, geom,
+                     lambda box: regions.jacobi2d(box, geom[1], n, n), mode)
+
+
+def test_c1_sequence_40800_bytes():
+    st_, _ = _jacobi_case(512, 2, 10)
+    assert st_["stale_bytes"] == 40800 == 10 * cf.jacobi2d_stale_per_iter(512, 2)
+    assert st_["launches"] == 10 and st_["kernel_launches"] == 20
+
+
+@pytest.mark.parametrize("mode", [0, abi.PK_MODE_SINGLE_OWNER])
+def test_c1_misaligned_p3_both_tracker_modes(mode):
+    _jacobi_case(64, 3, 6, mode)
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+def test_hotspot_sequence(P):
+    h = w = 64
+    geom = K.hotspot2d_launch(h, w, 4, 32)
+    launches = [[("t0" if t % 2 == 0 else "t1"), "pw", ("t1" if t % 2 == 0 else "t0"), h, w, 4] for t in range(5)]
+    st_, sh = _run_pair(P, "hotspot2d", {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False),
+                                         "pw": ((h, w), 4, True)}, launches, geom,
+                        lambda box: regions.hotspot2d(box, geom[1], h, w, 4))
+    # every iteration moves exactly the halo rows when the linear upload of t0 is
+    # row-aligned with the partitions (P | 16 blocks); otherwise launch 1 also redistributes
+    if 16 % P == 0:
+        assert st_["stale_bytes"] == 5 * cf.hotspot2d_stale_per_iter(w, P)
+    else:
+        assert st_["stale_bytes"] > 5 * cf.hotspot2d_stale_per_iter(w, P)
+    assert len(sh.buffers["t0"].rle()) <= 2 * P - 1
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_heat_sequence(P):
+    d, h, w = 12, 8, 64
+    geom = K.heat3d_launch(d, h, w, 2, 4)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), d, h, w, 2] for t in range(4)]
+    _run_pair(P, "heat3d", {"u0": ((d, h, w), 4, True), "u1": ((d, h, w), 4, False)}, launches, geom,
+              lambda box: regions.heat3d(box, geom[1], d, h, w, 2))
+
+
+@pytest.mark.parametrize("mode", [0, abi.PK_MODE_SINGLE_OWNER])
+def test_nbody_sequence(mode):
+    n, P = 1024, 8
+    geom = K.nbody_launch(n, 64)
+    launches = [[("p0" if s % 2 == 0 else "p1"), "v", ("p1" if s % 2 == 0 else "p0"), n] for s in range(3)]
+    st_, _ = _run_pair(P, "nbody", {"p0": ((n,), 16, True), "p1": ((n,), 16, False), "v": ((n,), 16, True)},
+                       launches, geom, lambda box: regions.nbody(box, geom[1], n, K.NBODY_PER_THREAD), mode)
+    assert st_["stale_bytes"] == 3 * cf.nbody_stale_per_step(n, P)
+
+
+# ------------------------------------------------------------ error paths / modes
+def test_write_overlap_rejected_before_anything():
+    ctx = host_ctx(2)
+    k = abi.pk_register_kernel(ctx, "bad", None, [abi.PK_ARG_BUFFER])
+    buf = abi.pk_register_buffer(ctx, (64,), 4)
+    # every block writes [b*8, b*8+12): blocks overlap -> partitions overlap
+    abi.pk_declare_affine_access(ctx, k, 0, abi.PK_WRITE, abi.affine_access([abi.dim_map(0, 8, 12, guard=(0, 64))]))
+    before = abi.pk_tracker_dump(ctx, buf)
+    with pytest.raises(abi.PkError) as ei:
+        abi.pk_launch_partitioned(ctx, k, (8, 1, 1), (1, 1, 1), [buf])
+    assert ei.value.name == "PK_ERR_WRITE_OVERLAP"
+    assert abi.pk_tracker_dump(ctx, buf) == before
+    assert abi.pk_get_stats(ctx)["launches"] == 0
+    abi.pk_finalize(ctx)
+
+
+def test_out_of_bounds_overflow_and_non_separable():
+    ctx = host_ctx(1)
+    k = abi.pk_register_kernel(ctx, "oob", None, [abi.PK_ARG_BUFFER])
+    buf = abi.pk_register_buffer(ctx, (10,), 4)
+    abi.pk_declare_affine_access(ctx, k, 0, abi.PK_READ, abi.affine_access([abi.dim_map(0, 4, 4, offset=1)]))
+    with pytest.raises(abi.PkError) as ei:
+        abi.pk_launch_partitioned(ctx, k, (3, 1, 1), (1, 1, 1), [buf])
+    assert ei.value.name == "PK_ERR_OUT_OF_BOUNDS"
+    k2 = abi.pk_register_kernel(ctx, "ovf", None, [abi.PK_ARG_BUFFER])
+    abi.pk_declare_affine_access(ctx, k2, 0, abi.PK_READ,
+                                 abi.affine_access([abi.dim_map(0, abi.expr(1 << 62), 4, clamp=True)]))
+    with pytest.raises(abi.PkError) as ei:
+        abi.pk_launch_partitioned(ctx, k2, (3, 1, 1), (1, 1, 1), [buf])
+    assert ei.value.name == "PK_ERR_OVERFLOW"
+    k3 = abi.pk_register_kernel(ctx, "nonsep", None, [abi.PK_ARG_BUFFER])
+    b2 = abi.pk_register_buffer(ctx, (4, 4), 4)
+    with pytest.raises(abi.PkError) as ei:
+        abi.pk_declare_affine_access(ctx, k3, 0, abi.PK_READ,
+                                     abi.affine_access([abi.dim_map(0, 1, 1), abi.dim_map(0, 1, 1)]))
+    assert ei.value.name == "PK_ERR_INVALID"
+    del b2
+    abi.pk_finalize(ctx)
+
+
+def test_no_tracking_and_no_transfers_modes():
+    # gamma: no resolution, no tracker -> no stale bytes counted, tracker untouched
+    n = 64
+    ctx = host_ctx(2, abi.PK_MODE_NO_TRACKING)
+    pr, _ = K.jacobi2d_program(ctx, np.zeros((n, n), np.float32), 4)
+    s = abi.pk_get_stats(ctx)
+    assert s["stale_bytes"] == 0 and s["launches"] == 4
+    abi.pk_finalize(ctx)
+    # beta: resolution + tracking still run
+    ctx = host_ctx(2, abi.PK_MODE_NO_TRANSFERS)
+    K.jacobi2d_program(ctx, np.zeros((n, n), np.float32), 4)
+    s = abi.pk_get_stats(ctx)
+    assert s["stale_bytes"] == 4 * cf.jacobi2d_stale_per_iter(n, 2) and s["moved_bytes"] == 0
+    abi.pk_finalize(ctx)
+
+
+def test_h2d_linear_distribution_tracker():
+    ctx = host_ctx(3)
+    b = abi.pk_register_buffer(ctx, (10,), 4, host_init=np.zeros(10, np.float32))
+    sb = shadow.ShadowBuffer(10, 4, 3)
+    sb.h2d_linear()
+    assert abi.pk_tracker_dump(ctx, b) == sb.rle()
+    b2 = abi.pk_register_buffer(ctx, (7, 3), 4)
+    assert abi.pk_tracker_dump(ctx, b2) == [(0, 84, 7)]           # reading Q3
+    abi.pk_finalize(ctx)

@@ -65,9 +65,11 @@ def test_hotspot_heat_nbody_gemm_sets_shape():
     assert regions.to_byte_ranges(acc[(0, "r")], 1) == [(2 * 256, 7 * 256)]
     assert regions.to_byte_ranges(acc[(1, "w")], 1) == [(3 * 256, 6 * 256)]
     # nbody: everything read, own slab written
-    acc = regions.nbody((0, 1, 0, 1, 2, 3), (64,), 300)
+    acc = regions.nbody((0, 1, 0, 1, 1, 2), (64,), 300)      # 2 bodies per thread
     assert regions.to_byte_ranges(acc[(0, "r")], 16) == [(0, 300 * 16)]
-    assert regions.to_byte_ranges(acc[(2, "w")], 16) == [(128 * 16, 192 * 16)]
+    assert regions.to_byte_ranges(acc[(2, "w")], 16) == [(128 * 16, 256 * 16)]
+    acc = regions.nbody((0, 1, 0, 1, 2, 3), (64,), 300)      # ragged last block
+    assert regions.to_byte_ranges(acc[(1, "w")], 16) == [(256 * 16, 300 * 16)]
     # gemm: A row band, B whole, C tile rows
     acc = regions.gemm((0, 1, 1, 2, 0, 2), 10, 12, 5, 4, 8)
     assert regions.to_byte_ranges(acc[(0, "r")], 1) == [(20, 40)]
@@ -141,7 +143,7 @@ def test_nbody_allgather_and_validity_vs_single_owner():
     sh.register("p0", n, 16, True)
     sh.register("p1", n, 16, False)
     sh.register("v", n, 16, True)
-    g = (n // 64, 1, 1)
+    g = (n // 128, 1, 1)
     tot = 0
     for s in range(3):
         a, b = ("p0", "p1") if s % 2 == 0 else ("p1", "p0")
