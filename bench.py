@@ -43,6 +43,7 @@ WORKLOADS = {
     "heat3d": ("C3 3D 7-point heat stencil 1024^3 fp32, 50 iterations/step", 50),
     "jacobi2d": ("C1 2D 5-point Jacobi 512x512 fp32, 10 iterations/step", 10),
     "nbody": ("C5 all-pairs N-body 2^20 bodies fp32, 10 steps/step", 10),
+    "sgemm": ("C4 dense SGEMM 16384^3 fp32 (3xTF32 on tcgen05), 1 launch/step", 1),
 }
 
 
@@ -165,17 +166,29 @@ class Workload:
             self.units_per_iter = n * n
             self.bytes_per_unit = 0
             self.unit, self.metric = "Ginteractions/s", "nbody_ginteractions"
+        elif name == "sgemm":
+            m = n = k = 16384
+            self.shape = (m, n, k)
+            self.host = synth.gemm_operands(m, n, k)
+            self.units_per_iter = 2 * m * n * k          # FP32-equivalent flops
+            self.bytes_per_unit = 0
+            self.scale = 1e12
+            self.unit, self.metric = "TFLOP/s", "sgemm_fp32_equiv_tflops"
         else:
             raise SystemExit(f"unknown workload {name}")
+        self.scale = getattr(self, "scale", 1e9)
 
     def setup(self, ctx):
         K = self.K
         if self.name == "hotspot2d":
-            self.pr = K.hotspot2d_setup(ctx, *self.host)
+            self.pr = K.hotspot2d_setup(ctx, *self.host, kernel=getattr(self, "variant", None) or "hotspot2d")
             self.upload_bufs = [(self.pr.tb[0], self.host[0]), (self.pr.tb[2], self.host[1])]
         elif self.name == "heat3d":
-            self.pr = K.heat3d_setup(ctx, self.host[0])
+            self.pr = K.heat3d_setup(ctx, self.host[0], kernel=getattr(self, "variant", None) or "heat3d")
             self.upload_bufs = [(self.pr.ub[0], self.host[0])]
+        elif self.name == "sgemm":
+            self.pr, _ = K.sgemm_program(ctx, *self.host, launches=0)
+            self.upload_bufs = [(self.pr.abc[0], self.host[0]), (self.pr.abc[1], self.host[1])]
         elif self.name == "jacobi2d":
             self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0)
             self.upload_bufs = [(b, self.host[0]) for b in self.pr.bufs]
@@ -198,12 +211,21 @@ class Workload:
                 a, b = (b0, b1) if t % 2 == 0 else (b1, b0)
                 pr.launch(grid, blk, [a, b, h, w], sc)
             out = b1 if (self.t + self.iters) % 2 == 1 else b0
+        elif self.name == "sgemm":
+            grid, blk, sc = pr.geom
+            a, b, c = pr.abc
+            m, n, k = pr.mnk
+            for _ in range(self.iters):
+                pr.launch(grid, blk, [a, b, c, m, n, k], sc)
+            out = c
         else:
             out, _ = K.nbody_iterate(pr, self.iters, self.t)
         self.t += self.iters
         return out
 
     def out_shape(self):
+        if self.name == "sgemm":
+            return (self.shape[0], self.shape[1])
         return (self.shape[0], 4) if self.name == "nbody" else self.shape
 
     def stale_min(self, P):
@@ -212,11 +234,12 @@ class Workload:
             "heat3d": lambda: 2 * self.shape[1] * self.shape[2] * 4 * (P - 1),
             "jacobi2d": lambda: 2 * (self.shape[1] - 2) * 4 * (P - 1),
             "nbody": lambda: self.shape[0] * 16 * (P - 1),
+            "sgemm": lambda: 0,   # B moves once (first launch): (P-1) K N 4 B, reported by the stats
         }
         return from_cf[self.name]() * self.iters
 
 
-def cpu_oracle_rate(w: Workload, budget_s=10.0, max_iters=50):
+def cpu_oracle_rate(w: Workload, budget_s=10.0, max_iters=1000):
     """Time the oracle as it stands on a bounded sample of the same workload."""
     import ctypes
     from oracle import kernels as ok
@@ -315,6 +338,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "pk":
         print("warning: fewer than 3 warm-up steps", file=sys.stderr)
@@ -325,6 +349,7 @@ def main():
         import torch.distributed as dist
         dist.init_process_group("gloo")
     w = Workload(args.workload, args.iters or WORKLOADS[args.workload][1])
+    w.variant = args.variant
 
     if args.impl == "reference":
         line = run_reference(args, w, rank)
@@ -378,12 +403,21 @@ def main():
         return
 
     units = w.units_per_iter * w.iters * args.steps
-    value = units / (elapsed_ms / 1e3) / 1e9
+    value = units / (elapsed_ms / 1e3) / w.scale
     peaks = load_peaks()
     kname = w.name
     avg_kernel_ms = st["kernel_ms"] / max(1, st["timed_kernels"])
     per_launch_units = w.units_per_iter / P
-    if w.name == "nbody":
+    if w.name == "sgemm":
+        # tensor bound: 3 TF32 MMAs per FP32-equivalent product; TF32 peak = measured bf16 x (1.1/2.25)
+        bf16 = (peaks or {}).get("bf16_tflops_sustained", 1392.4)
+        peak = bf16 * 1.1 / 2.25
+        achieved = 3 * per_launch_units / (avg_kernel_ms / 1e3) / 1e12
+        roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                    "frac": achieved / peak, "traffic": ncu_traffic(kname),
+                    "peak_source": "MEASURED_PEAKS.json bf16_tflops_sustained x 1.1/2.25 (TF32/BF16 nominal ratio); "
+                                   "achieved = 3 x 2MNK TF32 flops / (split + GEMM kernel time)"}
+    elif w.name == "nbody":
         # FP32-ALU bound: 12 FP32-pipe instructions per interaction on 128 lanes/SM
         sm_mhz = clocks.get("sm_mhz") or (peaks or {}).get("sm_max_mhz", 1965.0)
         peak = 148 * 128 / 12 * (sm_mhz * 1e6) / 1e9
@@ -433,7 +467,7 @@ def main():
             abi.pk_sync_to_host(ctx, out, out_host)
             d2h += out_host.numel() * out_host.element_size()
         el = time.perf_counter() - t0
-        result["e2e"] = {"value": w.units_per_iter * w.iters * args.e2e_steps / el / 1e9, "unit": w.unit,
+        result["e2e"] = {"value": w.units_per_iter * w.iters * args.e2e_steps / el / w.scale, "unit": w.unit,
                          "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
                          "steps": args.e2e_steps, "timing": "wall clock around pk_copy_from_host + launches + "
                                                            "pk_sync_to_host (pinned host buffers)"}

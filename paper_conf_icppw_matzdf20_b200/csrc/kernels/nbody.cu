@@ -6,14 +6,17 @@
 //   a_i = sum_j m_j d_ij (|d_ij|^2 + eps^2)^(-3/2),  d_ij = p_j - p_i,
 //   v' = v + a dt,  x' = x + v' dt  (kick-drift Euler), G = 1.
 // Positions are float4 (x, y, z, m) and ping-pong between launches; velocities
-// are updated in place (each thread reads and writes only its own body).
+// are updated in place (each thread reads and writes only its own bodies).
 //
-// FP32-ALU bound (12 FP32-pipe ops + 1 MUFU per interaction): sources are staged
-// in shared memory 256 at a time and broadcast to the warp; each thread keeps
-// two bodies to double the FMA chains per shared-memory read.  Accumulation is
-// two-level (partial sums over 1024-source chunks, then added into the total),
-// which keeps the FP32 error of a 1M-term sum near 1e-6 (reading Q16).
+// FP32-ALU / issue bound.  Sources are staged in shared memory 256 at a time,
+// pre-duplicated as (x,x,y,y) (z,z,m,m) so that two LDS.128 broadcasts yield
+// packed pairs; each thread owns 4 bodies as two f32x2 pairs and evaluates the
+// interaction with Blackwell's packed FADD2/FFMA2/FMUL2 (one instruction per two
+// bodies) + 2 MUFU.RSQ -- about 7 issued instructions per interaction instead of
+// 13+.  Accumulation is two-level (partial sums over 1024-source chunks added
+// into the total), keeping the FP32 error of a 1M-term sum near 1e-6 (Q16).
 #include <cuda_runtime.h>
+#include <stdint.h>
 
 #include "../runtime/builtins.h"
 
@@ -24,65 +27,119 @@ constexpr float kEps2 = 1e-4f;
 constexpr float kDt = 1e-3f;
 constexpr int kTile = 256;   // sources per shared-memory tile
 constexpr int kChunk = 1024; // sources per partial sum
-constexpr int kBodies = 2;   // bodies per thread
+constexpr int kBodies = 4;   // bodies per thread = 2 packed pairs
 
-// Block = kThreads threads; block b owns bodies [b*kBodies*bdx, (b+1)*kBodies*bdx):
-// thread t holds bodies base + t and base + t + bdx.
+typedef unsigned long long u64;
+
+__device__ __forceinline__ u64 pk2(float a, float b) {
+    u64 r;
+    asm("mov.b64 %0, {%1,%2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ void up2(u64 v, float& a, float& b) { asm("mov.b64 {%0,%1}, %2;" : "=f"(a), "=f"(b) : "l"(v)); }
+__device__ __forceinline__ u64 sub2(u64 a, u64 b) {
+    u64 r;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64 add2(u64 a, u64 b) {
+    u64 r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64 mul2(u64 a, u64 b) {
+    u64 r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64 fma2(u64 a, u64 b, u64 c) {
+    u64 r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
+// r2 >= eps^2 = 1e-4 is never denormal, so the flush-to-zero MUFU.RSQ is exact
+// enough and skips rsqrtf's denormal scaling (2 FMUL per call).
+__device__ __forceinline__ float rsqrt_ftz(float x) {
+    float r;
+    asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+__device__ __forceinline__ u64 rsqrt2(u64 v) {
+    float a, b;
+    up2(v, a, b);
+    return pk2(rsqrt_ftz(a), rsqrt_ftz(b));
+}
+
+// Block = bdx threads; block b owns bodies [b*4*bdx, (b+1)*4*bdx): thread t holds
+// bodies base + t + u*bdx (u = 0..3), paired as (u=0, u=1) and (u=2, u=3).
 __global__ void __launch_bounds__(256) k_nbody(const float4* __restrict__ pin, float4* __restrict__ vel,
                                                float4* __restrict__ pout, int64_t N, pk_partition part) {
-    __shared__ float4 sh[kTile];
+    __shared__ float4 sh[2 * kTile];
     const int64_t bx = part.min[0] + blockIdx.x;  // Eq. 8
     const int64_t base = bx * (int64_t)kBodies * blockDim.x;
     float4 pi[kBodies];
-    float ax[kBodies], ay[kBodies], az[kBodies];
 #pragma unroll
     for (int u = 0; u < kBodies; ++u) {
         const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
         pi[u] = i < N ? pin[i] : make_float4(0.f, 0.f, 0.f, 0.f);
-        ax[u] = ay[u] = az[u] = 0.f;
+    }
+    u64 px[2], py[2], pz[2], ax[2], ay[2], az[2];
+    const u64 zero = pk2(0.f, 0.f), eps = pk2(kEps2, kEps2);
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        px[h] = pk2(pi[2 * h].x, pi[2 * h + 1].x);
+        py[h] = pk2(pi[2 * h].y, pi[2 * h + 1].y);
+        pz[h] = pk2(pi[2 * h].z, pi[2 * h + 1].z);
+        ax[h] = ay[h] = az[h] = zero;
     }
     for (int64_t c0 = 0; c0 < N; c0 += kChunk) {
-        float px[kBodies], py[kBodies], pz[kBodies];
-#pragma unroll
-        for (int u = 0; u < kBodies; ++u) px[u] = py[u] = pz[u] = 0.f;
+        u64 sx[2] = {zero, zero}, sy[2] = {zero, zero}, sz[2] = {zero, zero};
         const int64_t c1 = c0 + kChunk < N ? c0 + kChunk : N;
         for (int64_t t0 = c0; t0 < c1; t0 += kTile) {
             __syncthreads();
             for (int s = threadIdx.x; s < kTile; s += blockDim.x) {
                 const int64_t j = t0 + s;
-                sh[s] = j < c1 ? pin[j] : make_float4(0.f, 0.f, 0.f, 0.f);  // m = 0 pads contribute 0
+                const float4 q = j < c1 ? pin[j] : make_float4(0.f, 0.f, 0.f, 0.f);  // m = 0 pads add 0
+                sh[2 * s] = make_float4(q.x, q.x, q.y, q.y);
+                sh[2 * s + 1] = make_float4(q.z, q.z, q.w, q.w);
             }
             __syncthreads();
-#pragma unroll 8
+#pragma unroll 4
             for (int s = 0; s < kTile; ++s) {
-                const float4 q = sh[s];
+                const float4 A = sh[2 * s], B = sh[2 * s + 1];
+                const u64 qx = pk2(A.x, A.y), qy = pk2(A.z, A.w), qz = pk2(B.x, B.y), qm = pk2(B.z, B.w);
 #pragma unroll
-                for (int u = 0; u < kBodies; ++u) {
-                    const float dx = q.x - pi[u].x, dy = q.y - pi[u].y, dz = q.z - pi[u].z;
-                    const float r2 = fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, kEps2)));
-                    const float inv = rsqrtf(r2);
-                    const float sc = q.w * (inv * inv * inv);
-                    px[u] = fmaf(dx, sc, px[u]);
-                    py[u] = fmaf(dy, sc, py[u]);
-                    pz[u] = fmaf(dz, sc, pz[u]);
+                for (int h = 0; h < 2; ++h) {
+                    const u64 dx = sub2(qx, px[h]), dy = sub2(qy, py[h]), dz = sub2(qz, pz[h]);
+                    const u64 r2 = fma2(dx, dx, fma2(dy, dy, fma2(dz, dz, eps)));
+                    const u64 inv = rsqrt2(r2);
+                    const u64 sc = mul2(qm, mul2(mul2(inv, inv), inv));
+                    sx[h] = fma2(dx, sc, sx[h]);
+                    sy[h] = fma2(dy, sc, sy[h]);
+                    sz[h] = fma2(dz, sc, sz[h]);
                 }
             }
         }
 #pragma unroll
-        for (int u = 0; u < kBodies; ++u) {
-            ax[u] += px[u];
-            ay[u] += py[u];
-            az[u] += pz[u];
+        for (int h = 0; h < 2; ++h) {
+            ax[h] = add2(ax[h], sx[h]);
+            ay[h] = add2(ay[h], sy[h]);
+            az[h] = add2(az[h], sz[h]);
         }
     }
 #pragma unroll
     for (int u = 0; u < kBodies; ++u) {
         const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
         if (i >= N) continue;
+        float a0, a1, b0, b1, c0_, c1_;
+        up2(ax[u / 2], a0, a1);
+        up2(ay[u / 2], b0, b1);
+        up2(az[u / 2], c0_, c1_);
+        const float axu = (u & 1) ? a1 : a0, ayu = (u & 1) ? b1 : b0, azu = (u & 1) ? c1_ : c0_;
         float4 v = vel[i];
-        v.x = fmaf(ax[u], kDt, v.x);
-        v.y = fmaf(ay[u], kDt, v.y);
-        v.z = fmaf(az[u], kDt, v.z);
+        v.x = fmaf(axu, kDt, v.x);
+        v.y = fmaf(ayu, kDt, v.y);
+        v.z = fmaf(azu, kDt, v.z);
         vel[i] = v;
         pout[i] = make_float4(fmaf(v.x, kDt, pi[u].x), fmaf(v.y, kDt, pi[u].y), fmaf(v.z, kDt, pi[u].z), pi[u].w);
     }
@@ -90,7 +147,7 @@ __global__ void __launch_bounds__(256) k_nbody(const float4* __restrict__ pin, f
 
 int describe_nbody(pk_ctx c, pk_kernel k) {
     // scalars: 0 = N.  Buffers are [N] float4 bodies.  Block b owns bodies
-    // [b*2*bdx, (b+1)*2*bdx) n [0, N); it reads every body of pos_in.
+    // [b*4*bdx, (b+1)*4*bdx) n [0, N); it reads every body of pos_in.
     pk_affine_access all{};
     all.ndim = 1;
     all.dim[0] = DimMap(-1, E(0), S(0), E(0), 0);

@@ -180,38 +180,58 @@ __device__ __forceinline__ Pl4 load_pl(const float* __restrict__ u, int64_t off,
     return x;
 }
 
-// Block = (32, bdy): warp ty owns row i = by*bdy + ty, 128 columns
-// j0 = bx*128 + 4*tx, and marches the ZC planes [bz*ZC, bz*ZC + ZC).
-__global__ void __launch_bounds__(256) k_heat3d(const float* __restrict__ uin, float* __restrict__ uout,
+// Block = (32, bdy <= kHeatMaxBdy): warp ty owns row i = by*bdy + ty, 128 columns
+// j0 = bx*128 + 4*tx, and marches the ZC planes [bz*ZC, bz*ZC + ZC).  The z
+// neighbours live in a per-thread register window; the y neighbours are the
+// adjacent warps' centre rows, exchanged through a double-buffered shared-memory
+// plane (one barrier per plane keeps the CTA's warps in lock-step, so every input
+// row is fetched from HBM once); only the two CTA-boundary halo rows are loaded
+// extra (by warps 0 and bdy-1), one plane ahead.
+constexpr int kHeatMaxBdy = 32;
+
+__global__ void __launch_bounds__(1024) k_heat3d(const float* __restrict__ uin, float* __restrict__ uout,
                                                 int64_t D, int64_t H, int64_t W, int64_t ZC, pk_partition part) {
+    __shared__ float4 ysh[2][kHeatMaxBdy + 2][32];
     const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y, bz = part.min[2] + blockIdx.z;
     const int lane = threadIdx.x;  // blockDim.x == 32
-    const int64_t i = by * blockDim.y + threadIdx.y;
+    const int ty = threadIdx.y, bdy = blockDim.y;
+    const int64_t i = by * bdy + ty;
     const int64_t j0 = bx * 128 + 4 * (int64_t)lane;
-    if (i >= H || bx * 128 >= W) return;                       // warp-uniform
     const int64_t k0 = bz * ZC;
-    if (k0 >= D) return;
+    if (bx * 128 >= W || by * bdy >= H || k0 >= D) return;     // block-uniform
     const int64_t k1 = min(k0 + ZC, D);
-    const bool active = j0 < W;
-    const int64_t jl = active ? j0 : W - 4;
+    const bool active = j0 < W && i < H;
+    const int64_t il = i < H ? i : H - 1;                       // rows past H mirror the last row
+    const int64_t jl = j0 < W ? j0 : W - 4;
     const int64_t jw = jl > 0 ? jl - 1 : 0, je = jl + 4 < W ? jl + 4 : W - 1;
     const bool west_edge = jl == 0, east_edge = jl + 4 >= W;
     const int64_t HW = H * W;
-    const int64_t rowc = i * W, rowm = (i > 0 ? i - 1 : 0) * W, rowp = (i + 1 < H ? i + 1 : H - 1) * W;
+    const int64_t rowc = il * W;
+    // CTA-boundary halo rows (clamped): warp 0 fetches row i0-1, warp bdy-1 row i0+bdy
+    const bool halo_lo = ty == 0, halo_hi = ty == bdy - 1;
+    const int64_t i0 = by * bdy;
+    const int64_t rowh = halo_lo ? (i0 > 0 ? i0 - 1 : 0) * W : (i0 + bdy < H ? i0 + bdy : H - 1) * W;
 
     Pl4 Zm = load_pl(uin, (k0 > 0 ? k0 - 1 : 0) * HW + rowc, jl, jw, je, lane);
     Pl4 Zc = load_pl(uin, k0 * HW + rowc, jl, jw, je, lane);
     Pl4 Zp = load_pl(uin, (k0 + 1 < D ? k0 + 1 : D - 1) * HW + rowc, jl, jw, je, lane);
-    float4 Ym = ld_l1(uin + k0 * HW + rowm + jl);
-    float4 Yp = ld_l1(uin + k0 * HW + rowp + jl);
+    float4 Hr = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (halo_lo || halo_hi) Hr = ld_stream4(uin + k0 * HW + rowh + jl);
+    int buf = 0;
     for (int64_t k = k0; k < k1; ++k) {
         Pl4 Zn = Zp;
-        float4 Ym2 = Ym, Yp2 = Yp;
+        float4 Hn = Hr;
         if (k + 1 < k1) {
             Zn = load_pl(uin, (k + 2 < D ? k + 2 : D - 1) * HW + rowc, jl, jw, je, lane);
-            Ym2 = ld_l1(uin + (k + 1) * HW + rowm + jl);
-            Yp2 = ld_l1(uin + (k + 1) * HW + rowp + jl);
+            if (halo_lo || halo_hi) Hn = ld_stream4(uin + (k + 1) * HW + rowh + jl);
         }
+        ysh[buf][ty + 1][lane] = Zc.c;
+        if (halo_lo) ysh[buf][0][lane] = Hr;
+        if (halo_hi) ysh[buf][bdy + 1][lane] = Hr;
+        __syncthreads();
+        const float4 Ym = ysh[buf][ty][lane];
+        const float4 Yp = ysh[buf][ty + 2][lane];
+        buf ^= 1;
         float wv = __shfl_up_sync(0xffffffffu, Zc.c.w, 1);
         float ev = __shfl_down_sync(0xffffffffu, Zc.c.x, 1);
         if (lane == 0) wv = Zc.w;
@@ -228,8 +248,7 @@ __global__ void __launch_bounds__(256) k_heat3d(const float* __restrict__ uin, f
         Zm = Zc;
         Zc = Zp;
         Zp = Zn;
-        Ym = Ym2;
-        Yp = Yp2;
+        Hr = Hn;
     }
 }
 
@@ -254,7 +273,9 @@ int describe_heat3d(pk_ctx c, pk_kernel k) {
 cudaError_t launch_heat3d(const LaunchInfo& li) {
     if (li.nscalars < 4) return cudaErrorInvalidValue;
     int64_t D = li.scalars[0], H = li.scalars[1], W = li.scalars[2], ZC = li.scalars[3];
-    if (W % 4 || W < 4 || ZC < 1 || li.block.x != 32 || li.block.z != 1) return cudaErrorInvalidValue;
+    if (W % 4 || W < 4 || ZC < 1 || li.block.x != 32 || li.block.y < 2 || li.block.y > kHeatMaxBdy ||
+        li.block.z != 1)
+        return cudaErrorInvalidValue;
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &D, &H, &W, &ZC, (void*)&li.part};
     return cudaLaunchKernel(li.fn, li.grid, li.block, argv, 0, li.stream);
 }
@@ -265,11 +286,11 @@ const Builtin kBuiltinJacobi2d = {
     "jacobi2d", (const void*)k_jacobi2d, 4,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1, describe_jacobi2d, launch_jacobi2d};
 const Builtin kBuiltinHotspot2d = {
-    "hotspot2d", (const void*)k_hotspot2d, 6,
+    "hotspot2d_regs", (const void*)k_hotspot2d, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
     describe_hotspot2d, launch_hotspot2d};
 const Builtin kBuiltinHeat3d = {
-    "heat3d", (const void*)k_heat3d, 6,
+    "heat3d_regs", (const void*)k_heat3d, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
     describe_heat3d, launch_heat3d};
 

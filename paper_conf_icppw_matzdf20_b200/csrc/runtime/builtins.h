@@ -35,12 +35,16 @@ struct Builtin {
 };
 
 const Builtin* find_builtin(const char* name);
+LauncherFn find_builtin_launcher(const void* fn);
 
 // Per-kernel-file registration (defined in kernels/*.cu)
 extern const Builtin kBuiltinJacobi2d;
-extern const Builtin kBuiltinHotspot2d;
+extern const Builtin kBuiltinHotspot2d;     // hotspot2d_regs (register window)
+extern const Builtin kBuiltinHotspot2dTma;  // hotspot2d (TMA bulk ring, default)
 extern const Builtin kBuiltinHeat3d;
+extern const Builtin kBuiltinHeat3dTma;      // heat3d (TMA plane ring, default); kBuiltinHeat3d = heat3d_regs
 extern const Builtin kBuiltinNbody;
+extern const Builtin kBuiltinSgemm;          // sgemm_tf32x3 (tcgen05 3xTF32)
 
 // Descriptor helpers used by the kernel files' describe() functions.
 inline pk_expr E(int64_t c0) {

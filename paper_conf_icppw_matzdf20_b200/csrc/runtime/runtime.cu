@@ -542,6 +542,7 @@ int pk_register_kernel(pk_ctx c, const char* name, const void* fn, int nargs, co
     Kernel k;
     k.name = name ? name : "";
     k.fn = fn;
+    k.launcher = find_builtin_launcher(fn);  // a builtin __global__ keeps its own launch geometry
     k.nargs = nargs;
     k.partition_dim = partition_dim;
     for (int i = 0; i < nargs; ++i) {
@@ -898,9 +899,19 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
 }  // extern "C"
 
 namespace pk {
+LauncherFn find_builtin_launcher(const void* fn) {
+    if (!fn) return nullptr;
+    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "heat3d", "heat3d_regs", "nbody",
+                          "sgemm_tf32x3"}) {
+        const Builtin* b = find_builtin(n);
+        if (b && b->fn == fn) return b->launcher;
+    }
+    return nullptr;
+}
 const Builtin* find_builtin(const char* name) {
     if (!name) return nullptr;
-    static const Builtin* all[] = {&kBuiltinJacobi2d, &kBuiltinHotspot2d, &kBuiltinHeat3d, &kBuiltinNbody};
+    static const Builtin* all[] = {&kBuiltinJacobi2d, &kBuiltinHotspot2dTma, &kBuiltinHotspot2d, &kBuiltinHeat3dTma,
+                                   &kBuiltinHeat3d, &kBuiltinNbody, &kBuiltinSgemm};
     for (const Builtin* b : all)
         if (std::strcmp(b->name, name) == 0) return b;
     return nullptr;

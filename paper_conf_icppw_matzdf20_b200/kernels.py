@@ -15,9 +15,9 @@ from . import abi
 
 # ---------------------------------------------------------------- geometry
 JACOBI_BLOCK = (32, 8, 1)
-HOTSPOT_BDX, HOTSPOT_TY = 128, 64
-HEAT_BDY, HEAT_ZC = 8, 64
-NBODY_BDX, NBODY_PER_THREAD = 256, 2
+HOTSPOT_BDX, HOTSPOT_TY = 128, 64     # "hotspot2d" (TMA ring) requires bdx = 128
+HEAT_BDY, HEAT_ZC = 32, 128
+NBODY_BDX, NBODY_PER_THREAD = 256, 4
 
 
 def _cdiv(a, b):
@@ -38,6 +38,31 @@ def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
 
 def nbody_launch(n, bdx=NBODY_BDX):
     return (_cdiv(n, NBODY_PER_THREAD * bdx), 1, 1), (bdx, 1, 1), [n]
+
+
+GEMM_BM, GEMM_BN = 128, 256
+
+
+def sgemm_launch(m, n, k):
+    """Logical block = one 128 x 256 C tile (the kernel runs 8 warps per tile)."""
+    return (_cdiv(n, GEMM_BN), _cdiv(m, GEMM_BM), 1), (256, 1, 1), [m, n, k]
+
+
+def sgemm_program(ctx, a_host, b_host, launches=1):
+    """C4: upload A (M x K) and B (K x N) (linear H2D), C = A B through the
+    partitioned launch; returns (problem, C buffer id)."""
+    m, k = a_host.shape
+    k2, n = b_host.shape
+    assert k == k2
+    pr = Problem(ctx, "sgemm_tf32x3")
+    a = pr.buffer((m, k), 4, host=a_host)
+    b = pr.buffer((k, n), 4, host=b_host)
+    c = pr.buffer((m, n), 4)
+    grid, blk, sc = sgemm_launch(m, n, k)
+    for _ in range(launches):
+        pr.launch(grid, blk, [a, b, c, m, n, k], sc)
+    pr.geom, pr.mnk, pr.abc = (grid, blk, sc), (m, n, k), (a, b, c)
+    return pr, c
 
 
 # ---------------------------------------------------------------- programs
@@ -72,9 +97,10 @@ def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK):
     return pr, (u0 if iters % 2 == 0 else u1)
 
 
-def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None):
+def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None,
+                    kernel="hotspot2d"):
     h, w = temp_host.shape
-    pr = Problem(ctx, "hotspot2d")
+    pr = Problem(ctx, kernel)
     t0 = pr.buffer((h, w), 4, host=temp_host, dev_ptrs=dev_ptrs[0] if dev_ptrs else None)
     t1 = pr.buffer((h, w), 4, dev_ptrs=dev_ptrs[1] if dev_ptrs else None)   # undefined (reading Q3)
     pw = pr.buffer((h, w), 4, host=power_host, dev_ptrs=dev_ptrs[2] if dev_ptrs else None)
@@ -93,9 +119,9 @@ def hotspot2d_iterate(pr, iters, start=0):
     return t1 if (start + iters) % 2 == 1 else t0
 
 
-def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY):
+def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY, kernel="heat3d"):
     d, h, w = u_host.shape
-    pr = Problem(ctx, "heat3d")
+    pr = Problem(ctx, kernel)
     u0 = pr.buffer((d, h, w), 4, host=u_host)
     u1 = pr.buffer((d, h, w), 4)
     pr.geom = heat3d_launch(d, h, w, zc, bdy)

@@ -1,0 +1,7 @@
+timeout 1200 python -m pytest tests -m gpu -q -x 2>&1 | tail -30 > gpurun_out/pytest_gpu.log
+timeout 600 python bench.py --workload heat3d --no-cpu-baseline --no-e2e > gpurun_out/bench_heat3d.log 2>&1
+timeout 600 python bench.py --workload nbody --steps 3 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_nbody.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:heat -s 5 -c 1 -o gpurun_out/prof_heat3 python bench.py --workload heat3d --steps 1 --warmup 1 --iters 4 --no-e2e --no-cpu-baseline > gpurun_out/prof_heat3.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:nbody -s 1 -c 1 -o gpurun_out/prof_nbody2 python bench.py --workload nbody --steps 1 --warmup 1 --iters 1 --no-e2e --no-cpu-baseline > gpurun_out/prof_nbody2.log 2>&1
+cat gpurun_out/pytest_gpu.log
+for f in gpurun_out/bench_heat3d.log gpurun_out/bench_nbody.log; do tail -n 1 $f | cut -c1-300; done

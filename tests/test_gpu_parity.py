@@ -15,7 +15,7 @@ from oracle import closed_forms as cf
 from oracle import kernels as ok
 from paper_conf_icppw_matzdf20_b200 import abi
 from paper_conf_icppw_matzdf20_b200 import kernels as K
-from tests.gpu_util import fetch, gpu_ctx, rel_ok
+from gpu_util import fetch, gpu_ctx, rel_ok
 
 pytestmark = pytest.mark.gpu
 
@@ -73,9 +73,9 @@ def test_no_transfers_negative_control_and_barrier_mode():
 
 
 # ------------------------------------------------------------------ C2 Hotspot
-def _hotspot(t, p, iters, P, ty=16, bdx=128, mode=0):
+def _hotspot(t, p, iters, P, ty=16, bdx=128, mode=0, kernel="hotspot2d"):
     ctx = gpu_ctx(P, mode)
-    pr = K.hotspot2d_setup(ctx, t, p, ty, bdx)
+    pr = K.hotspot2d_setup(ctx, t, p, ty, bdx, kernel=kernel)
     out = K.hotspot2d_iterate(pr, iters)
     res = fetch(ctx, out, t.shape)
     st = abi.pk_get_stats(ctx)
@@ -83,15 +83,17 @@ def _hotspot(t, p, iters, P, ty=16, bdx=128, mode=0):
     return res, st
 
 
-@pytest.mark.parametrize("h,w,ty,bdx", [(200, 520, 16, 128), (64, 64, 4, 32), (129, 1028, 64, 128)])
-def test_hotspot_oracle_and_bitwise(h, w, ty, bdx):
+@pytest.mark.parametrize("kernel,h,w,ty,bdx", [("hotspot2d", 200, 520, 16, 128), ("hotspot2d", 129, 1028, 64, 128),
+                                               ("hotspot2d", 3, 4, 64, 128), ("hotspot2d", 300, 2048, 7, 128),
+                                               ("hotspot2d_regs", 64, 64, 4, 32), ("hotspot2d_regs", 200, 520, 16, 128)])
+def test_hotspot_oracle_and_bitwise(kernel, h, w, ty, bdx):
     t, p = synth.hotspot_grids(h, w)
     iters = 20
     ref = ok.hotspot2d(t, p, iters)
-    g1, _ = _hotspot(t, p, iters, 1, ty, bdx)
+    g1, _ = _hotspot(t, p, iters, 1, ty, bdx, kernel=kernel)
     assert rel_ok(g1, ref, 1e-5)[0]
     for P in (2, 3, 4, 8):
-        gp, st = _hotspot(t, p, iters, P, ty, bdx)
+        gp, st = _hotspot(t, p, iters, P, ty, bdx, kernel=kernel)
         assert np.array_equal(g1, gp), P
         assert st["moved_bytes"] == st["stale_bytes"]
 
@@ -114,9 +116,9 @@ def test_hotspot_uniform_closed_form_on_gpu():
 
 
 # ------------------------------------------------------------------ C3 Heat
-def _heat(u, iters, P, zc=8, bdy=8):
+def _heat(u, iters, P, zc=8, bdy=8, kernel="heat3d"):
     ctx = gpu_ctx(P)
-    pr = K.heat3d_setup(ctx, u, zc, bdy)
+    pr = K.heat3d_setup(ctx, u, zc, bdy, kernel=kernel)
     out = K.heat3d_iterate(pr, iters)
     res = fetch(ctx, out, u.shape)
     st = abi.pk_get_stats(ctx)
@@ -124,15 +126,18 @@ def _heat(u, iters, P, zc=8, bdy=8):
     return res, st
 
 
-@pytest.mark.parametrize("d,h,w,zc", [(40, 36, 132, 8), (17, 9, 256, 4), (64, 64, 64, 64)])
-def test_heat_oracle_and_bitwise(d, h, w, zc):
+@pytest.mark.parametrize("kernel,d,h,w,zc,bdy", [("heat3d", 40, 36, 132, 8, 8), ("heat3d", 17, 9, 256, 4, 32),
+                                                  ("heat3d", 64, 64, 64, 64, 32), ("heat3d", 9, 70, 260, 3, 1),
+                                                  ("heat3d_regs", 40, 36, 132, 8, 8),
+                                                  ("heat3d_regs", 17, 9, 256, 4, 32)])
+def test_heat_oracle_and_bitwise(kernel, d, h, w, zc, bdy):
     u = synth.heat_grid(d, h, w)
     iters = 10
     ref = ok.heat3d(u, iters)
-    g1, _ = _heat(u, iters, 1, zc)
+    g1, _ = _heat(u, iters, 1, zc, bdy, kernel)
     assert rel_ok(g1, ref, 1e-5)[0]
     for P in (2, 3, 5):
-        gp, st = _heat(u, iters, P, zc)
+        gp, st = _heat(u, iters, P, zc, bdy, kernel)
         assert np.array_equal(g1, gp), P
         assert st["moved_bytes"] == st["stale_bytes"]
 
@@ -158,12 +163,24 @@ def _nbody(pos, vel, steps, P, bdx=256):
 
 @pytest.mark.parametrize("n", [3000, 1024, 4097])
 def test_nbody_oracle_and_bitwise(n):
+    """Per step, the oracle advances the GPU's own previous state (fp64), so fp32
+    storage rounding of positions is not compounded through close encounters
+    (SURVEY §8(c) N-body pin: per-step recomputation from the GPU state)."""
     pos, vel = synth.nbody_bodies(n)
     steps = 3
-    rp, rv = ok.nbody(pos, vel, steps)
+    ctx = gpu_ctx(2)
+    pr = K.nbody_setup(ctx, pos, vel)
+    prev_p, prev_v = pos, vel
+    for s in range(steps):
+        pb, vb = K.nbody_iterate(pr, 1, start=s)
+        gp, gv = fetch(ctx, pb, pos.shape), fetch(ctx, vb, vel.shape)
+        rp, rv = ok.nbody(prev_p, prev_v, 1)
+        assert rel_ok(gv[:, :3], rv[:, :3], 1e-5)[0], rel_ok(gv[:, :3], rv[:, :3], 1e-5)
+        assert rel_ok(gp[:, :3], rp[:, :3], 1e-5)[0]
+        assert np.array_equal(gp[:, 3], pos[:, 3])
+        prev_p, prev_v = gp, gv
+    abi.pk_finalize(ctx)
     p1, v1, _ = _nbody(pos, vel, steps, 1)
-    assert rel_ok(v1[:, :3], rv[:, :3], 1e-5)[0]
-    assert rel_ok(p1[:, :3], rp[:, :3], 1e-5)[0]
     for P in (2, 3, 8):
         pp, vp, st = _nbody(pos, vel, steps, P)
         assert np.array_equal(p1, pp) and np.array_equal(v1, vp)
@@ -232,3 +249,51 @@ def test_caller_owned_torch_instances_and_timer():
     # partition 0's instance holds its own rows of the result
     torch.cuda.synchronize()
     assert np.array_equal(tens[0][0][: h // 2].cpu().numpy(), ref[: h // 2])
+
+
+# ------------------------------------------------------------------ C4 SGEMM (tcgen05 3xTF32)
+def _gemm(a, b, P):
+    ctx = gpu_ctx(P)
+    pr, c = K.sgemm_program(ctx, a, b)
+    out = fetch(ctx, c, (a.shape[0], b.shape[1]))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return out, st
+
+
+def test_gemm_identity_and_rank1_exact():
+    rng = np.random.default_rng(21)
+    n = 512
+    b = rng.uniform(-1, 1, size=(n, n)).astype(np.float32)
+    g, _ = _gemm(np.eye(n, dtype=np.float32), b, 1)
+    # hi + lo reproduces b to within 2^-21 relative (lo rounded to TF32)
+    assert np.max(np.abs(g - b)) <= 2.0 ** -20
+    m, nn, k = 256, 512, 64
+    u = np.arange(1, m + 1, dtype=np.float32) % 17 + 1
+    v = np.arange(1, nn + 1, dtype=np.float32) % 13 + 1
+    a = np.repeat(u[:, None], k, axis=1)
+    bb = np.repeat(v[None, :], k, axis=0)
+    g, _ = _gemm(a, bb, 1)
+    assert np.array_equal(g, (k * np.outer(u, v)).astype(np.float32))
+
+
+def test_gemm_tf32_sensitive_pin():
+    # A = 1 + 2^-12 is not a TF32 value: 1xTF32 would give K, 3xTF32 gives K (1 + 2^-12) exactly
+    m, n, k = 128, 256, 256
+    a = np.full((m, k), 1.0 + 2.0 ** -12, np.float32)
+    b = np.ones((k, n), np.float32)
+    g, _ = _gemm(a, b, 1)
+    assert np.all(g == np.float32(k * (1.0 + 2.0 ** -12)))
+
+
+@pytest.mark.parametrize("m,n,k", [(300, 520, 200), (512, 512, 512), (1024, 768, 1040)])
+def test_gemm_oracle_and_bitwise(m, n, k):
+    a, b = synth.gemm_operands(m, n, k)
+    ref = ok.gemm(a, b)
+    g1, _ = _gemm(a, b, 1)
+    ok_, err = rel_ok(g1, ref, 1e-4)
+    assert ok_, err
+    for P in (2, 3):
+        gp, st = _gemm(a, b, P)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]

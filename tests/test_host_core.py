@@ -67,11 +67,13 @@ def test_jacobi_regions(h, w, block, P):
     abi.pk_finalize(ctx)
 
 
-@pytest.mark.parametrize("h,w,ty,bdx", [(64, 64, 4, 32), (100, 36, 16, 32), (33, 520, 4, 128), (5, 4, 64, 128)])
+@pytest.mark.parametrize("kernel,h,w,ty,bdx", [("hotspot2d_regs", 64, 64, 4, 32), ("hotspot2d_regs", 100, 36, 16, 32),
+                                               ("hotspot2d_regs", 33, 520, 4, 128), ("hotspot2d", 33, 1100, 4, 128),
+                                               ("hotspot2d", 5, 4, 64, 128), ("hotspot2d", 200, 1028, 16, 128)])
 @pytest.mark.parametrize("P", [1, 2, 3, 4, 7])
-def test_hotspot_regions(h, w, ty, bdx, P):
+def test_hotspot_regions(kernel, h, w, ty, bdx, P):
     ctx = host_ctx(P)
-    k = abi.pk_builtin_kernel(ctx, "hotspot2d")
+    k = abi.pk_builtin_kernel(ctx, kernel)
     bufs = [abi.pk_register_buffer(ctx, (h, w), 4) for _ in range(3)]
     grid, blk, sc = K.hotspot2d_launch(h, w, ty, bdx)
     for p in range(P):
@@ -285,7 +287,7 @@ def test_hotspot_sequence(P):
     h = w = 64
     geom = K.hotspot2d_launch(h, w, 4, 32)
     launches = [[("t0" if t % 2 == 0 else "t1"), "pw", ("t1" if t % 2 == 0 else "t0"), h, w, 4] for t in range(5)]
-    st_, sh = _run_pair(P, "hotspot2d", {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False),
+    st_, sh = _run_pair(P, "hotspot2d_regs", {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False),
                                          "pw": ((h, w), 4, True)}, launches, geom,
                         lambda box: regions.hotspot2d(box, geom[1], h, w, 4))
     # every iteration moves exactly the halo rows when the linear upload of t0 is
@@ -295,6 +297,15 @@ def test_hotspot_sequence(P):
     else:
         assert st_["stale_bytes"] > 5 * cf.hotspot2d_stale_per_iter(w, P)
     assert len(sh.buffers["t0"].rle()) <= 2 * P - 1
+
+
+@pytest.mark.parametrize("P", [2, 5])
+def test_hotspot_tma_sequence(P):
+    h, w = 40, 1100
+    geom = K.hotspot2d_launch(h, w, 4, 128)
+    launches = [[("t0" if t % 2 == 0 else "t1"), "pw", ("t1" if t % 2 == 0 else "t0"), h, w, 4] for t in range(4)]
+    _run_pair(P, "hotspot2d", {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False), "pw": ((h, w), 4, True)},
+              launches, geom, lambda box: regions.hotspot2d(box, geom[1], h, w, 4))
 
 
 @pytest.mark.parametrize("P", [2, 3])
@@ -309,7 +320,7 @@ def test_heat_sequence(P):
 @pytest.mark.parametrize("mode", [0, abi.PK_MODE_SINGLE_OWNER])
 def test_nbody_sequence(mode):
     n, P = 1024, 8
-    geom = K.nbody_launch(n, 64)
+    geom = K.nbody_launch(n, 32)            # 8 blocks of 128 bodies: one per partition
     launches = [[("p0" if s % 2 == 0 else "p1"), "v", ("p1" if s % 2 == 0 else "p0"), n] for s in range(3)]
     st_, _ = _run_pair(P, "nbody", {"p0": ((n,), 16, True), "p1": ((n,), 16, False), "v": ((n,), 16, True)},
                        launches, geom, lambda box: regions.nbody(box, geom[1], n, K.NBODY_PER_THREAD), mode)
@@ -380,4 +391,31 @@ def test_h2d_linear_distribution_tracker():
     assert abi.pk_tracker_dump(ctx, b) == sb.rle()
     b2 = abi.pk_register_buffer(ctx, (7, 3), 4)
     assert abi.pk_tracker_dump(ctx, b2) == [(0, 84, 7)]           # reading Q3
+    abi.pk_finalize(ctx)
+
+
+@pytest.mark.parametrize("m,n,k", [(300, 520, 200), (1024, 512, 64)])
+@pytest.mark.parametrize("P", [1, 2, 3])
+def test_gemm_regions(m, n, k, P):
+    ctx = host_ctx(P)
+    kern = abi.pk_builtin_kernel(ctx, "sgemm_tf32x3")
+    bufs = [abi.pk_register_buffer(ctx, s, 4) for s in ((m, k), (k, n), (m, n))]
+    grid, blk, sc = K.sgemm_launch(m, n, k)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, kern, grid, p)
+        lib = _lib_sets(ctx, kern, 6, bufs + [None] * 3, box, blk, sc)
+        ora = _oracle_sets(regions.gemm(box, m, n, k, K.GEMM_BM, K.GEMM_BN), {0: 4, 1: 4, 2: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
+def test_gemm_b_broadcast_stale_bytes():
+    m = n = k = 512
+    P = 4
+    ctx = host_ctx(P)
+    K.sgemm_program(ctx, np.zeros((m, k), np.float32), np.zeros((k, n), np.float32), launches=2)
+    s = abi.pk_get_stats(ctx)
+    # first launch: every partition pulls the (P-1)/P of B it lacks; A's linear upload
+    # matches the row partition; the second launch moves nothing (validity map, Q4)
+    assert s["stale_bytes"] == cf.gemm_stale(k, n, P)
     abi.pk_finalize(ctx)
