@@ -363,44 +363,53 @@ def main():
     from paper_conf_icppw_matzdf20_b200 import abi
 
     ngpu = max(1, args.gpus)
-    P = args.parts or ngpu
-    elapsed_ms = 0.0
     result = {}
-    if rank == 0:
+    if world > 1:
+        # SPMD: one process per GPU, one partition per rank; the
+        # replicated plan's cross-rank copies are NCCL send/recv pairs.
+        P = world
+        local_rank = env_int("LOCAL_RANK", rank)
+        torch.cuda.set_device(local_rank)
+        nid = [abi.pk_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(nid, src=0)
+        ctx = abi.pk_init_spmd(P, rank, world, list(range(world)), part_device=[local_rank] * P, nccl_id=nid[0])
+        devices = list(range(ngpu))
+        process_model = "SPMD: one process per GPU, replicated tracker, NCCL send/recv for cross-rank copies"
+    else:
+        P = args.parts or ngpu
         ndev = torch.cuda.device_count()
         if ndev < ngpu:
             raise SystemExit(f"--gpus {ngpu} but only {ndev} visible")
-        part_device = [p % ngpu for p in range(P)]
-        ctx = abi.pk_init(P, part_device=part_device)
-        w.setup(ctx)
-        for _ in range(args.warmup):
-            w.step()
-        abi.pk_synchronize(ctx)
-        abi.pk_reset_stats(ctx)
-        abi.pk_set_mode(ctx, abi.PK_MODE_TIME_KERNELS)
+        ctx = abi.pk_init(P, part_device=[p % ngpu for p in range(P)])
+        devices = sorted(set(p % ngpu for p in range(P)))
+        process_model = "one host process drives all partitions"
+    w.setup(ctx)
+    for _ in range(args.warmup):
+        w.step()
+    abi.pk_synchronize(ctx)
+    abi.pk_reset_stats(ctx)
+    abi.pk_set_mode(ctx, abi.PK_MODE_TIME_KERNELS)
     if dist:
         dist.barrier()
     sampler = ClockSampler(range(ngpu)) if rank == 0 else None
-    if rank == 0:
+    if sampler:
         sampler.start()
         time.sleep(0.3)
-        abi.pk_synchronize(ctx)
-        abi.pk_timer_begin(ctx)
-        for _ in range(args.steps):
-            w.step()
-        elapsed_ms = abi.pk_timer_end(ctx)
-        clocks = sampler.stop()
-        st = abi.pk_get_stats(ctx)
-        abi.pk_set_mode(ctx, 0)
+    abi.pk_synchronize(ctx)
+    abi.pk_timer_begin(ctx)
+    for _ in range(args.steps):
+        w.step()
+    elapsed_ms = abi.pk_timer_end(ctx)
+    clocks = sampler.stop() if sampler else {}
+    st = abi.pk_get_stats(ctx)
+    abi.pk_set_mode(ctx, 0)
     if dist:
-        import torch as _t
-        tt = _t.tensor([elapsed_ms], dtype=_t.float64)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        elapsed_ms = float(tt.item())
-    if rank != 0:
-        if dist:
-            dist.barrier()
-        return
+        tt = torch.tensor([elapsed_ms, st["kernel_launches"], st["moved_bytes"], st["copies"]], dtype=torch.float64)
+        mx = tt.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tt, op=dist.ReduceOp.SUM)
+        elapsed_ms = float(mx[0])                 # max over ranks
+        st["kernel_launches"], st["moved_bytes"], st["copies"] = int(tt[1]), int(tt[2]), int(tt[3])
 
     units = w.units_per_iter * w.iters * args.steps
     value = units / (elapsed_ms / 1e3) / w.scale
@@ -437,10 +446,10 @@ def main():
         "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": WORKLOADS[w.name][0], "iterations_per_step": w.iters, "partitions": P,
-                   "partition_devices": sorted(set(p % ngpu for p in range(P))),
+                   "partition_devices": devices,
                    "l2": "inputs larger than the 126 MB L2 (no flush)" if w.name != "jacobi2d"
                    else "1 MB working set stays in L2 (latency-bound C1)",
-                   "process_model": "one host process drives all partitions (rank 0)"},
+                   "process_model": process_model},
         "gpu_launches": int(st["kernel_launches"]),
         "clocks": clocks,
         "roofline": roofline,
@@ -456,6 +465,8 @@ def main():
         pinned = [(b, torch.from_numpy(h).pin_memory()) for b, h in w.upload_bufs]
         out_host = torch.empty(w.out_shape(), dtype=torch.float32).pin_memory()
         abi.pk_synchronize(ctx)
+        if dist:
+            dist.barrier()
         t0 = time.perf_counter()
         h2d = d2h = 0
         for _ in range(args.e2e_steps):
@@ -467,6 +478,10 @@ def main():
             abi.pk_sync_to_host(ctx, out, out_host)
             d2h += out_host.numel() * out_host.element_size()
         el = time.perf_counter() - t0
+        if dist:
+            te = torch.tensor([el], dtype=torch.float64)
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+            el = float(te[0])
         result["e2e"] = {"value": w.units_per_iter * w.iters * args.e2e_steps / el / w.scale, "unit": w.unit,
                          "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
                          "steps": args.e2e_steps, "timing": "wall clock around pk_copy_from_host + launches + "
@@ -476,7 +491,8 @@ def main():
         result["cpu_baseline"] = cpu_oracle_rate(w)
     if dist:
         dist.barrier()
-    print(json.dumps(result), flush=True)
+    if rank == 0:
+        print(json.dumps(result), flush=True)
 
 
 if __name__ == "__main__":

@@ -89,6 +89,24 @@ typedef struct {
 int pk_init(const pk_init_params* params, pk_ctx* out);
 int pk_finalize(pk_ctx ctx);
 
+/* ---- multi-process SPMD (one process per GPU) ----
+ * Every rank runs the same host program and calls the same pk_* sequence, so the
+ * partitioning, regions, tracker and transfer plan are computed identically
+ * (replicated, deterministic) on every rank; a rank executes only the kernels of
+ * the partitions it owns (part_rank[p] == my_rank) and its side of each copy.
+ * Copies between partitions of different ranks are NCCL send/recv pairs on the
+ * owning partitions' streams (NCCL is loaded at run time from libnccl.so.2).
+ * Execution requires exactly one partition per rank; host-only contexts accept
+ * any mapping (planning / tests).
+ * pk_nccl_unique_id writes the 128-byte ncclUniqueId (rank 0 creates it, the
+ * caller broadcasts it, e.g. with torch.distributed); pk_init_spmd is pk_init
+ * plus that id (ignored for host-only contexts; may be NULL then).
+ * pk_sync_to_host is collective in SPMD mode: rank 0 receives every segment it
+ * does not hold and writes `host`; other ranks may pass host = NULL.
+ * Errors: PK_ERR_NCCL (library missing or an NCCL call failed), PK_ERR_STATE. */
+int pk_nccl_unique_id(void* out, size_t bytes);
+int pk_init_spmd(const pk_init_params* params, const void* nccl_unique_id, pk_ctx* out);
+
 /* ---------------------------------------------------------------- buffers */
 /* Virtual buffer = one full-size device instance per partition + a tracker
  * (§8.1; full-size instances keep the kernels' global indices, reading

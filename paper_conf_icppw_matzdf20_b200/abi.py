@@ -87,9 +87,22 @@ def lib():
     if not os.path.exists(LIB_PATH):
         raise RuntimeError(f"{LIB_PATH} is missing: build the CUDA extension first "
                            "(python -m paper_conf_icppw_matzdf20_b200.build); there is no fallback")
+    if "PK_NCCL_LIB" not in os.environ:      # NCCL is dlopen'ed only by SPMD contexts
+        try:
+            import importlib.util
+            spec = importlib.util.find_spec("nvidia")
+            for base in (spec.submodule_search_locations or []) if spec else []:
+                cand = os.path.join(base, "nccl", "lib", "libnccl.so.2")
+                if os.path.exists(cand):
+                    os.environ["PK_NCCL_LIB"] = cand
+                    break
+        except Exception:
+            pass
     L = C.CDLL(LIB_PATH)
     sig = {
         "pk_init": [C.POINTER(pk_init_params), C.POINTER(C.c_void_p)],
+        "pk_init_spmd": [C.POINTER(pk_init_params), C.c_void_p, C.POINTER(C.c_void_p)],
+        "pk_nccl_unique_id": [C.c_void_p, C.c_size_t],
         "pk_finalize": [C.c_void_p],
         "pk_register_buffer": [C.c_void_p, C.c_int, _I64P, C.c_int, C.POINTER(C.c_void_p), C.c_void_p, _I64P],
         "pk_copy_from_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
@@ -177,6 +190,22 @@ def pk_init(nparts, part_device=None, part_rank=None, my_rank=0, world_size=1, f
     return ctx
 
 
+def pk_nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    _check(lib().pk_nccl_unique_id(buf, 128), "pk_nccl_unique_id")
+    return buf.raw
+
+
+def pk_init_spmd(nparts, my_rank, world_size, part_rank, part_device=None, nccl_id=None, flags=0):
+    """Multi-process SPMD context: this rank owns the partitions p with part_rank[p] == my_rank."""
+    p = pk_init_params(nparts, my_rank, world_size, flags,
+                       _i32(part_device) if part_device is not None else None, _i32(part_rank))
+    ctx = C.c_void_p()
+    idbuf = C.create_string_buffer(nccl_id, 128) if nccl_id is not None else None
+    _check(lib().pk_init_spmd(C.byref(p), idbuf, C.byref(ctx)), "pk_init_spmd")
+    return ctx
+
+
 def pk_finalize(ctx):
     _check(lib().pk_finalize(ctx), "pk_finalize")
 
@@ -198,6 +227,7 @@ def pk_copy_from_host(ctx, buf, host, nbytes=None):
 
 
 def pk_sync_to_host(ctx, buf, host, nbytes=None):
+    """host may be None on SPMD ranks other than 0 (then pass nbytes)."""
     _check(lib().pk_sync_to_host(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
            "pk_sync_to_host")
 

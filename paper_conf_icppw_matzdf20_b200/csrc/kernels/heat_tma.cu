@@ -71,8 +71,10 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const float* __restrict__ u
             ptx::bulk_g2s(slot + (size_t)r * kRowF + toff, uin + p * HW + row * W + tlo, rbytes, &full[s]);
         }
     };
+    // fill every slot; after plane q is computed (barrier), slot (q - 1) % kNS is
+    // refilled with sequence q - 1 + kNS, so sequences are issued in order
     if (warp == 0)
-        for (int q = 0; q < kNS - 1 && q < nq; ++q) issue(q);
+        for (int q = 0; q < kNS && q < nq; ++q) issue(q);
 
     const int64_t i = i0 + ty, j0 = c0 + 4 * lane;
     const bool active = i < H && j0 < W;

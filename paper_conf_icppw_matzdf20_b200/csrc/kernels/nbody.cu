@@ -18,6 +18,10 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <mutex>
+#include <unordered_map>
+#include <utility>
+
 #include "../runtime/builtins.h"
 
 namespace pk {
@@ -70,12 +74,31 @@ __device__ __forceinline__ u64 rsqrt2(u64 v) {
     return pk2(rsqrt_ftz(a), rsqrt_ftz(b));
 }
 
-// Block = bdx threads; block b owns bodies [b*4*bdx, (b+1)*4*bdx): thread t holds
+// Source split (fixed, independent of P and of the physical grid): the
+// ceil(N / 1024) source chunks are cut into kSplit contiguous parts; part s of
+// body i is accumulated chunk by chunk into partial[s][i]; the finalize kernel
+// adds the kSplit partials in order s = 0..kSplit-1.  The persistent grid walks
+// (logical block, part) items, so ~kSplit x more, smaller work items than blocks
+// keep every SM busy to the end (no 2.3-wave tail).
+constexpr int kSplit = 8;
+
+__device__ __forceinline__ void part_chunks(int64_t N, int s, int64_t& c_begin, int64_t& c_end) {
+    const int64_t nch = (N + kChunk - 1) / kChunk;
+    c_begin = (nch * s) / kSplit * kChunk;
+    c_end = (nch * (s + 1)) / kSplit * kChunk;
+    if (c_end > N) c_end = N;
+}
+
+// Logical block = bdx threads owning bodies [b*4*bdx, (b+1)*4*bdx): thread t holds
 // bodies base + t + u*bdx (u = 0..3), paired as (u=0, u=1) and (u=2, u=3).
-__global__ void __launch_bounds__(256) k_nbody(const float4* __restrict__ pin, float4* __restrict__ vel,
-                                               float4* __restrict__ pout, int64_t N, pk_partition part) {
+__global__ void __launch_bounds__(256) k_nbody_partial(const float4* __restrict__ pin, float4* __restrict__ partial,
+                                                       int64_t N, pk_partition part) {
     __shared__ float4 sh[2 * kTile];
-    const int64_t bx = part.min[0] + blockIdx.x;  // Eq. 8
+    const int64_t nb = part.max[0] - part.min[0];
+    const int64_t nitems = nb * kSplit;
+    for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
+    const int64_t bx = part.min[0] + it % nb;  // Eq. 8
+    const int s_part = (int)(it / nb);
     const int64_t base = bx * (int64_t)kBodies * blockDim.x;
     float4 pi[kBodies];
 #pragma unroll
@@ -92,7 +115,9 @@ __global__ void __launch_bounds__(256) k_nbody(const float4* __restrict__ pin, f
         pz[h] = pk2(pi[2 * h].z, pi[2 * h + 1].z);
         ax[h] = ay[h] = az[h] = zero;
     }
-    for (int64_t c0 = 0; c0 < N; c0 += kChunk) {
+    int64_t cb, ce;
+    part_chunks(N, s_part, cb, ce);
+    for (int64_t c0 = cb; c0 < ce; c0 += kChunk) {
         u64 sx[2] = {zero, zero}, sy[2] = {zero, zero}, sz[2] = {zero, zero};
         const int64_t c1 = c0 + kChunk < N ? c0 + kChunk : N;
         for (int64_t t0 = c0; t0 < c1; t0 += kTile) {
@@ -135,14 +160,34 @@ __global__ void __launch_bounds__(256) k_nbody(const float4* __restrict__ pin, f
         up2(ax[u / 2], a0, a1);
         up2(ay[u / 2], b0, b1);
         up2(az[u / 2], c0_, c1_);
-        const float axu = (u & 1) ? a1 : a0, ayu = (u & 1) ? b1 : b0, azu = (u & 1) ? c1_ : c0_;
-        float4 v = vel[i];
-        v.x = fmaf(axu, kDt, v.x);
-        v.y = fmaf(ayu, kDt, v.y);
-        v.z = fmaf(azu, kDt, v.z);
-        vel[i] = v;
-        pout[i] = make_float4(fmaf(v.x, kDt, pi[u].x), fmaf(v.y, kDt, pi[u].y), fmaf(v.z, kDt, pi[u].z), pi[u].w);
+        partial[(int64_t)s_part * N + i] =
+            make_float4((u & 1) ? a1 : a0, (u & 1) ? b1 : b0, (u & 1) ? c1_ : c0_, 0.f);
     }
+    __syncthreads();  // the next item reuses the shared-memory tile
+    }
+}
+
+// a_i = sum of the kSplit partials in order; kick-drift (reading Q16).
+__global__ void __launch_bounds__(256) k_nbody_final(const float4* __restrict__ pin, float4* __restrict__ vel,
+                                                     float4* __restrict__ pout, const float4* __restrict__ partial,
+                                                     int64_t N, int64_t i0, int64_t i1) {
+    const int64_t i = i0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= i1) return;
+    float4 a = partial[i];
+#pragma unroll
+    for (int s = 1; s < kSplit; ++s) {
+        const float4 q = partial[(int64_t)s * N + i];
+        a.x += q.x;
+        a.y += q.y;
+        a.z += q.z;
+    }
+    const float4 p = pin[i];
+    float4 v = vel[i];
+    v.x = fmaf(a.x, kDt, v.x);
+    v.y = fmaf(a.y, kDt, v.y);
+    v.z = fmaf(a.z, kDt, v.z);
+    vel[i] = v;
+    pout[i] = make_float4(fmaf(v.x, kDt, p.x), fmaf(v.y, kDt, p.y), fmaf(v.z, kDt, p.z), p.w);
 }
 
 int describe_nbody(pk_ctx c, pk_kernel k) {
@@ -162,14 +207,54 @@ int describe_nbody(pk_ctx c, pk_kernel k) {
 cudaError_t launch_nbody(const LaunchInfo& li) {
     if (li.nscalars < 1) return cudaErrorInvalidValue;
     int64_t N = li.scalars[0];
-    if (li.block.x > kTile || li.block.y != 1 || li.block.z != 1) return cudaErrorInvalidValue;
-    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &N, (void*)&li.part};
-    return cudaLaunchKernel(li.fn, li.grid, li.block, argv, 0, li.stream);
+    if (li.block.x > kTile || li.block.x < 1 || li.block.y != 1 || li.block.z != 1) return cudaErrorInvalidValue;
+    if (N < 1) return cudaSuccess;
+    // per-stream scratch for the kSplit partial accelerations
+    static std::mutex mu;
+    static std::unordered_map<cudaStream_t, std::pair<float4*, size_t>> scratch;
+    float4* partial = nullptr;
+    {
+        std::lock_guard<std::mutex> g(mu);
+        auto& sc = scratch[li.stream];
+        const size_t need = (size_t)kSplit * (size_t)N;
+        if (sc.second < need) {
+            if (sc.first) cudaFree(sc.first);
+            sc.first = nullptr;
+            sc.second = 0;
+            cudaError_t e = cudaMalloc(&sc.first, need * sizeof(float4));
+            if (e != cudaSuccess) return e;
+            sc.second = need;
+        }
+        partial = sc.first;
+    }
+    static int resident[64] = {0}, sms[64] = {0};
+    const int d = li.device;
+    if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
+    if (!resident[d]) {
+        int nb = 0;
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_nbody_partial, li.block.x, 0);
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms[d], cudaDevAttrMultiProcessorCount, d);
+        if (e != cudaSuccess) return e;
+        resident[d] = nb > 0 ? nb : 1;
+    }
+    const int64_t items = (int64_t)li.grid.x * kSplit;
+    const int64_t cap = (int64_t)resident[d] * sms[d];
+    dim3 grid((unsigned)(items < cap ? items : cap));
+    void* argv[] = {(void*)&li.inst[0], &partial, &N, (void*)&li.part};
+    cudaError_t e = cudaLaunchKernel((const void*)k_nbody_partial, grid, li.block, argv, 0, li.stream);
+    if (e != cudaSuccess) return e;
+    const int64_t per_block = (int64_t)kBodies * li.block.x;
+    int64_t i0 = (int64_t)li.part.min[0] * per_block, i1 = (int64_t)li.part.max[0] * per_block;
+    if (i1 > N) i1 = N;
+    if (i1 <= i0) return cudaSuccess;
+    void* argf[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &partial, &N, &i0, &i1};
+    return cudaLaunchKernel((const void*)k_nbody_final, dim3((unsigned)((i1 - i0 + 255) / 256)), dim3(256), argf, 0,
+                            li.stream);
 }
 
 }  // namespace
 
-const Builtin kBuiltinNbody = {"nbody", (const void*)k_nbody, 4,
+const Builtin kBuiltinNbody = {"nbody", (const void*)k_nbody_partial, 4,
                                {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR}, 0,
                                describe_nbody, launch_nbody};
 

@@ -14,6 +14,7 @@
 //        that read (b,p) since its last write ("readers").
 // PK_MODE_GLOBAL_BARRIER restores the literal host-side barrier.
 #include <cuda_runtime.h>
+#include <dlfcn.h>
 
 #include <algorithm>
 #include <chrono>
@@ -55,6 +56,47 @@ uint64_t now_ns() {
 }
 
 enum : uint8_t { W_NONE = 0, W_KERNEL = 1, W_COPY = 2 };
+
+// ---- NCCL, loaded at run time (only multi-process SPMD contexts need it) ----
+struct NcclId {
+    char internal[128];  // layout of ncclUniqueId
+};
+struct NcclApi {
+    bool ok = false;
+    int (*GetUniqueId)(NcclId*) = nullptr;
+    int (*CommInitRank)(void** comm, int nranks, NcclId id, int rank) = nullptr;
+    int (*CommDestroy)(void* comm) = nullptr;
+    int (*Send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+    int (*Recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+    int (*GroupStart)() = nullptr;
+    int (*GroupEnd)() = nullptr;
+    const char* (*GetErrorString)(int) = nullptr;
+};
+constexpr int kNcclUint8 = 1;  // ncclUint8
+
+const NcclApi& nccl() {
+    static NcclApi api;
+    static bool tried = false;
+    if (tried) return api;
+    tried = true;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) {
+        const char* p = getenv("PK_NCCL_LIB");
+        if (p) h = dlopen(p, RTLD_NOW | RTLD_GLOBAL);
+    }
+    if (!h) return api;
+    api.GetUniqueId = (int (*)(NcclId*))dlsym(h, "ncclGetUniqueId");
+    api.CommInitRank = (int (*)(void**, int, NcclId, int))dlsym(h, "ncclCommInitRank");
+    api.CommDestroy = (int (*)(void*))dlsym(h, "ncclCommDestroy");
+    api.Send = (int (*)(const void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclSend");
+    api.Recv = (int (*)(void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclRecv");
+    api.GroupStart = (int (*)())dlsym(h, "ncclGroupStart");
+    api.GroupEnd = (int (*)())dlsym(h, "ncclGroupEnd");
+    api.GetErrorString = (const char* (*)(int))dlsym(h, "ncclGetErrorString");
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv && api.GroupStart &&
+             api.GroupEnd && api.GetErrorString;
+    return api;
+}
 
 struct Buffer {
     bool alive = false;
@@ -129,6 +171,8 @@ struct pk_ctx_s {
     int cur_device = -1;
     cudaEvent_t timer_start = nullptr, timer_stop = nullptr;
     bool timer_running = false;
+    int first_local = -1;    // lowest partition owned by this rank
+    void* comm = nullptr;    // ncclComm_t (SPMD only)
 
     bool local(int p) const { return prank[p] == rank; }
     int set_device(int d) {
@@ -225,7 +269,23 @@ extern "C" {
 const char* pk_last_error(void) { return g_err.c_str(); }
 const char* pk_version(void) { return "pk 0.1 (sm_100a)"; }
 
-int pk_init(const pk_init_params* prm, pk_ctx* out) {
+int pk_nccl_unique_id(void* out, size_t bytes) {
+    if (!out || bytes < sizeof(NcclId)) return fail(PK_ERR_INVALID, "need a 128-byte buffer");
+    const NcclApi& n = nccl();
+    if (!n.ok) return fail(PK_ERR_NCCL, "libnccl.so.2 could not be loaded (set PK_NCCL_LIB)");
+    NcclId id;
+    int r = n.GetUniqueId(&id);
+    if (r) return fail(PK_ERR_NCCL, std::string("ncclGetUniqueId: ") + n.GetErrorString(r));
+    std::memcpy(out, &id, sizeof id);
+    return PK_OK;
+}
+
+static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out);
+
+int pk_init(const pk_init_params* prm, pk_ctx* out) { return init_impl(prm, nullptr, out); }
+int pk_init_spmd(const pk_init_params* prm, const void* nccl_id, pk_ctx* out) { return init_impl(prm, nccl_id, out); }
+
+static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out) {
     if (!prm || !out) return fail(PK_ERR_INVALID, "null argument");
     if (prm->nparts < 1 || prm->nparts > PK_MAX_PARTS)
         return fail(PK_ERR_INVALID, "nparts must be in [1, 64]");
@@ -246,18 +306,27 @@ int pk_init(const pk_init_params* prm, pk_ctx* out) {
             c->prank[p] = prm->part_rank[p];
         }
     }
+    c->first_local = -1;
+    for (int p = 0; p < c->P; ++p)
+        if (c->local(p)) { c->first_local = p; break; }
     if (!c->host_only) {
-        if (c->world != 1)
-            return fail(PK_ERR_STATE, "multi-process execution is not implemented (host-only planning only)");
+        int nlocal = 0;
+        for (int p = 0; p < c->P; ++p) nlocal += c->local(p);
+        if (c->world > 1 && nlocal != 1)
+            return fail(PK_ERR_STATE, "SPMD execution needs exactly one partition per rank");
+        if (c->world > 1 && !nccl_id) return fail(PK_ERR_INVALID, "SPMD execution needs an NCCL unique id");
         int ndev = 0;
         PK_CUDA(cudaGetDeviceCount(&ndev));
         if (ndev < 1) return fail(PK_ERR_CUDA, "no CUDA device");
         for (int p = 0; p < c->P; ++p) {
-            c->dev[p] = prm->part_device ? prm->part_device[p] : p % ndev;
+            if (!c->local(p)) continue;
+            c->dev[p] = prm->part_device ? prm->part_device[p] : (c->world > 1 ? 0 : p % ndev);
             if (c->dev[p] < 0 || c->dev[p] >= ndev) return fail(PK_ERR_INVALID, "part_device out of range");
         }
-        // peer access between every pair of distinct devices in use
-        std::vector<int> used(c->dev);
+        // peer access between every pair of distinct local devices in use
+        std::vector<int> used;
+        for (int p = 0; p < c->P; ++p)
+            if (c->local(p)) used.push_back(c->dev[p]);
         std::sort(used.begin(), used.end());
         used.erase(std::unique(used.begin(), used.end()), used.end());
         for (int a : used)
@@ -277,12 +346,22 @@ int pk_init(const pk_init_params* prm, pk_ctx* out) {
         c->ev_copy.resize(c->P);
         c->event_pool.resize(c->P);
         for (int p = 0; p < c->P; ++p) {
+            if (!c->local(p)) continue;
             PK_CUDA(cudaSetDevice(c->dev[p]));
             PK_CUDA(cudaStreamCreateWithFlags(&c->stream[p], cudaStreamNonBlocking));
             PK_CUDA(cudaEventCreateWithFlags(&c->ev_kernel[p], cudaEventDisableTiming));
             PK_CUDA(cudaEventCreateWithFlags(&c->ev_copy[p], cudaEventDisableTiming));
+            c->cur_device = c->dev[p];
         }
-        c->cur_device = c->dev[c->P - 1];
+        if (c->world > 1) {
+            const NcclApi& n = nccl();
+            if (!n.ok) return fail(PK_ERR_NCCL, "libnccl.so.2 could not be loaded (set PK_NCCL_LIB)");
+            if (int r = c->set_device(c->dev[c->first_local])) return r;
+            NcclId id;
+            std::memcpy(&id, nccl_id, sizeof id);
+            int r = n.CommInitRank(&c->comm, c->world, id, c->rank);
+            if (r) return fail(PK_ERR_NCCL, std::string("ncclCommInitRank: ") + n.GetErrorString(r));
+        }
     }
     *out = c.release();
     return PK_OK;
@@ -302,16 +381,17 @@ int pk_synchronize(pk_ctx c) {
 int pk_timer_begin(pk_ctx c) {
     if (!c) return fail(PK_ERR_INVALID, "null ctx");
     if (c->host_only) return fail(PK_ERR_STATE, "host-only context has no device timer");
+    const int p0 = c->first_local;
     if (!c->timer_start) {
         for (cudaEvent_t* e : {&c->timer_start, &c->timer_stop}) {
-            if (int r = c->set_device(c->dev[0])) return r;
+            if (int r = c->set_device(c->dev[p0])) return r;
             PK_CUDA(cudaEventCreate(e));
         }
     }
-    if (int r = c->set_device(c->dev[0])) return r;
-    PK_CUDA(cudaEventRecord(c->timer_start, c->stream[0]));
-    for (int p = 1; p < c->P; ++p) {
-        if (!c->local(p)) continue;
+    if (int r = c->set_device(c->dev[p0])) return r;
+    PK_CUDA(cudaEventRecord(c->timer_start, c->stream[p0]));
+    for (int p = 0; p < c->P; ++p) {
+        if (!c->local(p) || p == p0) continue;
         if (int r = c->set_device(c->dev[p])) return r;
         PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->timer_start, 0));
     }
@@ -322,15 +402,16 @@ int pk_timer_begin(pk_ctx c) {
 int pk_timer_end(pk_ctx c, double* ms) {
     if (!c || !ms) return fail(PK_ERR_INVALID, "null argument");
     if (c->host_only || !c->timer_running) return fail(PK_ERR_STATE, "timer not running");
-    for (int p = 1; p < c->P; ++p) {
-        if (!c->local(p)) continue;
+    const int p0 = c->first_local;
+    for (int p = 0; p < c->P; ++p) {
+        if (!c->local(p) || p == p0) continue;
         if (int r = c->set_device(c->dev[p])) return r;
         PK_CUDA(cudaEventRecord(c->ev_kernel[p], c->stream[p]));
-        if (int r = c->set_device(c->dev[0])) return r;
-        PK_CUDA(cudaStreamWaitEvent(c->stream[0], c->ev_kernel[p], 0));
+        if (int r = c->set_device(c->dev[p0])) return r;
+        PK_CUDA(cudaStreamWaitEvent(c->stream[p0], c->ev_kernel[p], 0));
     }
-    if (int r = c->set_device(c->dev[0])) return r;
-    PK_CUDA(cudaEventRecord(c->timer_stop, c->stream[0]));
+    if (int r = c->set_device(c->dev[p0])) return r;
+    PK_CUDA(cudaEventRecord(c->timer_stop, c->stream[p0]));
     PK_CUDA(cudaEventSynchronize(c->timer_stop));
     float f = 0.f;
     PK_CUDA(cudaEventElapsedTime(&f, c->timer_start, c->timer_stop));
@@ -375,14 +456,16 @@ int pk_finalize(pk_ctx c) {
                     if (B.inst[p]) { cudaSetDevice(c->dev[p]); cudaFree(B.inst[p]); }
         }
         for (int p = 0; p < c->P; ++p) {
+            if (!c->local(p)) continue;
             cudaSetDevice(c->dev[p]);
             cudaStreamDestroy(c->stream[p]);
             cudaEventDestroy(c->ev_kernel[p]);
             cudaEventDestroy(c->ev_copy[p]);
             for (cudaEvent_t e : c->event_pool[p]) cudaEventDestroy(e);
         }
+        if (c->comm) nccl().CommDestroy(c->comm);
         if (c->timer_start) {
-            cudaSetDevice(c->dev[0]);
+            cudaSetDevice(c->dev[c->first_local]);
             cudaEventDestroy(c->timer_start);
             cudaEventDestroy(c->timer_stop);
         }
@@ -507,11 +590,57 @@ int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
     return PK_OK;
 }
 
+static int sync_to_host_spmd(pk_ctx c, Buffer& B, void* host) {
+    // collective n:1 gather to rank 0: segments rank 0's partition lacks are sent
+    // by their lowest holder straight into rank 0's instance, which then holds them
+    int r0 = -1;
+    for (int p = 0; p < c->P; ++p)
+        if (c->prank[p] == 0) { r0 = p; break; }
+    if (r0 < 0) return fail(PK_ERR_STATE, "rank 0 owns no partition");
+    struct Piece { uint64_t b, e; int src; };
+    std::vector<Piece> pieces;
+    RangeList received;
+    for (const Seg& s : B.tracker.segments()) {
+        int src = ((s.mask >> r0) & 1) ? r0 : -1;
+        for (int q = 0; q < c->P && src < 0; ++q)
+            if ((s.mask >> q) & 1) src = q;
+        if (src < 0) return fail(PK_ERR_STATE, "segment held by no partition");
+        if (!pieces.empty() && pieces.back().src == src && pieces.back().e == s.b) pieces.back().e = s.e;
+        else pieces.push_back({s.b, s.e, src});
+    }
+    const NcclApi& n = nccl();
+    const bool is_root = c->rank == 0;
+    if (int r = c->set_device(c->dev[c->first_local])) return r;
+    n.GroupStart();
+    for (const Piece& pc : pieces) {
+        if (pc.src == r0) continue;
+        received.push_back(Range{pc.b, pc.e});
+        int r = 0;
+        if (c->local(pc.src))
+            r = n.Send((const char*)B.inst[pc.src] + pc.b, pc.e - pc.b, kNcclUint8, 0, c->comm, c->stream[pc.src]);
+        else if (is_root)
+            r = n.Recv((char*)B.inst[r0] + pc.b, pc.e - pc.b, kNcclUint8, c->prank[pc.src], c->comm, c->stream[r0]);
+        if (r) { n.GroupEnd(); return fail(PK_ERR_NCCL, std::string("ncclSend/Recv: ") + n.GetErrorString(r)); }
+    }
+    if (int r = n.GroupEnd()) return fail(PK_ERR_NCCL, std::string("ncclGroupEnd: ") + n.GetErrorString(r));
+    if (is_root)
+        PK_CUDA(cudaMemcpyAsync(host, B.inst[r0], B.bytes, cudaMemcpyDeviceToHost, c->stream[r0]));
+    if (int r = pk_synchronize(c)) return r;
+    if (!(c->mode & PK_MODE_SINGLE_OWNER)) {  // replicated on every rank: r0 now holds what it received
+        canonicalize(&received);
+        B.tracker.add_bit(received, r0);
+    }
+    c->stats.d2h_bytes += is_root ? B.bytes : 0;
+    return PK_OK;
+}
+
 int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
-    if (!valid_buf(c, b) || !host) return fail(PK_ERR_INVALID, "bad argument");
+    if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "bad argument");
     Buffer& B = c->bufs[b];
     if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (D2H gathers the whole virtual buffer)");
     if (c->host_only) return fail(PK_ERR_STATE, "host-only context holds no data");
+    if (!host && (c->world == 1 || c->rank == 0)) return fail(PK_ERR_INVALID, "null host buffer");
+    if (c->world > 1) return sync_to_host_spmd(c, B, host);
     // query all segments, copy each from a partition that holds it.
     struct Piece { uint64_t b, e; int src; };
     std::vector<Piece> pieces;
@@ -774,11 +903,13 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
                 const int p = c->last_plan[i].dst;
                 size_t j = i;
                 while (j < c->last_plan.size() && c->last_plan[j].dst == p) ++j;
+                if (!c->local(p)) { i = j; continue; }  // another rank pulls (NCCL pass below)
                 if (int r = c->set_device(c->dev[p])) return r;
                 // WAR on the destination instances + RAW on each source's last writer
                 uint64_t waited_src = 0;
                 for (size_t t = i; t < j; ++t) {
                     const CopyOp& o = c->last_plan[t];
+                    if (!c->local(o.src)) continue;
                     Buffer& B = c->bufs[o.buf];
                     if (B.readers[p]) if (int r = wait_readers(c, B, p)) return r;
                     const uint8_t lw = B.last_writer[o.src];
@@ -791,6 +922,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
                 }
                 for (size_t t = i; t < j; ++t) {
                     const CopyOp& o = c->last_plan[t];
+                    if (!c->local(o.src)) continue;
                     Buffer& B = c->bufs[o.buf];
                     char* dst = (char*)B.inst[p] + o.b;
                     const char* src = (const char*)B.inst[o.src] + o.b;
@@ -805,11 +937,46 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
                 PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
                 for (size_t t = i; t < j; ++t) {
                     const CopyOp& o = c->last_plan[t];
+                    if (!c->local(o.src)) continue;
                     Buffer& B = c->bufs[o.buf];
                     B.readers[o.src] |= 1ull << p;
                     B.last_writer[p] = W_COPY;
                 }
                 i = j;
+            }
+            // SPMD: copies between ranks are NCCL send/recv pairs issued in the
+            // global plan order on both sides (one partition per rank, so stream
+            // order on that partition covers RAW and both WARs).
+            if (c->world > 1) {
+                const NcclApi& n = nccl();
+                bool open = false;
+                for (const CopyOp& o : c->last_plan) {
+                    const bool sl = c->local(o.src), dl = c->local(o.dst);
+                    if (sl == dl) continue;
+                    if (!open) {
+                        if (int r = c->set_device(c->dev[c->first_local])) return r;
+                        n.GroupStart();
+                        open = true;
+                    }
+                    Buffer& B = c->bufs[o.buf];
+                    int r;
+                    if (sl)
+                        r = n.Send((const char*)B.inst[o.src] + o.b, o.e - o.b, kNcclUint8, c->prank[o.dst], c->comm,
+                                   c->stream[o.src]);
+                    else
+                        r = n.Recv((char*)B.inst[o.dst] + o.b, o.e - o.b, kNcclUint8, c->prank[o.src], c->comm,
+                                   c->stream[o.dst]);
+                    if (r) { n.GroupEnd(); return fail(PK_ERR_NCCL, std::string("ncclSend/Recv: ") + n.GetErrorString(r)); }
+                    if (dl) {
+                        c->stats.copies += 1;
+                        c->stats.moved_bytes += o.e - o.b;
+                        if (o.src < 16 && o.dst < 16) c->stats.pair_bytes[o.src][o.dst] += o.e - o.b;
+                    }
+                }
+                if (open) {
+                    int r = n.GroupEnd();
+                    if (r) return fail(PK_ERR_NCCL, std::string("ncclGroupEnd: ") + n.GetErrorString(r));
+                }
             }
         }
         if (mode & PK_MODE_GLOBAL_BARRIER)  // Fig. 4 line 8, literally
