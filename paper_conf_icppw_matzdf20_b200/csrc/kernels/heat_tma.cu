@@ -4,40 +4,68 @@
 // replicate-clamped, alpha = 1/8) and logical block contract as heat3d_regs in
 // stencils.cu: block (bx, by, bz) = 128 columns x bdy rows x ZC planes.
 //
-// Memory side: a ring of NS shared-memory planes, each holding the block's
-// bdy + 2 rows (one halo row above and below, clamped) x (128 + 2 x 4) columns.
-// Warp 0 streams whole row segments of plane z + NS - 2 with cp.async.bulk (TMA
-// engine, one copy per row issued by the warp's lanes, one mbarrier per slot)
-// while every warp computes plane z from slots z-1, z, z+1: all seven neighbours
-// come from shared memory (x neighbours by warp shuffle + the column halo).  One
-// barrier per plane releases the oldest slot.  Bytes in flight per CTA ~ (NS-3)
-// planes, independent of registers.  Each input byte is fetched from HBM once,
-// plus the two CTA-boundary halo rows (2/bdy) and two halo planes (2/ZC).
+// Memory side (warp-specialised, no CTA-wide barrier in the main loop):
+//   * a ring of NS shared-memory planes, each one 3-D tensor-TMA box of
+//     (128 + 2 x 4) columns x (bdy + 2) rows x 1 plane -- the block's rows with one
+//     halo row above and below and a 4-float column halo each side (out-of-grid
+//     rows/columns are zero-filled by the TMA unit; the consumer applies the
+//     replicate clamp at the grid border itself);
+//   * a producer warp (the launcher adds it: physical block = (32, bdy + 1))
+//     issues ONE cp.async.bulk.tensor.3d per plane (plane index clamped to the
+//     grid) into slot q % NS once that slot's `empty` mbarrier shows every
+//     consumer warp released it;
+//   * each consumer warp computes its row of plane z from slots z-1, z, z+1 (all
+//     seven neighbours from shared memory, x neighbours by shuffle + the column
+//     halo) and releases slot z-1 with one mbarrier arrival.
+// Consumer warps free-run within the ring (no barrier stalls); every input byte
+// is fetched once per CTA plus the 2/bdy halo rows and 2/ZC halo planes; up to
+// NS - 3 planes (~18 KB each) are in flight per CTA.
+#include <cuda.h>
 #include <cuda_runtime.h>
+
+#include <mutex>
+#include <unordered_map>
 
 #include "../runtime/builtins.h"
 #include "ptx.cuh"
+#include "tma_host.h"
 
 namespace pk {
 namespace {
 
 constexpr float kAlpha = 0.125f;
-constexpr int kMaxBdy = 32;
+constexpr int kRPW = 2;                 // rows per consumer warp
+constexpr int kMaxBdy = 62;             // 31 consumer warps + 1 producer warp = 1024 threads
 constexpr int kHalo = 4;
-constexpr int kRowF = 128 + 2 * kHalo;  // floats per smem row (544 B, 16-B multiple)
-constexpr int kNS = 6;                  // ring depth (planes)
+constexpr int kRowF = 128 + 2 * kHalo;  // floats per box row (544 B)
+constexpr int kNS = 6;                  // ring depth (planes of up to 64 rows)
 
-__host__ __device__ constexpr size_t slot_floats(int bdy) { return (size_t)(bdy + 2) * kRowF; }
-__host__ __device__ constexpr size_t smem_bytes(int bdy) { return kNS * slot_floats(bdy) * 4 + kNS * 8; }
+__host__ __device__ constexpr int warp_count(int bdy) { return (bdy + kRPW - 1) / kRPW; }
 
-__global__ void __launch_bounds__(1024) k_heat3d_tma(const float* __restrict__ uin, float* __restrict__ uout,
-                                                    int64_t D, int64_t H, int64_t W, int64_t ZC,
-                                                    pk_partition part) {
-    extern __shared__ __align__(128) unsigned char smem[];
-    const int bdy = blockDim.y;
-    float* ring = reinterpret_cast<float*>(smem);
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + kNS * slot_floats(bdy) * 4);
-    const int lane = threadIdx.x, ty = threadIdx.y, warp = ty;
+__host__ __device__ constexpr size_t slot_bytes(int bdy) {
+    return (((size_t)(bdy + 2) * kRowF * 4) + 127) / 128 * 128;  // TMA destinations: 128-B aligned
+}
+__host__ __device__ constexpr size_t smem_bytes(int bdy) { return kNS * slot_bytes(bdy) + 2 * kNS * 8 + 128; }
+
+__device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, int32_t z,
+                                       uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+        "[%5];" ::"r"(ptx::smem_u32(dst)),
+        "l"(map), "r"(x), "r"(y), "r"(z), "r"(ptx::smem_u32(bar))
+        : "memory");
+}
+
+__global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUtensorMap tm_u,
+                                                    float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
+                                                    int64_t ZC, int bdy, pk_partition part) {
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
+    // bdy = logical rows per block; warps 0..nw-1 consume (kRPW rows each), warp nw produces
+    const size_t sb = slot_bytes(bdy);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + kNS * sb);
+    uint64_t* empty = full + kNS;
+    const int lane = threadIdx.x, warp = threadIdx.y;
     const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y, bz = part.min[2] + blockIdx.z;
     const int64_t c0 = bx * 128, i0 = by * bdy, k0 = bz * ZC;
     if (c0 >= W || i0 >= H || k0 >= D) return;  // block-uniform
@@ -45,75 +73,90 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const float* __restrict__ u
     const int nz = (int)(k1 - k0);             // planes computed
     const int nq = nz + 2;                     // planes streamed: k0-1 .. k1 (clamped)
     const int64_t HW = H * W;
-    // column segment [c0 - 4, c0 + 132) clipped to [0, W)
-    const int64_t tlo = max(c0 - kHalo, (int64_t)0), thi = min(c0 + 128 + kHalo, W);
-    const uint32_t rbytes = (uint32_t)(thi - tlo) * 4u;
-    const int toff = (int)(tlo - (c0 - kHalo));
-    const int nrows = bdy + 2;
 
     if (warp == 0 && lane == 0) {
-        for (int s = 0; s < kNS; ++s) ptx::mbar_init(&full[s], 1);
+        for (int s = 0; s < kNS; ++s) {
+            ptx::mbar_init(&full[s], 1);
+            ptx::mbar_init(&empty[s], warp_count(bdy));
+        }
         ptx::fence_mbar_init();
+        asm volatile("prefetch.tensormap [%0];" ::"l"(&tm_u) : "memory");
     }
     __syncthreads();
 
-    // stream plane sequence index q (plane k0 - 1 + q, clamped) into slot q % kNS
-    auto issue = [&](int q) {
-        const int s = q % kNS;
-        int64_t p = k0 - 1 + q;
-        p = p < 0 ? 0 : (p >= D ? D - 1 : p);
-        float* slot = ring + (size_t)s * slot_floats(bdy);
-        if (lane == 0) ptx::mbar_arrive_expect_tx(&full[s], rbytes * (uint32_t)nrows);
-        __syncwarp();
-        for (int r = lane; r < nrows; r += 32) {
-            int64_t row = i0 - 1 + r;
-            row = row < 0 ? 0 : (row >= H ? H - 1 : row);
-            ptx::bulk_g2s(slot + (size_t)r * kRowF + toff, uin + p * HW + row * W + tlo, rbytes, &full[s]);
+    if (warp == warp_count(bdy)) {
+        // ---------------- producer: one elected thread, one TMA per plane
+        if (lane != 0) return;
+        const uint32_t bytes = (uint32_t)((bdy + 2) * kRowF * 4);
+        for (int q = 0; q < nq; ++q) {
+            const int s = q % kNS;
+            ptx::mbar_wait(&empty[s], ((q / kNS) & 1u) ^ 1u);   // first pass: free
+            int64_t p = k0 - 1 + q;
+            p = p < 0 ? 0 : (p >= D ? D - 1 : p);
+            ptx::mbar_arrive_expect_tx(&full[s], bytes);
+            tma_3d(smem + (size_t)s * sb, &tm_u, (int32_t)(c0 - kHalo), (int32_t)(i0 - 1), (int32_t)p, &full[s]);
         }
-    };
-    // fill every slot; after plane q is computed (barrier), slot (q - 1) % kNS is
-    // refilled with sequence q - 1 + kNS, so sequences are issued in order
-    if (warp == 0)
-        for (int q = 0; q < kNS && q < nq; ++q) issue(q);
+        return;
+    }
 
-    const int64_t i = i0 + ty, j0 = c0 + 4 * lane;
-    const bool active = i < H && j0 < W;
+    // ---------------- consumer warp `warp` owns rows i0 + warp + r * nw (r < kRPW)
+    const int nw = warp_count(bdy);
+    const int64_t j0 = c0 + 4 * lane;
     const bool west_edge = j0 == 0, east_edge = j0 + 4 >= W;
     const int cx = kHalo + 4 * lane;
+    // ring slots of planes z-1, z, z+1 and the parity of z+1, advanced incrementally
+    int s_m = 0, s_c = 1, s_p = 2 % kNS;
+    uint32_t par_p = (2 / kNS) & 1;
     ptx::mbar_wait(&full[0], 0);
     ptx::mbar_wait(&full[1 % kNS], (1 / kNS) & 1);
     for (int q = 1; q <= nz; ++q) {
-        ptx::mbar_wait(&full[(q + 1) % kNS], ((q + 1) / kNS) & 1);
-        const float* sm = ring + (size_t)((q - 1) % kNS) * slot_floats(bdy);
-        const float* sc = ring + (size_t)(q % kNS) * slot_floats(bdy);
-        const float* sp = ring + (size_t)((q + 1) % kNS) * slot_floats(bdy);
-        const float4 c = *reinterpret_cast<const float4*>(sc + (ty + 1) * kRowF + cx);
-        const float4 zm = *reinterpret_cast<const float4*>(sm + (ty + 1) * kRowF + cx);
-        const float4 zp = *reinterpret_cast<const float4*>(sp + (ty + 1) * kRowF + cx);
-        const float4 ym = *reinterpret_cast<const float4*>(sc + ty * kRowF + cx);
-        const float4 yp = *reinterpret_cast<const float4*>(sc + (ty + 2) * kRowF + cx);
-        float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
-        float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
-        if (lane == 0) wv = sc[(ty + 1) * kRowF + cx - 1];
-        if (lane == 31) ev = sc[(ty + 1) * kRowF + cx + 4];
-        if (west_edge) wv = c.x;
-        if (east_edge) ev = c.w;
-        if (active) {
+        ptx::mbar_wait(&full[s_p], par_p);
+        const float* sm = reinterpret_cast<const float*>(smem + (size_t)s_m * sb);
+        const float* sc = reinterpret_cast<const float*>(smem + (size_t)s_c * sb);
+        const float* sp = reinterpret_cast<const float*>(smem + (size_t)s_p * sb);
+        const int64_t kout = (k0 + q - 1) * HW;
+#pragma unroll
+        for (int r = 0; r < kRPW; ++r) {
+            const int ty = warp + r * nw;
+            const int64_t i = i0 + ty;
+            const int so = ((ty < bdy ? ty : bdy - 1) + 1) * kRowF + cx;  // rows past bdy: stay in the slot
+            const float4 c = *reinterpret_cast<const float4*>(sc + so);
+            const float4 zm = *reinterpret_cast<const float4*>(sm + so);
+            const float4 zp = *reinterpret_cast<const float4*>(sp + so);
+            float4 ym = *reinterpret_cast<const float4*>(sc + so - kRowF);
+            float4 yp = *reinterpret_cast<const float4*>(sc + so + kRowF);
+            float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
+            float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
+            if (lane == 0) wv = sc[so - 1];
+            if (lane == 31) ev = sc[so + 4];
+            if (ty >= bdy || i >= H || j0 >= W) continue;
+            if (west_edge) wv = c.x;
+            if (east_edge) ev = c.w;
+            if (i == 0) ym = c;        // replicate clamp (the TMA zero-filled row -1)
+            if (i == H - 1) yp = c;    // ... and row H
             float4 o;
             o.x = c.x + kAlpha * ((zm.x + zp.x + ym.x + yp.x + wv + c.y) - 6.0f * c.x);
             o.y = c.y + kAlpha * ((zm.y + zp.y + ym.y + yp.y + c.x + c.z) - 6.0f * c.y);
             o.z = c.z + kAlpha * ((zm.z + zp.z + ym.z + yp.z + c.y + c.w) - 6.0f * c.z);
             o.w = c.w + kAlpha * ((zm.w + zp.w + ym.w + yp.w + c.z + ev) - 6.0f * c.w);
-            *reinterpret_cast<float4*>(uout + (k0 + q - 1) * HW + i * W + j0) = o;
+            *reinterpret_cast<float4*>(uout + kout + i * W + j0) = o;
         }
-        __syncthreads();  // everyone is done with slot (q - 1): refill it NS planes ahead
-        const int qn = q - 1 + kNS;
-        if (warp == 0 && qn < nq) issue(qn);
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&empty[s_m]);  // slot z-1 no longer needed by this warp
+        s_m = s_c;
+        s_c = s_p;
+        if (++s_p == kNS) { s_p = 0; par_p ^= 1u; }
+    }
+    __syncwarp();
+    if (lane == 0) {
+        ptx::mbar_arrive(&empty[nz % kNS]);
+        ptx::mbar_arrive(&empty[(nz + 1) % kNS]);
     }
 }
 
 int describe_heat3d_tma(pk_ctx c, pk_kernel k) {
-    // identical contract to heat3d_regs (stencils.cu): scalars 0 = D, 1 = H, 2 = W, 3 = ZC
+    // identical contract to heat3d_regs (stencils.cu): scalars 0 = D, 1 = H, 2 = W, 3 = ZC;
+    // the logical block is (32, bdy) -- the launcher adds the producer warp
     const int32_t off[7][3] = {{0, 0, 0}, {-1, 0, 0}, {1, 0, 0}, {0, -1, 0}, {0, 1, 0}, {0, 0, -1}, {0, 0, 1}};
     const uint32_t f = PK_DIM_GUARD | PK_DIM_CLAMP;
     for (int t = 0; t < 7; ++t) {
@@ -132,18 +175,38 @@ int describe_heat3d_tma(pk_ctx c, pk_kernel k) {
 cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
     if (li.nscalars < 4) return cudaErrorInvalidValue;
     int64_t D = li.scalars[0], H = li.scalars[1], W = li.scalars[2], ZC = li.scalars[3];
-    if (W % 4 || W < 4 || ZC < 1 || li.block.x != 32 || li.block.y < 1 || li.block.y > kMaxBdy || li.block.z != 1)
+    const int bdy = (int)li.block.y;
+    if (W % 4 || W < 4 || ZC < 1 || li.block.x != 32 || bdy < 1 || bdy > kMaxBdy || li.block.z != 1)
         return cudaErrorInvalidValue;
-    const size_t smem = smem_bytes(li.block.y);
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_heat3d_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)smem_bytes(kMaxBdy));
-        if (e != cudaSuccess) return e;
-        attr = true;
+    static std::once_flag once;
+    static cudaError_t attr_err = cudaSuccess;
+    std::call_once(once, [] {
+        attr_err = cudaFuncSetAttribute(k_heat3d_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)smem_bytes(kMaxBdy));
+    });
+    if (attr_err != cudaSuccess) return attr_err;
+    // tensor map of this instance: dims (W, H, D), box (136, bdy + 2, 1), OOB zero fill
+    static std::mutex mu;
+    static std::unordered_map<const void*, std::pair<uint64_t, CUtensorMap>> cache;
+    CUtensorMap tm;
+    {
+        std::lock_guard<std::mutex> g(mu);
+        const uint64_t key = ((uint64_t)W * 1315423911ull) ^ ((uint64_t)H << 20) ^ ((uint64_t)D << 40) ^ (uint64_t)bdy;
+        auto it = cache.find(li.inst[0]);
+        if (it != cache.end() && it->second.first == key) {
+            tm = it->second.second;
+        } else {
+            cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)D};
+            cuuint32_t box[3] = {(cuuint32_t)kRowF, (cuuint32_t)(bdy + 2), 1};
+            if (!tma_encode_f32(&tm, li.inst[0], 3, dims, box, CU_TENSOR_MAP_SWIZZLE_NONE))
+                return cudaErrorInvalidValue;
+            cache[li.inst[0]] = {key, tm};
+        }
     }
-    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &D, &H, &W, &ZC, (void*)&li.part};
-    return cudaLaunchKernel((const void*)k_heat3d_tma, li.grid, li.block, argv, smem, li.stream);
+    int bdy_arg = bdy;
+    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part};
+    return cudaLaunchKernel((const void*)k_heat3d_tma, li.grid, dim3(32, warp_count(bdy) + 1), argv, smem_bytes(bdy),
+                            li.stream);
 }
 
 }  // namespace

@@ -155,8 +155,20 @@ __global__ void __launch_bounds__(256, 1)
     uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tmem_full + 1);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int64_t m0 = (int64_t)(part.min[1] + blockIdx.y) * BM;  // Eq. 8
-    const int64_t n0 = (int64_t)(part.min[0] + blockIdx.x) * BN;
+    // Grouped rasterisation: the CTAs running at the same time cover kGroup tile
+    // rows x (wave / kGroup) tile columns, so each B panel k-slice is read from
+    // HBM once per kGroup rows (not once per row) and each A slice once per wave.
+    // The CTA -> logical tile map is a bijection onto the partition's box, so the
+    // launch still computes exactly the blocks [min, max) (Eq. 8-10).
+    constexpr int kGroup = 16;
+    const int64_t gx = part.max[0] - part.min[0], gy = part.max[1] - part.min[1];
+    const int64_t L = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
+    const int64_t grp = L / (kGroup * gx);
+    const int64_t row0 = grp * kGroup;
+    const int64_t gsz = (gy - row0) < kGroup ? (gy - row0) : kGroup;
+    const int64_t in = L - grp * kGroup * gx;
+    const int64_t m0 = (int64_t)(part.min[1] + row0 + in % gsz) * BM;  // Eq. 8
+    const int64_t n0 = (int64_t)(part.min[0] + in / gsz) * BN;
     const int nk = (int)((K + BK - 1) / BK);
 
     if (warp == 0 && lane == 0) {

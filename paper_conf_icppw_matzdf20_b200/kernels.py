@@ -15,8 +15,8 @@ from . import abi
 
 # ---------------------------------------------------------------- geometry
 JACOBI_BLOCK = (32, 8, 1)
-HOTSPOT_BDX, HOTSPOT_TY = 128, 64     # "hotspot2d" (TMA ring) requires bdx = 128
-HEAT_BDY, HEAT_ZC = 32, 128
+HOTSPOT_BDX, HOTSPOT_TY = 128, 128    # "hotspot2d" (TMA ring) requires bdx = 128
+HEAT_BDY, HEAT_ZC = 62, 128           # "heat3d" (TMA ring): bdy <= 62 rows (2 per consumer warp)
 NBODY_BDX, NBODY_PER_THREAD = 256, 4
 
 

@@ -126,8 +126,10 @@ def _heat(u, iters, P, zc=8, bdy=8, kernel="heat3d"):
     return res, st
 
 
-@pytest.mark.parametrize("kernel,d,h,w,zc,bdy", [("heat3d", 40, 36, 132, 8, 8), ("heat3d", 17, 9, 256, 4, 32),
-                                                  ("heat3d", 64, 64, 64, 64, 32), ("heat3d", 9, 70, 260, 3, 1),
+@pytest.mark.parametrize("kernel,d,h,w,zc,bdy", [("heat3d", 40, 36, 132, 8, 8), ("heat3d", 17, 9, 256, 4, 31),
+                                                  ("heat3d", 64, 64, 64, 64, 62), ("heat3d", 9, 70, 260, 3, 1),
+                                                  ("heat3d", 20, 130, 132, 7, 61),
+                                                  ("heat3d", 130, 62, 132, 128, 31),
                                                   ("heat3d_regs", 40, 36, 132, 8, 8),
                                                   ("heat3d_regs", 17, 9, 256, 4, 32)])
 def test_heat_oracle_and_bitwise(kernel, d, h, w, zc, bdy):
