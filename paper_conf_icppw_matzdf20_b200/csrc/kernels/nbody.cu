@@ -69,9 +69,17 @@ __device__ __forceinline__ float rsqrt_ftz(float x) {
     return r;
 }
 __device__ __forceinline__ u64 rsqrt2(u64 v) {
-    float a, b;
-    up2(v, a, b);
-    return pk2(rsqrt_ftz(a), rsqrt_ftz(b));
+    // one asm block so that ptxas can keep both MUFU results in the register pair
+    // (separate unpack / MUFU / pack statements cost ~3 MOVs per interaction)
+    u64 r;
+    asm("{\n\t.reg .f32 a, b;\n\t"
+        "mov.b64 {a, b}, %1;\n\t"
+        "rsqrt.approx.ftz.f32 a, a;\n\t"
+        "rsqrt.approx.ftz.f32 b, b;\n\t"
+        "mov.b64 %0, {a, b};\n\t}"
+        : "=l"(r)
+        : "l"(v));
+    return r;
 }
 
 // Source split (fixed, independent of P and of the physical grid): the
@@ -90,80 +98,82 @@ __device__ __forceinline__ void part_chunks(int64_t N, int s, int64_t& c_begin, 
 }
 
 // Logical block = bdx threads owning bodies [b*4*bdx, (b+1)*4*bdx): thread t holds
-// bodies base + t + u*bdx (u = 0..3), paired as (u=0, u=1) and (u=2, u=3).
+// bodies base + t + u*bdx (u = 0..3).  The packed f32x2 lanes carry two SOURCES
+// (even / odd within the tile) against a scalar body coordinate, which FADD2 /
+// FFMA2 take as a free broadcast operand; each body accumulates two interleaved
+// partial sums (even and odd sources) that are added at the end -- a fixed,
+// position-only order.
 __global__ void __launch_bounds__(256) k_nbody_partial(const float4* __restrict__ pin, float4* __restrict__ partial,
                                                        int64_t N, pk_partition part) {
-    __shared__ float4 sh[2 * kTile];
+    __shared__ float4 sh[kTile];  // kTile / 2 source pairs: (x0,x1,y0,y1), (z0,z1,m0,m1)
     const int64_t nb = part.max[0] - part.min[0];
     const int64_t nitems = nb * kSplit;
-    for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
-    const int64_t bx = part.min[0] + it % nb;  // Eq. 8
-    const int s_part = (int)(it / nb);
-    const int64_t base = bx * (int64_t)kBodies * blockDim.x;
-    float4 pi[kBodies];
-#pragma unroll
-    for (int u = 0; u < kBodies; ++u) {
-        const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
-        pi[u] = i < N ? pin[i] : make_float4(0.f, 0.f, 0.f, 0.f);
-    }
-    u64 px[2], py[2], pz[2], ax[2], ay[2], az[2];
     const u64 zero = pk2(0.f, 0.f), eps = pk2(kEps2, kEps2);
+    for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
+        const int64_t bx = part.min[0] + it % nb;  // Eq. 8
+        const int s_part = (int)(it / nb);
+        const int64_t base = bx * (int64_t)kBodies * blockDim.x;
+        u64 px[kBodies], py[kBodies], pz[kBodies], ax[kBodies], ay[kBodies], az[kBodies];
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        px[h] = pk2(pi[2 * h].x, pi[2 * h + 1].x);
-        py[h] = pk2(pi[2 * h].y, pi[2 * h + 1].y);
-        pz[h] = pk2(pi[2 * h].z, pi[2 * h + 1].z);
-        ax[h] = ay[h] = az[h] = zero;
-    }
-    int64_t cb, ce;
-    part_chunks(N, s_part, cb, ce);
-    for (int64_t c0 = cb; c0 < ce; c0 += kChunk) {
-        u64 sx[2] = {zero, zero}, sy[2] = {zero, zero}, sz[2] = {zero, zero};
-        const int64_t c1 = c0 + kChunk < N ? c0 + kChunk : N;
-        for (int64_t t0 = c0; t0 < c1; t0 += kTile) {
-            __syncthreads();
-            for (int s = threadIdx.x; s < kTile; s += blockDim.x) {
-                const int64_t j = t0 + s;
-                const float4 q = j < c1 ? pin[j] : make_float4(0.f, 0.f, 0.f, 0.f);  // m = 0 pads add 0
-                sh[2 * s] = make_float4(q.x, q.x, q.y, q.y);
-                sh[2 * s + 1] = make_float4(q.z, q.z, q.w, q.w);
-            }
-            __syncthreads();
+        for (int u = 0; u < kBodies; ++u) {
+            const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
+            const float4 p = i < N ? pin[i] : make_float4(0.f, 0.f, 0.f, 0.f);
+            px[u] = pk2(p.x, p.x);  // broadcast pairs: ptxas uses the scalar .F32 operand form
+            py[u] = pk2(p.y, p.y);
+            pz[u] = pk2(p.z, p.z);
+            ax[u] = ay[u] = az[u] = zero;
+        }
+        int64_t cb, ce;
+        part_chunks(N, s_part, cb, ce);
+        for (int64_t c0 = cb; c0 < ce; c0 += kChunk) {
+            u64 sx[kBodies], sy[kBodies], sz[kBodies];
+#pragma unroll
+            for (int u = 0; u < kBodies; ++u) sx[u] = sy[u] = sz[u] = zero;
+            const int64_t c1 = c0 + kChunk < N ? c0 + kChunk : N;
+            for (int64_t t0 = c0; t0 < c1; t0 += kTile) {
+                __syncthreads();
+                for (int s = threadIdx.x; s < kTile / 2; s += blockDim.x) {
+                    const int64_t j = t0 + 2 * s;
+                    const float4 q0 = j < c1 ? pin[j] : make_float4(0.f, 0.f, 0.f, 0.f);  // m = 0 pads add 0
+                    const float4 q1 = j + 1 < c1 ? pin[j + 1] : make_float4(0.f, 0.f, 0.f, 0.f);
+                    sh[2 * s] = make_float4(q0.x, q1.x, q0.y, q1.y);
+                    sh[2 * s + 1] = make_float4(q0.z, q1.z, q0.w, q1.w);
+                }
+                __syncthreads();
 #pragma unroll 4
-            for (int s = 0; s < kTile; ++s) {
-                const float4 A = sh[2 * s], B = sh[2 * s + 1];
-                const u64 qx = pk2(A.x, A.y), qy = pk2(A.z, A.w), qz = pk2(B.x, B.y), qm = pk2(B.z, B.w);
+                for (int s = 0; s < kTile / 2; ++s) {
+                    const float4 A = sh[2 * s], B = sh[2 * s + 1];
+                    const u64 qx = pk2(A.x, A.y), qy = pk2(A.z, A.w), qz = pk2(B.x, B.y), qm = pk2(B.z, B.w);
 #pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    const u64 dx = sub2(qx, px[h]), dy = sub2(qy, py[h]), dz = sub2(qz, pz[h]);
-                    const u64 r2 = fma2(dx, dx, fma2(dy, dy, fma2(dz, dz, eps)));
-                    const u64 inv = rsqrt2(r2);
-                    const u64 sc = mul2(qm, mul2(mul2(inv, inv), inv));
-                    sx[h] = fma2(dx, sc, sx[h]);
-                    sy[h] = fma2(dy, sc, sy[h]);
-                    sz[h] = fma2(dz, sc, sz[h]);
+                    for (int u = 0; u < kBodies; ++u) {
+                        const u64 dx = sub2(qx, px[u]), dy = sub2(qy, py[u]), dz = sub2(qz, pz[u]);
+                        const u64 r2 = fma2(dx, dx, fma2(dy, dy, fma2(dz, dz, eps)));
+                        const u64 inv = rsqrt2(r2);
+                        const u64 sc = mul2(qm, mul2(mul2(inv, inv), inv));
+                        sx[u] = fma2(dx, sc, sx[u]);
+                        sy[u] = fma2(dy, sc, sy[u]);
+                        sz[u] = fma2(dz, sc, sz[u]);
+                    }
                 }
             }
+#pragma unroll
+            for (int u = 0; u < kBodies; ++u) {
+                ax[u] = add2(ax[u], sx[u]);
+                ay[u] = add2(ay[u], sy[u]);
+                az[u] = add2(az[u], sz[u]);
+            }
         }
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            ax[h] = add2(ax[h], sx[h]);
-            ay[h] = add2(ay[h], sy[h]);
-            az[h] = add2(az[h], sz[h]);
+        for (int u = 0; u < kBodies; ++u) {
+            const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
+            if (i >= N) continue;
+            float a0, a1, b0, b1, c0_, c1_;
+            up2(ax[u], a0, a1);
+            up2(ay[u], b0, b1);
+            up2(az[u], c0_, c1_);
+            partial[(int64_t)s_part * N + i] = make_float4(a0 + a1, b0 + b1, c0_ + c1_, 0.f);
         }
-    }
-#pragma unroll
-    for (int u = 0; u < kBodies; ++u) {
-        const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
-        if (i >= N) continue;
-        float a0, a1, b0, b1, c0_, c1_;
-        up2(ax[u / 2], a0, a1);
-        up2(ay[u / 2], b0, b1);
-        up2(az[u / 2], c0_, c1_);
-        partial[(int64_t)s_part * N + i] =
-            make_float4((u & 1) ? a1 : a0, (u & 1) ? b1 : b0, (u & 1) ? c1_ : c0_, 0.f);
-    }
-    __syncthreads();  // the next item reuses the shared-memory tile
+        __syncthreads();  // the next item reuses the shared-memory tile
     }
 }
 
