@@ -103,7 +103,7 @@ __device__ __forceinline__ void part_chunks(int64_t N, int s, int64_t& c_begin, 
 // FFMA2 take as a free broadcast operand; each body accumulates two interleaved
 // partial sums (even and odd sources) that are added at the end -- a fixed,
 // position-only order.
-__global__ void __launch_bounds__(256) k_nbody_partial(const float4* __restrict__ pin, float4* __restrict__ partial,
+__global__ void __launch_bounds__(256, 3) k_nbody_partial(const float4* __restrict__ pin, float4* __restrict__ partial,
                                                        int64_t N, pk_partition part) {
     __shared__ float4 sh[kTile];  // kTile / 2 source pairs: (x0,x1,y0,y1), (z0,z1,m0,m1)
     const int64_t nb = part.max[0] - part.min[0];
