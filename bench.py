@@ -467,6 +467,9 @@ def main():
                       "analytic_min_bytes": w.stale_min(P) * args.steps, "copies": int(st["copies"])},
         "host_us_per_launch": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"]
                                + st["host_ns_issue"] + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
+        "host_us_per_launch_phases": {k: st["host_ns_" + k] / 1e3 / max(1, st["launches"])
+                                      for k in ("partition", "regions", "plan", "issue", "update")},
+        "us_per_launch": elapsed_ms * 1e3 / max(1, w.iters * args.steps),
     })
 
     # ---- alpha / beta / gamma (§9.2) ----

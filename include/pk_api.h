@@ -127,6 +127,15 @@ int pk_copy_from_host(pk_ctx ctx, pk_buf buf, const void* host, size_t bytes);
 /* cudaMemcpy(DeviceToHost) replacement: n:1 gather, one copy per tracker segment
  * from a partition holding it (§8.2).  Blocking. */
 int pk_sync_to_host(pk_ctx ctx, pk_buf buf, void* host, size_t bytes);
+/* Read-pattern-aware H2D (the paper's linear distribution is
+ * "hoping that this pattern matches the read pattern of the following kernels",
+ * P:L888-895, and its mismatch limits Matmul scaling): every
+ * partition receives, straight from the host, the bytes its partition of the
+ * given launch (kernel, grid, block, scalars) reads through argument `arg_index`;
+ * bytes nobody reads go linearly as in pk_copy_from_host.  Partitions that
+ * receive the same bytes all become holders.  Blocking w.r.t. host memory. */
+int pk_copy_from_host_for(pk_ctx ctx, pk_buf buf, const void* host, size_t bytes, pk_kernel k, int arg_index,
+                          const int32_t grid[3], const int32_t block[3], const int64_t* scalars, int nscalars);
 /* cudaFree replacement.  Library-owned instances are freed after pending work. */
 int pk_unregister_buffer(pk_ctx ctx, pk_buf buf);
 /* Device pointer of partition `part`'s instance (tests / caller-side kernels). */

@@ -45,6 +45,21 @@ class ShadowBuffer:
         for p in range(P):
             self.mask[(p * n) // P:((p + 1) * n) // P] = np.uint64(1 << p)
 
+    def h2d_for(self, read_sets):
+        """Read-pattern-aware upload (SURVEY NEXT-1 of P:L888-895): element e goes to
+        every partition whose read set contains it; unread elements keep the linear slab."""
+        n, P = self.nelem, self.nparts
+        m = np.zeros(n, dtype=np.uint64)
+        for p, r in enumerate(read_sets):
+            if r is not None and len(r):
+                m[np.asarray(r, dtype=np.int64)] |= np.uint64(1 << p)
+        for p in range(P):
+            sl = slice((p * n) // P, ((p + 1) * n) // P)
+            part = m[sl]
+            part[part == 0] = np.uint64(1 << p)
+            m[sl] = part
+        self.mask = m
+
     def rle(self):
         """Canonical (begin_byte, end_byte, mask) runs covering the buffer."""
         m = self.mask

@@ -107,6 +107,8 @@ def lib():
         "pk_register_buffer": [C.c_void_p, C.c_int, _I64P, C.c_int, C.POINTER(C.c_void_p), C.c_void_p, _I64P],
         "pk_copy_from_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
         "pk_sync_to_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
+        "pk_copy_from_host_for": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t, C.c_int64, C.c_int, _I32P, _I32P,
+                                  _I64P, C.c_int],
         "pk_unregister_buffer": [C.c_void_p, C.c_int64],
         "pk_buffer_instance": [C.c_void_p, C.c_int64, C.c_int, C.POINTER(C.c_void_p)],
         "pk_register_kernel": [C.c_void_p, C.c_char_p, C.c_void_p, C.c_int, _I32P, C.c_int32, _I64P],
@@ -224,6 +226,14 @@ def pk_register_buffer(ctx, shape, elem_bytes, dev_ptrs=None, host_init=None, np
 def pk_copy_from_host(ctx, buf, host, nbytes=None):
     _check(lib().pk_copy_from_host(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
            "pk_copy_from_host")
+
+
+def pk_copy_from_host_for(ctx, buf, host, kernel, arg_index, grid, block, scalars=(), nbytes=None):
+    """Read-pattern-aware H2D: each partition receives what `kernel`'s launch reads via `arg_index`."""
+    sc = list(scalars)
+    _check(lib().pk_copy_from_host_for(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host),
+                                       kernel, arg_index, _i32(grid), _i32(block), _i64(sc), len(sc)),
+           "pk_copy_from_host_for")
 
 
 def pk_sync_to_host(ctx, buf, host, nbytes=None):

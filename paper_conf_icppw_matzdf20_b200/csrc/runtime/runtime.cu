@@ -590,6 +590,62 @@ int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
     return PK_OK;
 }
 
+int pk_copy_from_host_for(pk_ctx c, pk_buf b, const void* host, size_t bytes, pk_kernel k, int arg,
+                          const int32_t grid[3], const int32_t block[3], const int64_t* scalars, int ns) {
+    if (!valid_buf(c, b) || !host || !valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
+    if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
+    Buffer& B = c->bufs[b];
+    if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (H2D copies the whole virtual buffer)");
+    const Kernel& K = c->kernels[k];
+    if (arg < 0 || arg >= K.nargs || K.kinds[arg] != PK_ARG_BUFFER) return fail(PK_ERR_INVALID, "bad arg index");
+    const int P = c->P;
+    const int w = split_dim(grid, K.partition_dim);
+    EvalEnv env{scalars, ns, {block[0], block[1], block[2]}};
+    std::vector<RangeList> U(P);
+    RangeList covered;
+    for (int p = 0; p < P; ++p) {
+        int64_t box[6];
+        partition_box(grid, P, p, w, box);
+        if (box_empty(box)) continue;
+        Status st = arg_ranges(K, arg, PK_READ, box, B, env, &U[p]);
+        if (!st.ok()) return fail(st);
+        covered = union_ranges(covered, U[p]);
+    }
+    // bytes nobody reads keep the linear distribution
+    const uint64_t n = B.bytes / B.eb;
+    for (int p = 0; p < P; ++p) {
+        const uint64_t lo = (uint64_t)p * n / P * B.eb, hi = (uint64_t)(p + 1) * n / P * B.eb;
+        uint64_t cur = lo;
+        RangeList extra;
+        for (const Range& r : covered) {
+            if (r.e <= cur) continue;
+            if (r.b >= hi) break;
+            if (r.b > cur) extra.push_back(Range{cur, std::min(r.b, hi)});
+            cur = std::max(cur, r.e);
+            if (cur >= hi) break;
+        }
+        if (cur < hi) extra.push_back(Range{cur, hi});
+        if (!extra.empty()) U[p] = union_ranges(U[p], extra);
+    }
+    if (!c->host_only) {
+        if (int r = pk_synchronize(c)) return r;
+        for (int p = 0; p < P; ++p) {
+            if (!c->local(p)) continue;
+            if (int r = c->set_device(c->dev[p])) return r;
+            for (const Range& r : U[p])
+                PK_CUDA(cudaMemcpyAsync((char*)B.inst[p] + r.b, (const char*)host + r.b, r.e - r.b,
+                                        cudaMemcpyHostToDevice, c->stream[p]));
+        }
+        if (int r = pk_synchronize(c)) return r;
+        for (int p = 0; p < P; ++p) { B.last_writer[p] = W_NONE; B.readers[p] = 0; }
+    }
+    B.tracker.init(B.bytes, 0);
+    for (int p = 0; p < P; ++p)
+        if (!U[p].empty()) B.tracker.add_bit(U[p], p);
+    for (int p = 0; p < P; ++p) c->stats.h2d_bytes += total_bytes(U[p]);
+    return PK_OK;
+}
+
 static int sync_to_host_spmd(pk_ctx c, Buffer& B, void* host) {
     // collective n:1 gather to rank 0: segments rank 0's partition lacks are sent
     // by their lowest holder straight into rank 0's instance, which then holds them

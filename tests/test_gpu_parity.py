@@ -299,3 +299,22 @@ def test_gemm_oracle_and_bitwise(m, n, k):
         gp, st = _gemm(a, b, P)
         assert np.array_equal(g1, gp), P
         assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def test_gemm_read_pattern_placement_moves_nothing():
+    """NEXT-1: operands uploaded where the launch reads them (pk_copy_from_host_for)."""
+    m, n, k = 768, 512, 256
+    a, b = synth.gemm_operands(m, n, k)
+    ref, _ = _gemm(a, b, 1)
+    ctx = gpu_ctx(3)
+    pr = K.Problem(ctx, "sgemm_tf32x3")
+    ab, bb, cb = pr.buffer((m, k), 4), pr.buffer((k, n), 4), pr.buffer((m, n), 4)
+    grid, blk, sc = K.sgemm_launch(m, n, k)
+    abi.pk_copy_from_host_for(ctx, ab, a, pr.k, 0, grid, blk, sc)
+    abi.pk_copy_from_host_for(ctx, bb, b, pr.k, 1, grid, blk, sc)
+    pr.launch(grid, blk, [ab, bb, cb, m, n, k], sc)
+    g = fetch(ctx, cb, (m, n))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, ref)
+    assert st["stale_bytes"] == 0 == st["moved_bytes"]

@@ -419,3 +419,38 @@ def test_gemm_b_broadcast_stale_bytes():
     # matches the row partition; the second launch moves nothing (validity map, Q4)
     assert s["stale_bytes"] == cf.gemm_stale(k, n, P)
     abi.pk_finalize(ctx)
+
+
+# ------------------------------------------------------------ read-pattern-aware placement (NEXT-1)
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_placement_for_gemm_b_and_hotspot_halo(P):
+    # GEMM: B placed where the launch reads it -> the launch moves nothing
+    m, n, k = 768, 256, 256                  # 6 row tiles: no empty partition for P <= 4
+    ctx = host_ctx(P)
+    pr = K.Problem(ctx, "sgemm_tf32x3")
+    a = pr.buffer((m, k), 4)
+    b = pr.buffer((k, n), 4)
+    c = pr.buffer((m, n), 4)
+    grid, blk, sc = K.sgemm_launch(m, n, k)
+    abi.pk_copy_from_host_for(ctx, a, np.zeros((m, k), np.float32), pr.k, 0, grid, blk, sc)
+    abi.pk_copy_from_host_for(ctx, b, np.zeros((k, n), np.float32), pr.k, 1, grid, blk, sc)
+    assert abi.pk_tracker_dump(ctx, b) == [(0, k * n * 4, (1 << P) - 1)]
+    pr.launch(grid, blk, [a, b, c, m, n, k], sc)
+    assert abi.pk_get_stats(ctx)["stale_bytes"] == 0
+    abi.pk_finalize(ctx)
+    # Hotspot: halo rows land on both neighbours; tracker == shadow oracle; first launch moves nothing
+    h, w = 40, 1100
+    ctx = host_ctx(P)
+    geom = K.hotspot2d_launch(h, w, 4, 128)
+    pr = K.Problem(ctx, "hotspot2d")
+    t0 = pr.buffer((h, w), 4)
+    t1 = pr.buffer((h, w), 4)
+    pw = pr.buffer((h, w), 4)
+    abi.pk_copy_from_host_for(ctx, t0, np.zeros((h, w), np.float32), pr.k, 0, *geom)
+    sb = shadow.ShadowBuffer(h * w, 4, P)
+    sb.h2d_for([regions.hotspot2d(og.partition_box(geom[0], P, p), geom[1], h, w, 4)[(0, "r")]
+                for p in range(P)])
+    assert abi.pk_tracker_dump(ctx, t0) == sb.rle()
+    pr.launch(geom[0], geom[1], [t0, pw, t1, h, w, 4], geom[2])
+    assert abi.pk_get_stats(ctx)["stale_bytes"] == 0
+    abi.pk_finalize(ctx)
