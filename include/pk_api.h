@@ -278,6 +278,8 @@ typedef struct {
     double kernel_ms;            /* sum over partition kernels (PK_MODE_TIME_KERNELS) */
     double kernel_ms_max_launch; /* per launch: max over partitions, summed */
     uint64_t timed_kernels;      /* kernels included in kernel_ms */
+    uint64_t graph_replays;      /* launches served by steady-state graph replay */
+    uint64_t graph_captures;     /* launches captured into a replay graph */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);
@@ -288,8 +290,17 @@ enum {
     PK_MODE_NO_TRANSFERS = 1u << 1,  /* beta of §9.2: resolve + track, do not copy */
     PK_MODE_NO_TRACKING = 1u << 2,   /* gamma of §9.2: no resolution, no tracker, no copies */
     PK_MODE_GLOBAL_BARRIER = 1u << 3,/* literal all_devs_synchronize() between sync and launch (Fig. 4 l. 8) */
-    PK_MODE_TIME_KERNELS = 1u << 4   /* CUDA events around every partition kernel -> pk_stats.kernel_ms */
+    PK_MODE_TIME_KERNELS = 1u << 4,  /* CUDA events around every partition kernel -> pk_stats.kernel_ms */
+    PK_MODE_NO_GRAPHS = 1u << 5      /* disable steady-state graph replay (see pk_launch_partitioned) */
 };
+/* Steady-state replay: when a launch repeats with the same kernel, bindings, geometry,
+ * scalars, mode and pre-launch tracker states of its buffers (e.g. the second sweep of
+ * a ping-pong pair), the library captures its copies + partition kernels once into a
+ * multi-stream (multi-device) CUDA graph and afterwards replays the graph and restores
+ * the memoised post-launch tracker states instead of re-planning and re-issuing every
+ * CUDA call -- the host overhead the paper measures as "patterns".
+ * Active for single-process contexts with more than one local partition, unless
+ * PK_MODE_TIME_KERNELS, PK_MODE_GLOBAL_BARRIER or PK_MODE_NO_GRAPHS is set. */
 int pk_set_mode(pk_ctx ctx, uint32_t flags);
 uint32_t pk_get_mode(pk_ctx ctx);
 

@@ -72,6 +72,13 @@ public:
     void init(uint64_t size, uint64_t mask);
     uint64_t size() const { return size_; }
     const std::vector<Seg>& segments() const { return segs_; }
+    void set_segments(const std::vector<Seg>& s) { segs_ = s; }  // restore a memoised state
+    uint64_t fingerprint() const {                                 // FNV-1a over the segments
+        uint64_t h = 1469598103934665603ull;
+        for (const Seg& s : segs_)
+            for (uint64_t v : {s.b, s.e, s.mask}) { h ^= v; h *= 1099511628211ull; }
+        return h;
+    }
     // Visit the pieces of [b,e) with their masks, in order.
     template <class F>
     void query(uint64_t b, uint64_t e, F&& f) const;

@@ -172,7 +172,20 @@ struct pk_ctx_s {
     cudaEvent_t timer_start = nullptr, timer_stop = nullptr;
     bool timer_running = false;
     int first_local = -1;    // lowest partition owned by this rank
+    int nlocal = 0;          // partitions owned by this rank
     void* comm = nullptr;    // ncclComm_t (SPMD only)
+    // steady-state graph replay (pk_api.h, PK_MODE_NO_GRAPHS)
+    struct Memo {
+        int seen = 0;
+        cudaGraphExec_t exec = nullptr;
+        std::vector<std::pair<int64_t, std::vector<Seg>>> post;  // tracker states after the launch
+        std::vector<CopyOp> plan;
+        pk_stats delta{};
+    };
+    std::unordered_map<std::string, Memo> memo;
+    bool graph_mode = false;  // all work is ordered on stream[first_local]
+    cudaEvent_t ev_fork = nullptr;
+    std::vector<cudaEvent_t> ev_join;
 
     bool local(int p) const { return prank[p] == rank; }
     int set_device(int d) {
@@ -308,7 +321,10 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
     }
     c->first_local = -1;
     for (int p = 0; p < c->P; ++p)
-        if (c->local(p)) { c->first_local = p; break; }
+        if (c->local(p)) {
+            if (c->first_local < 0) c->first_local = p;
+            c->nlocal++;
+        }
     if (!c->host_only) {
         int nlocal = 0;
         for (int p = 0; p < c->P; ++p) nlocal += c->local(p);
@@ -345,14 +361,19 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
         c->ev_kernel.resize(c->P);
         c->ev_copy.resize(c->P);
         c->event_pool.resize(c->P);
+        c->ev_join.assign(c->P, nullptr);
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
             PK_CUDA(cudaSetDevice(c->dev[p]));
             PK_CUDA(cudaStreamCreateWithFlags(&c->stream[p], cudaStreamNonBlocking));
             PK_CUDA(cudaEventCreateWithFlags(&c->ev_kernel[p], cudaEventDisableTiming));
             PK_CUDA(cudaEventCreateWithFlags(&c->ev_copy[p], cudaEventDisableTiming));
+            PK_CUDA(cudaEventCreateWithFlags(&c->ev_join[p], cudaEventDisableTiming));
             c->cur_device = c->dev[p];
         }
+        PK_CUDA(cudaSetDevice(c->dev[c->first_local]));
+        PK_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+        c->cur_device = c->dev[c->first_local];
         if (c->world > 1) {
             const NcclApi& n = nccl();
             if (!n.ok) return fail(PK_ERR_NCCL, "libnccl.so.2 could not be loaded (set PK_NCCL_LIB)");
@@ -367,6 +388,14 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
     return PK_OK;
 }
 
+static void clear_hazards(pk_ctx c) {
+    for (Buffer& B : c->bufs)
+        if (B.alive) {
+            std::fill(B.last_writer.begin(), B.last_writer.end(), (uint8_t)W_NONE);
+            std::fill(B.readers.begin(), B.readers.end(), 0ull);
+        }
+}
+
 int pk_synchronize(pk_ctx c) {
     if (!c) return fail(PK_ERR_INVALID, "null ctx");
     if (c->host_only) return PK_OK;
@@ -375,7 +404,50 @@ int pk_synchronize(pk_ctx c) {
         if (int r = c->set_device(c->dev[p])) return r;
         PK_CUDA(cudaStreamSynchronize(c->stream[p]));
     }
+    // nothing is in flight any more: event hazards and graph mode are void
+    c->graph_mode = false;
+    clear_hazards(c);
     return PK_OK;
+}
+
+// Graph mode: every partition stream's tail is joined into stream[p0] so that a
+// replayed graph (launched on p0, forking to the other streams internally) is
+// ordered after everything enqueued before it.
+static int enter_graph_mode(pk_ctx c) {
+    if (c->graph_mode) return PK_OK;
+    const int p0 = c->first_local;
+    for (int p = 0; p < c->P; ++p) {
+        if (!c->local(p) || p == p0) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        PK_CUDA(cudaEventRecord(c->ev_join[p], c->stream[p]));
+        if (int r = c->set_device(c->dev[p0])) return r;
+        PK_CUDA(cudaStreamWaitEvent(c->stream[p0], c->ev_join[p], 0));
+    }
+    c->graph_mode = true;
+    clear_hazards(c);  // stream order on p0 now covers every hazard
+    return PK_OK;
+}
+
+// Leave graph mode before eager work: every stream waits for p0's tail.
+static int exit_graph_mode(pk_ctx c) {
+    if (!c->graph_mode) return PK_OK;
+    const int p0 = c->first_local;
+    if (int r = c->set_device(c->dev[p0])) return r;
+    PK_CUDA(cudaEventRecord(c->ev_fork, c->stream[p0]));
+    for (int p = 0; p < c->P; ++p) {
+        if (!c->local(p) || p == p0) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_fork, 0));
+    }
+    c->graph_mode = false;
+    clear_hazards(c);
+    return PK_OK;
+}
+
+static void clear_memo(pk_ctx c) {
+    for (auto& kv : c->memo)
+        if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+    c->memo.clear();
 }
 
 int pk_timer_begin(pk_ctx c) {
@@ -455,14 +527,17 @@ int pk_finalize(pk_ctx c) {
                 for (int p = 0; p < c->P; ++p)
                     if (B.inst[p]) { cudaSetDevice(c->dev[p]); cudaFree(B.inst[p]); }
         }
+        clear_memo(c);
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
             cudaSetDevice(c->dev[p]);
             cudaStreamDestroy(c->stream[p]);
             cudaEventDestroy(c->ev_kernel[p]);
             cudaEventDestroy(c->ev_copy[p]);
+            cudaEventDestroy(c->ev_join[p]);
             for (cudaEvent_t e : c->event_pool[p]) cudaEventDestroy(e);
         }
+        if (c->ev_fork) { cudaSetDevice(c->dev[c->first_local]); cudaEventDestroy(c->ev_fork); }
         if (c->comm) nccl().CommDestroy(c->comm);
         if (c->timer_start) {
             cudaSetDevice(c->dev[c->first_local]);
@@ -538,8 +613,11 @@ int pk_buffer_instance(pk_ctx c, pk_buf b, int part, void** dev_ptr) {
 int pk_unregister_buffer(pk_ctx c, pk_buf b) {
     if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "bad buffer");
     Buffer& B = c->bufs[b];
-    if (!c->host_only && B.owned) {
+    if (!c->host_only) {
         if (int r = pk_synchronize(c)) return r;
+        clear_memo(c);  // replay graphs may reference the instances
+    }
+    if (!c->host_only && B.owned) {
         for (int p = 0; p < c->P; ++p)
             if (B.inst[p]) {
                 if (int r = c->set_device(c->dev[p])) return r;
@@ -697,6 +775,8 @@ int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
     if (c->host_only) return fail(PK_ERR_STATE, "host-only context holds no data");
     if (!host && (c->world == 1 || c->rank == 0)) return fail(PK_ERR_INVALID, "null host buffer");
     if (c->world > 1) return sync_to_host_spmd(c, B, host);
+    // replay graphs run on stream[p0]: fork the other streams from its tail first
+    if (int r = exit_graph_mode(c)) return r;
     // query all segments, copy each from a partition that holds it.
     struct Piece { uint64_t b, e; int src; };
     std::vector<Piece> pieces;
@@ -823,15 +903,139 @@ int pk_reset_stats(pk_ctx c) {
 
 int pk_set_mode(pk_ctx c, uint32_t flags) {
     if (!c) return fail(PK_ERR_INVALID, "bad argument");
-    if (flags & ~0x1Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
+    if (flags & ~0x3Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
     c->mode = flags;
     return PK_OK;
 }
 uint32_t pk_get_mode(pk_ctx c) { return c ? c->mode : 0; }
 
 // ------------------------------------------------------------------ Fig. 4
+static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
+                        const void* const* args, const int64_t* scalars, int ns);
+
+static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
+    a.launches += sign * d.launches;
+    a.kernel_launches += sign * d.kernel_launches;
+    a.copies += sign * d.copies;
+    a.stale_bytes += sign * d.stale_bytes;
+    a.moved_bytes += sign * d.moved_bytes;
+    for (int i = 0; i < 16; ++i)
+        for (int j = 0; j < 16; ++j) a.pair_bytes[i][j] += sign * d.pair_bytes[i][j];
+}
+
 int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
                           const void* const* args, const int64_t* scalars, int ns) {
+    if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
+    if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
+    const Kernel& K = c->kernels[k];
+    const uint32_t mode = c->mode;
+    // builtin launchers take every scalar from `scalars`, so the key below captures the launch
+    const bool can_graph = !c->host_only && c->world == 1 && c->nlocal > 1 && K.nargs && args && K.launcher &&
+                           !(mode & (PK_MODE_TIME_KERNELS | PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
+    if (!can_graph) {
+        if (!c->host_only)
+            if (int r = exit_graph_mode(c)) return r;
+        return launch_eager(c, k, grid, block, smem, args, scalars, ns);
+    }
+    // ---- memo key: launch identity + pre-launch tracker state of every bound buffer ----
+    uint64_t t0 = now_ns();
+    std::string key;
+    key.reserve(256);
+    auto put = [&key](const void* p, size_t n) { key.append((const char*)p, n); };
+    put(&k, sizeof k);
+    put(&K.version, sizeof K.version);
+    put(grid, 12);
+    put(block, 12);
+    put(&smem, sizeof smem);
+    put(&mode, sizeof mode);
+    put(&ns, sizeof ns);
+    if (ns) put(scalars, sizeof(int64_t) * ns);
+    std::vector<int64_t> bids;
+    for (int a = 0; a < K.nargs; ++a) {
+        if (K.kinds[a] == PK_ARG_BUFFER) {
+            if (!args[a]) return fail(PK_ERR_INVALID, "null buffer argument");
+            const pk_buf b = *(const pk_buf*)args[a];
+            if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "argument " + std::to_string(a) + " is not a live buffer");
+            put(&b, sizeof b);
+            if (std::find(bids.begin(), bids.end(), b) == bids.end()) bids.push_back(b);
+        }
+    }
+    for (int64_t b : bids) {
+        const uint64_t f = c->bufs[b].tracker.fingerprint();
+        put(&f, sizeof f);
+    }
+    auto it = c->memo.find(key);
+    if (it != c->memo.end() && it->second.exec) {
+        // ---- replay: one graph launch + restore the memoised tracker states ----
+        pk_ctx_s::Memo& m = it->second;
+        if (int r = enter_graph_mode(c)) return r;
+        if (int r = c->set_device(c->dev[c->first_local])) return r;
+        PK_CUDA(cudaGraphLaunch(m.exec, c->stream[c->first_local]));
+        for (auto& ps : m.post) c->bufs[ps.first].tracker.set_segments(ps.second);
+        c->last_plan = m.plan;
+        add_stats(c->stats, m.delta, 1);
+        c->stats.graph_replays += 1;
+        c->launch_counter++;
+        c->stats.host_ns_issue += now_ns() - t0;
+        return PK_OK;
+    }
+    const bool capture = it != c->memo.end() && it->second.seen >= 1;
+    pk_stats before = c->stats;
+    int rc;
+    if (!capture) {
+        if (int r = exit_graph_mode(c)) return r;
+        rc = launch_eager(c, k, grid, block, smem, args, scalars, ns);
+        if (rc) return rc;
+    } else {
+        // ---- capture the launch once into a multi-stream graph ----
+        if (int r = enter_graph_mode(c)) return r;
+        const int p0 = c->first_local;
+        if (int r = c->set_device(c->dev[p0])) return r;
+        PK_CUDA(cudaStreamBeginCapture(c->stream[p0], cudaStreamCaptureModeRelaxed));
+        cudaError_t ce = cudaEventRecord(c->ev_fork, c->stream[p0]);
+        for (int p = 0; p < c->P && ce == cudaSuccess; ++p)
+            if (c->local(p) && p != p0) {
+                c->set_device(c->dev[p]);
+                ce = cudaStreamWaitEvent(c->stream[p], c->ev_fork, 0);
+            }
+        rc = ce == cudaSuccess ? launch_eager(c, k, grid, block, smem, args, scalars, ns)
+                               : fail(PK_ERR_CUDA, std::string("graph fork: ") + cudaGetErrorName(ce));
+        for (int p = 0; p < c->P && rc == PK_OK; ++p)
+            if (c->local(p) && p != p0) {
+                c->set_device(c->dev[p]);
+                ce = cudaEventRecord(c->ev_join[p], c->stream[p]);
+                c->set_device(c->dev[p0]);
+                if (ce == cudaSuccess) ce = cudaStreamWaitEvent(c->stream[p0], c->ev_join[p], 0);
+                if (ce != cudaSuccess) rc = fail(PK_ERR_CUDA, std::string("graph join: ") + cudaGetErrorName(ce));
+            }
+        c->set_device(c->dev[p0]);
+        cudaGraph_t g = nullptr;
+        cudaError_t ee = cudaStreamEndCapture(c->stream[p0], &g);
+        clear_hazards(c);  // events recorded during capture are graph nodes, not real records
+        if (rc) { if (g) cudaGraphDestroy(g); return rc; }
+        if (ee != cudaSuccess) return fail(PK_ERR_CUDA, std::string("cudaStreamEndCapture: ") + cudaGetErrorName(ee));
+        cudaGraphExec_t ex = nullptr;
+        ee = cudaGraphInstantiate(&ex, g, 0);
+        cudaGraphDestroy(g);
+        if (ee != cudaSuccess) return fail(PK_ERR_CUDA, std::string("cudaGraphInstantiate: ") + cudaGetErrorName(ee));
+        PK_CUDA(cudaGraphLaunch(ex, c->stream[p0]));
+        if (c->memo.size() > 256) clear_memo(c);
+        c->memo[key].exec = ex;
+        c->stats.graph_captures += 1;
+    }
+    pk_ctx_s::Memo& m = c->memo[key];
+    m.seen += 1;
+    m.plan = c->last_plan;
+    m.delta = c->stats;
+    add_stats(m.delta, before, -1);
+    m.delta.graph_replays = m.delta.graph_captures = 0;
+    m.post.clear();
+    for (int64_t b : bids) m.post.emplace_back(b, c->bufs[b].tracker.segments());
+    return PK_OK;
+}
+
+static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
+                        const void* const* args, const int64_t* scalars, int ns) {
     if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
     if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
     const Kernel& K = c->kernels[k];

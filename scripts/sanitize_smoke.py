@@ -1,0 +1,44 @@
+"""Small invocation of every builtin kernel (P = 2 virtual partitions) for compute-sanitizer.
+
+    compute-sanitizer --tool memcheck python scripts/sanitize_smoke.py
+    compute-sanitizer --tool racecheck python scripts/sanitize_smoke.py
+"""
+import sys
+
+import numpy as np
+
+sys.path.insert(0, ".")
+import synth  # noqa: E402
+from paper_conf_icppw_matzdf20_b200 import abi  # noqa: E402
+from paper_conf_icppw_matzdf20_b200 import kernels as K  # noqa: E402
+
+
+def main():
+    P = 2
+    ctx = abi.pk_init(P, part_device=[0] * P)
+    u = synth.jacobi_grid(70, 90)
+    _, jb = K.jacobi2d_program(ctx, u, 3)
+    t, p = synth.hotspot_grids(150, 1100)
+    pr = K.hotspot2d_setup(ctx, t, p, ty=16)
+    hb = K.hotspot2d_iterate(pr, 3)
+    pr2 = K.hotspot2d_setup(ctx, t, p, ty=16, bdx=64, kernel="hotspot2d_regs")
+    K.hotspot2d_iterate(pr2, 2)
+    h = synth.heat_grid(20, 70, 260)
+    ph = K.heat3d_setup(ctx, h, zc=8, bdy=61)
+    K.heat3d_iterate(ph, 3)
+    ph2 = K.heat3d_setup(ctx, h, zc=8, bdy=8, kernel="heat3d_regs")
+    K.heat3d_iterate(ph2, 2)
+    pos, vel = synth.nbody_bodies(3000)
+    pn = K.nbody_setup(ctx, pos, vel)
+    K.nbody_iterate(pn, 2)
+    a, b = synth.gemm_operands(300, 520, 200)
+    _, cb = K.sgemm_program(ctx, a, b)
+    out = np.empty((300, 520), np.float32)
+    abi.pk_sync_to_host(ctx, cb, out)
+    abi.pk_synchronize(ctx)
+    abi.pk_finalize(ctx)
+    print("sanitize smoke done", float(out[0, 0]))
+
+
+if __name__ == "__main__":
+    main()

@@ -318,3 +318,38 @@ def test_gemm_read_pattern_placement_moves_nothing():
     abi.pk_finalize(ctx)
     assert np.array_equal(g, ref)
     assert st["stale_bytes"] == 0 == st["moved_bytes"]
+
+
+# ------------------------------------------------------------------ steady-state graph replay
+@pytest.mark.parametrize("P", [2, 4])
+def test_graph_replay_matches_eager_and_one_way(P):
+    t, p = synth.hotspot_grids(256, 1024)
+    iters = 24
+    ref, _ = _hotspot(t, p, iters, 1)
+    ge, se = _hotspot(t, p, iters, P, mode=abi.PK_MODE_NO_GRAPHS)
+    gg, sg = _hotspot(t, p, iters, P)
+    assert np.array_equal(ge, ref) and np.array_equal(gg, ref)
+    assert se["graph_replays"] == 0 and sg["graph_replays"] >= iters - 6 and sg["graph_captures"] >= 1
+    for key in ("stale_bytes", "moved_bytes", "copies", "kernel_launches", "launches"):
+        assert se[key] == sg[key], key
+
+
+def test_graph_mode_interleaved_with_eager_work():
+    """Graph replay, then a re-upload (H2D), eager launches (mode switch) and more replay."""
+    h, w = 200, 1028
+    t, p = synth.hotspot_grids(h, w)
+    ctx = gpu_ctx(3)
+    pr = K.hotspot2d_setup(ctx, t, p, ty=16)
+    K.hotspot2d_iterate(pr, 10)
+    abi.pk_copy_from_host(ctx, pr.tb[0], t)            # restart from the initial field
+    K.hotspot2d_iterate(pr, 6, start=0)
+    abi.pk_set_mode(ctx, abi.PK_MODE_NO_GRAPHS)
+    K.hotspot2d_iterate(pr, 3, start=6)
+    abi.pk_set_mode(ctx, 0)
+    out = K.hotspot2d_iterate(pr, 11, start=9)
+    g = fetch(ctx, out, (h, w))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    ref, _ = _hotspot(t, p, 20, 1)
+    assert np.array_equal(g, ref)
+    assert st["graph_replays"] > 0
