@@ -80,6 +80,22 @@ def hotspot2d(box, block, h, w, ty, vec=4):
     return {(0, READ): _uniq(reads_t), (1, READ): _uniq([c]), (2, WRITE): _uniq([c])}
 
 
+def hotspot2d_tb2(box, block, h, w, ty, vec=4):
+    """Two fused sweeps per launch (hotspot2d_tb2): every owned cell (same tile
+    contract as hotspot2d) reads the clamped 5x5 square of temp_in and the clamped
+    3x3 square of power around it and writes temp_out at the cell."""
+    bdx = block[0]
+    _, bys, bxs = _block_ranges(box)
+    i = (bys[:, None] * ty + np.arange(ty)[None, :]).ravel()
+    j = (bxs[:, None] * (vec * bdx) + np.arange(vec * bdx)[None, :]).ravel()
+    i = i[i < h]
+    j = j[j < w]
+    I, J = np.meshgrid(i, j, indexing="ij")
+    rt = [_ravel(_clamp(I + di, h), _clamp(J + dj, w), (h, w)) for di in range(-2, 3) for dj in range(-2, 3)]
+    rp = [_ravel(_clamp(I + di, h), _clamp(J + dj, w), (h, w)) for di in range(-1, 2) for dj in range(-1, 2)]
+    return {(0, READ): _uniq(rt), (1, READ): _uniq(rp), (2, WRITE): _uniq([_ravel(I, J, (h, w))])}
+
+
 # ---------------------------------------------------------------------------
 # C3 heat3d(u_in, u_out; D, H, W, ZC): block (bdx, bdy); thread owns VEC=4
 #   columns j = bx*4*bdx + 4*tx + v, row i = by*bdy + ty, and marches ZC planes

@@ -41,6 +41,7 @@ LauncherFn find_builtin_launcher(const void* fn);
 extern const Builtin kBuiltinJacobi2d;
 extern const Builtin kBuiltinHotspot2d;     // hotspot2d_regs (register window)
 extern const Builtin kBuiltinHotspot2dTma;  // hotspot2d (TMA bulk ring, default)
+extern const Builtin kBuiltinHotspot2dTb2;  // hotspot2d_tb2 (two sweeps per launch)
 extern const Builtin kBuiltinHeat3d;
 extern const Builtin kBuiltinHeat3dTma;      // heat3d (TMA plane ring, default); kBuiltinHeat3d = heat3d_regs
 extern const Builtin kBuiltinNbody;

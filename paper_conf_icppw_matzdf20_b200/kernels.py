@@ -107,16 +107,22 @@ def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, 
     pr.geom = hotspot2d_launch(h, w, ty, bdx)
     pr.hw = (h, w)
     pr.tb = (t0, t1, pw)
+    pr.sweeps = 2 if kernel == "hotspot2d_tb2" else 1   # time steps per launch
     return pr
 
 
 def hotspot2d_iterate(pr, iters, start=0):
+    """`iters` Hotspot time steps starting at step `start` (the tb2 kernel advances two
+    steps per launch: iters and start must then be even)."""
     (t0, t1, pw), (h, w) = pr.tb, pr.hw
     grid, blk, sc = pr.geom
-    for t in range(start, start + iters):
+    k = pr.sweeps
+    if iters % k or start % k:
+        raise ValueError("hotspot2d_tb2 advances two steps per launch")
+    for t in range(start // k, (start + iters) // k):
         a, b = (t0, t1) if t % 2 == 0 else (t1, t0)
         pr.launch(grid, blk, [a, pw, b, h, w, sc[2]], sc)
-    return t1 if (start + iters) % 2 == 1 else t0
+    return t1 if ((start + iters) // k) % 2 == 1 else t0
 
 
 def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY, kernel="heat3d"):

@@ -106,6 +106,22 @@ def test_hotspot_stale_bytes_closed_form():
         assert st["stale_bytes"] == 10 * cf.hotspot2d_stale_per_iter(w, P) == st["moved_bytes"]
 
 
+@pytest.mark.parametrize("h,w,ty", [(200, 520, 16), (129, 1028, 64), (3, 4, 64), (300, 2048, 7), (64, 1536, 128)])
+def test_hotspot_tb2_oracle_and_bitwise(h, w, ty):
+    """Two fused sweeps per launch (NEXT-3): oracle within 1e-5, P-way bit-identical."""
+    t, p = synth.hotspot_grids(h, w)
+    iters = 20
+    ref = ok.hotspot2d(t, p, iters)
+    g1, s1 = _hotspot(t, p, iters, 1, ty, kernel="hotspot2d_tb2")
+    ok_, err = rel_ok(g1, ref, 1e-5)
+    assert ok_, err
+    assert s1["kernel_launches"] == iters // 2
+    for P in (2, 3, 4, 8):
+        gp, st = _hotspot(t, p, iters, P, ty, kernel="hotspot2d_tb2")
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
 def test_hotspot_uniform_closed_form_on_gpu():
     h, w = 96, 256
     t = np.full((h, w), 323.0, np.float32)

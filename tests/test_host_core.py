@@ -454,3 +454,31 @@ def test_placement_for_gemm_b_and_hotspot_halo(P):
     pr.launch(geom[0], geom[1], [t0, pw, t1, h, w, 4], geom[2])
     assert abi.pk_get_stats(ctx)["stale_bytes"] == 0
     abi.pk_finalize(ctx)
+
+
+# ------------------------------------------------------------ temporally blocked Hotspot (NEXT-3)
+@pytest.mark.parametrize("h,w,ty", [(33, 1100, 4), (200, 1028, 16), (5, 8, 64)])
+@pytest.mark.parametrize("P", [1, 2, 3, 7])
+def test_hotspot_tb2_regions(h, w, ty, P):
+    ctx = host_ctx(P)
+    k = abi.pk_builtin_kernel(ctx, "hotspot2d_tb2")
+    bufs = [abi.pk_register_buffer(ctx, (h, w), 4) for _ in range(3)]
+    grid, blk, sc = K.hotspot2d_launch(h, w, ty, 128)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, k, grid, p)
+        lib = _lib_sets(ctx, k, 6, bufs + [None] * 3, box, blk, sc)
+        ora = _oracle_sets(regions.hotspot2d_tb2(box, blk, h, w, ty), {0: 4, 1: 4, 2: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_hotspot_tb2_sequence(P):
+    h, w = 64, 1024
+    geom = K.hotspot2d_launch(h, w, 4, 128)
+    launches = [[("t0" if t % 2 == 0 else "t1"), "pw", ("t1" if t % 2 == 0 else "t0"), h, w, 4] for t in range(4)]
+    st_, _ = _run_pair(P, "hotspot2d_tb2", {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False),
+                                            "pw": ((h, w), 4, True)}, launches, geom,
+                       lambda box: regions.hotspot2d_tb2(box, geom[1], h, w, 4))
+    # 2 halo rows of temp each way per boundary per launch, + the 1-row power halo once
+    assert st_["stale_bytes"] == 4 * 2 * cf.hotspot2d_stale_per_iter(w, P) + cf.hotspot2d_stale_per_iter(w, P)
