@@ -108,18 +108,22 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
         const int ce = j0 + 4 >= W ? cx + 3 : cx + 4;
         ptx::mbar_wait(&full[g % kNS], (g / kNS) & 1u);
         ptx::mbar_wait(&full[(g + 1) % kNS], ((g + 1) / kNS) & 1u);
-        for (int64_t t = 2; t < nr + 4; ++t) {
+        static_assert((kNS & (kNS - 1)) == 0 && (kS1 & (kS1 - 1)) == 0, "rings are powers of two");
+        const int nt = (int)nr + 4;
+        int row1 = (int)(rstart + dir);              // sweep-1 row of iteration t = 2
+        float* outp = tout + (rstart + 2 * dir) * W + j0;  // sweep-2 row of iteration t = 4
+        const int64_t dW = dir * W;
+        for (int t = 2; t < nt; ++t, row1 += (int)dir) {
             // input rows (sequence) t-2, t-1, t are in the ring; compute sweep-1 of
             // the row at sequence t-1 (rows r0-1 .. rend in march order), then sweep-2
             // of the row at sequence t-2 (rows r0 .. rend-1).
             const uint32_t gq = g + (uint32_t)t;
-            ptx::mbar_wait(&full[gq % kNS], (gq / kNS) & 1u);
-            const float* sa = ring + (size_t)((gq - 2) % kNS) * kStageFloats;  // seq t-2
-            const float* sb = ring + (size_t)((gq - 1) % kNS) * kStageFloats;  // seq t-1
-            const float* sc = ring + (size_t)(gq % kNS) * kStageFloats;        // seq t
-            const int64_t row1 = rstart + dir * (t - 1);                        // sweep-1 row
+            ptx::mbar_wait(&full[gq & (kNS - 1)], (gq / kNS) & 1u);
+            const float* sa = ring + ((gq - 2) & (kNS - 1)) * kStageFloats;  // seq t-2
+            const float* sb = ring + ((gq - 1) & (kNS - 1)) * kStageFloats;  // seq t-1
+            const float* sc = ring + (gq & (kNS - 1)) * kStageFloats;        // seq t
             const bool need1 = row1 >= 0 && row1 < H;      // rows outside the grid are never read
-            float* s1row = s1 + (size_t)(((t - 1) % kS1 + kS1) % kS1) * kRowF;
+            float* s1row = s1 + ((t - 1) & (kS1 - 1)) * kRowF;
             if (need1) {
                 // sweep 1 on columns j0..j0+3 (N/S = rows t-2 / t, order-independent)
                 const float4 c = *reinterpret_cast<const float4*>(sb + cx);
@@ -150,15 +154,15 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
                 }
             }
             consumer_bar();
-            const int64_t row2 = rstart + dir * (t - 2);  // sweep-2 row
-            const bool need2 = t - 2 >= 2 && t - 2 <= nr + 1;
+            const bool need2 = t >= 4;  // sweep-2 rows: sequence 2 .. nr+1
             if (need2) {  // uniform: every lane joins the shuffles
                 // sweep-1 rows t-3, t-2, t-1 (clamped to the grid: the row outside the grid
-                // mirrors row2 itself)
-                const float* m0 = s1 + (size_t)(((t - 2) % kS1 + kS1) % kS1) * kRowF;
-                const int64_t rn = row2 - dir, rs = row2 + dir;
-                const float* mn = (rn < 0 || rn >= H) ? m0 : s1 + (size_t)(((t - 3) % kS1 + kS1) % kS1) * kRowF;
-                const float* ms = (rs < 0 || rs >= H) ? m0 : s1 + (size_t)(((t - 1) % kS1 + kS1) % kS1) * kRowF;
+                // mirrors row2 = row1 - dir itself)
+                const int row2 = row1 - (int)dir;
+                const float* m0 = s1 + ((t - 2) & (kS1 - 1)) * kRowF;
+                const int rn = row2 - (int)dir, rs = row1;
+                const float* mn = (rn < 0 || rn >= H) ? m0 : s1 + ((t - 3) & (kS1 - 1)) * kRowF;
+                const float* ms = (rs < 0 || rs >= H) ? m0 : s1 + ((t - 1) & (kS1 - 1)) * kRowF;
                 const float4 c = *reinterpret_cast<const float4*>(m0 + cx);
                 const float4 a = *reinterpret_cast<const float4*>(mn + cx);
                 const float4 b = *reinterpret_cast<const float4*>(ms + cx);
@@ -173,10 +177,11 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
                 o.y = hs(c.y, a.y, b.y, c.z, c.x, p.y);
                 o.z = hs(c.z, a.z, b.z, c.w, c.y, p.z);
                 o.w = hs(c.w, a.w, b.w, ev, c.z, p.w);
-                if (active) *reinterpret_cast<float4*>(tout + row2 * W + j0) = o;
+                if (active) *reinterpret_cast<float4*>(outp) = o;
+                outp += dW;
             }
             __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&empty[(gq - 2) % kNS]);  // seq t-2 fully used
+            if (lane == 0) ptx::mbar_arrive(&empty[(gq - 2) & (kNS - 1)]);  // seq t-2 fully used
         }
         __syncwarp();
         if (lane == 0) {

@@ -63,11 +63,6 @@ __device__ __forceinline__ u64 fma2(u64 a, u64 b, u64 c) {
 }
 // r2 >= eps^2 = 1e-4 is never denormal, so the flush-to-zero MUFU.RSQ is exact
 // enough and skips rsqrtf's denormal scaling (2 FMUL per call).
-__device__ __forceinline__ float rsqrt_ftz(float x) {
-    float r;
-    asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
-    return r;
-}
 __device__ __forceinline__ u64 rsqrt2(u64 v) {
     // one asm block so that ptxas can keep both MUFU results in the register pair
     // (separate unpack / MUFU / pack statements cost ~3 MOVs per interaction)
