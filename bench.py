@@ -183,20 +183,21 @@ class Workload:
         tile = getattr(self, "tile", 0)
         if self.name == "hotspot2d":
             self.pr = K.hotspot2d_setup(ctx, *self.host, ty=tile or K.HOTSPOT_TY,
-                                        kernel=getattr(self, "variant", None) or "hotspot2d_tb2")
+                                        kernel=getattr(self, "variant", None) or "hotspot2d_tb2",
+                                        tiles=self.tiles)
             # sweeps fused per launch: 2 for hotspot2d_tb2 (one HBM pass = 12 B per cell per launch)
             self.sweeps = self.pr.sweeps
             self.bytes_per_unit = 12 / self.sweeps
             self.upload_bufs = [(self.pr.tb[0], self.host[0]), (self.pr.tb[2], self.host[1])]
         elif self.name == "heat3d":
             self.pr = K.heat3d_setup(ctx, self.host[0], zc=tile or K.HEAT_ZC,
-                                     kernel=getattr(self, "variant", None) or "heat3d")
+                                     kernel=getattr(self, "variant", None) or "heat3d", tiles=self.tiles)
             self.upload_bufs = [(self.pr.ub[0], self.host[0])]
         elif self.name == "sgemm":
             self.pr, _ = K.sgemm_program(ctx, *self.host, launches=0)
             self.upload_bufs = [(self.pr.abc[0], self.host[0]), (self.pr.abc[1], self.host[1])]
         elif self.name == "jacobi2d":
-            self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0)
+            self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0, tiles=self.tiles)
             self.upload_bufs = [(b, self.host[0]) for b in self.pr.bufs]
         elif self.name == "nbody":
             self.pr = K.nbody_setup(ctx, *self.host)
@@ -356,6 +357,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
     ap.add_argument("--tile", type=int, default=0, help="rows per block (hotspot2d TY) / planes per block (heat3d ZC)")
+    ap.add_argument("--tiles", default=None,
+                    help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")
     ap.add_argument("--abg", action="store_true",
                     help="also run the paper's alpha/beta/gamma overhead decomposition (P:L1164-1181)")
     args = ap.parse_args()
@@ -370,6 +373,10 @@ def main():
     w = Workload(args.workload, args.iters or WORKLOADS[args.workload][1])
     w.variant = args.variant
     w.tile = args.tile
+    w.tiles = None
+    if args.tiles:
+        t = [int(x) for x in args.tiles.lower().split("x")]
+        w.tiles = tuple(t + [1] * (3 - len(t)))
 
     if args.impl == "reference":
         line = run_reference(args, w, rank)
@@ -481,14 +488,17 @@ def main():
                    else "1 MB working set stays in L2 (latency-bound C1)",
                    "process_model": process_model,
                    "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tb2"}.get(w.name, w.name),
-                   "sweeps_per_launch": getattr(w, "sweeps", 1)},
-        "gpu_launches": int(st["kernel_launches"]),
+                   "sweeps_per_launch": getattr(w, "sweeps", 1),
+                   "partition_shape": list(w.tiles) if w.tiles else "1-D slabs of the slowest grid dim"},
+        "gpu_launches": int(st["kernel_launches"] + st["copy_kernels"]),
         "graph_replays": int(st.get("graph_replays", 0)),
         "clocks": clocks,
         "roofline": roofline,
         "kernel_ms_avg": avg_kernel_ms,
         "transfers": {"stale_bytes": int(st["stale_bytes"]), "moved_bytes": int(st["moved_bytes"]),
-                      "analytic_min_bytes": w.stale_min(P) * args.steps, "copies": int(st["copies"])},
+                      "analytic_min_bytes": w.stale_min(P) * args.steps if not w.tiles else None,
+                      "copies": int(st["copies"]), "strided_copies": int(st["strided_copies"]),
+                      "halo_copy_kernels": int(st["copy_kernels"])},
         "host_us_per_launch": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"]
                                + st["host_ns_issue"] + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
         "host_us_per_launch_phases": {k: st["host_ns_" + k] / 1e3 / max(1, st["launches"])

@@ -240,6 +240,21 @@ int pk_synchronize(pk_ctx ctx);
 int pk_timer_begin(pk_ctx ctx);
 int pk_timer_end(pk_ctx ctx, double* elapsed_ms);
 
+/* Tile partitions ("suggested partitioning
+ * strategy"): split the grid into tiles[0] x tiles[1] x tiles[2] (x, y, z) block
+ * boxes instead of P slabs of one dimension.  Partition p is tile
+ * (p % tx, (p / tx) % ty, p / (tx*ty)); each grid dimension d is split like the
+ * 1-D rule, [floor(i*G_d/t_d), floor((i+1)*G_d/t_d)).  tx*ty*tz must equal the
+ * context's P (PK_ERR_INVALID otherwise); tiles == NULL or {0,0,0} restores the
+ * 1-D split.  Halo columns become equal-length byte ranges at a constant pitch:
+ * the transfer engine issues each such run (and equal runs repeated at a
+ * constant slice stride, 3-D) as ONE copy: pieces up to 256 B by the
+ * destination's SMs (halo-copy kernel reading the source through its peer
+ * pointer), wider ones by cudaMemcpy2D/3D(Peer)Async (pk_stats.strided_copies,
+ * pk_stats.copy_kernels).
+ * Applies to later launches (bumps the kernel's descriptor version). */
+int pk_set_partition_shape(pk_ctx ctx, pk_kernel k, const int32_t tiles[3]);
+
 /* ---------------------------------------------------------------- introspection */
 /* Grid partition p of the kernel's launch (a1), as (zmin,zmax,ymin,ymax,xmin,xmax). */
 int pk_partition_grid(pk_ctx ctx, pk_kernel k, const int32_t grid[3], int part,
@@ -280,6 +295,8 @@ typedef struct {
     uint64_t timed_kernels;      /* kernels included in kernel_ms */
     uint64_t graph_replays;      /* launches served by steady-state graph replay */
     uint64_t graph_captures;     /* launches captured into a replay graph */
+    uint64_t strided_copies;     /* of `copies`: equal pieces at a constant pitch (2-D / 3-D) */
+    uint64_t copy_kernels;       /* of `strided_copies`: narrow runs moved by the SM halo-copy kernel */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);

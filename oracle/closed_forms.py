@@ -31,6 +31,19 @@ def heat3d_stale_per_iter(h: int, w: int, nparts: int, elem_bytes: int = 4) -> i
     return (nparts - 1) * 2 * h * w * elem_bytes
 
 
+def hotspot2d_tile_stale_per_iter(h: int, w: int, tx: int, ty: int, elem_bytes: int = 4) -> int:
+    """Tile partitions (NEXT-2), clamped 5-point: every internal horizontal cut moves
+    one full row (w cells) each way, every internal vertical cut one full column
+    (h cells) each way; the 5-point stencil reads no diagonal, so corners move nothing."""
+    return 2 * ((ty - 1) * w + (tx - 1) * h) * elem_bytes
+
+
+def jacobi2d_tile_stale_per_iter(h: int, w: int, tx: int, ty: int, elem_bytes: int = 4) -> int:
+    """Tile partitions, Dirichlet 5-point: only interior cells are read through a cut,
+    so a horizontal cut moves w - 2 cells and a vertical cut h - 2 cells each way."""
+    return 2 * ((ty - 1) * (w - 2) + (tx - 1) * (h - 2)) * elem_bytes
+
+
 def gemm_stale(k: int, n: int, nparts: int, elem_bytes: int = 4) -> int:
     """B (k x n) linearly distributed, read whole by every partition: (P-1) * |B|."""
     return (nparts - 1) * k * n * elem_bytes

@@ -35,5 +35,17 @@ def partition_box(grid, nparts: int, p: int, forced: int = -1):
     return (lo[Z], hi[Z], lo[Y], hi[Y], lo[X], hi[X])
 
 
+def tile_box(grid, tiles, p: int):
+    """Tile partitions ("suggested partitioning
+    strategy"; reading Q24 in DESIGN.md §3): tiles = (tx, ty, tz), tx*ty*tz = P.
+    Partition p is tile (p mod tx, (p div tx) mod ty, p div (tx*ty)), x fastest;
+    along every dimension the tile index i of t takes blocks [floor(iG/t), floor((i+1)G/t))."""
+    tx, ty, tz = (int(t) for t in tiles)
+    idx = (p % tx, (p // tx) % ty, p // (tx * ty))
+    lo = [idx[d] * int(grid[d]) // (tx, ty, tz)[d] for d in range(3)]
+    hi = [(idx[d] + 1) * int(grid[d]) // (tx, ty, tz)[d] for d in range(3)]
+    return (lo[Z], hi[Z], lo[Y], hi[Y], lo[X], hi[X])
+
+
 def box_empty(box) -> bool:
     return box[0] >= box[1] or box[2] >= box[3] or box[4] >= box[5]

@@ -70,7 +70,8 @@ class pk_stats(C.Structure):
                 ("host_ns_plan", C.c_uint64), ("host_ns_issue", C.c_uint64),
                 ("host_ns_update", C.c_uint64), ("kernel_ms", C.c_double),
                 ("kernel_ms_max_launch", C.c_double), ("timed_kernels", C.c_uint64),
-                ("graph_replays", C.c_uint64), ("graph_captures", C.c_uint64)]
+                ("graph_replays", C.c_uint64), ("graph_captures", C.c_uint64),
+                ("strided_copies", C.c_uint64), ("copy_kernels", C.c_uint64)]
 
 
 RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)
@@ -122,6 +123,7 @@ def lib():
         "pk_timer_begin": [C.c_void_p],
         "pk_timer_end": [C.c_void_p, C.POINTER(C.c_double)],
         "pk_partition_grid": [C.c_void_p, C.c_int64, _I32P, C.c_int, _I64P],
+        "pk_set_partition_shape": [C.c_void_p, C.c_int64, _I32P],
         "pk_enumerate": [C.c_void_p, C.c_int64, C.c_int, C.c_int, C.c_int64, _I64P, _I32P, _I64P,
                          C.c_int, RANGE_CB, C.c_void_p],
         "pk_tracker_dump": [C.c_void_p, C.c_int64, SEGMENT_CB, C.c_void_p],
@@ -298,6 +300,12 @@ def pk_timer_end(ctx) -> float:
     ms = C.c_double()
     _check(lib().pk_timer_end(ctx, C.byref(ms)), "pk_timer_end")
     return ms.value
+
+
+def pk_set_partition_shape(ctx, kernel, tiles=None):
+    """tiles = (tx, ty, tz) with tx*ty*tz == P, or None for the 1-D split (NEXT-2)."""
+    t = None if tiles is None else _i32(list(tiles))
+    _check(lib().pk_set_partition_shape(ctx, kernel, t), "pk_set_partition_shape")
 
 
 def pk_partition_grid(ctx, kernel, grid, part):

@@ -9,6 +9,7 @@
 
 #include <cstdint>
 #include <string>
+#include <memory>
 #include <vector>
 
 #include "pk_api.h"
@@ -67,17 +68,31 @@ struct Seg {
     uint64_t mask;
 };
 
+// Segment vectors are immutable and shared: a memoised state (graph replay) is
+// restored by pointer, and every mutation builds a fresh vector (copy-on-write).
+using SegVec = std::vector<Seg>;
+using SegState = std::shared_ptr<const SegVec>;
+
 class Tracker {
 public:
     void init(uint64_t size, uint64_t mask);
     uint64_t size() const { return size_; }
-    const std::vector<Seg>& segments() const { return segs_; }
-    void set_segments(const std::vector<Seg>& s) { segs_ = s; }  // restore a memoised state
-    uint64_t fingerprint() const {                                 // FNV-1a over the segments
-        uint64_t h = 1469598103934665603ull;
-        for (const Seg& s : segs_)
-            for (uint64_t v : {s.b, s.e, s.mask}) { h ^= v; h *= 1099511628211ull; }
-        return h;
+    const SegVec& segments() const { return *segs_; }
+    SegState state() const { return segs_; }
+    void set_state(SegState s, uint64_t fp) {  // restore a memoised state in O(1)
+        segs_ = std::move(s);
+        fp_ = fp;
+        fp_valid_ = true;
+    }
+    uint64_t fingerprint() const {  // FNV-1a over the segments, cached until the next mutation
+        if (!fp_valid_) {
+            uint64_t h = 1469598103934665603ull;
+            for (const Seg& s : *segs_)
+                for (uint64_t v : {s.b, s.e, s.mask}) { h ^= v; h *= 1099511628211ull; }
+            fp_ = h;
+            fp_valid_ = true;
+        }
+        return fp_;
     }
     // Visit the pieces of [b,e) with their masks, in order.
     template <class F>
@@ -96,39 +111,43 @@ public:
 private:
     size_t first_overlapping(uint64_t b) const;
     uint64_t size_ = 0;
-    std::vector<Seg> segs_;
+    SegState segs_ = std::make_shared<const SegVec>();
+    mutable uint64_t fp_ = 0;
+    mutable bool fp_valid_ = false;
 };
 
 inline size_t Tracker::first_overlapping(uint64_t b) const {
-    size_t lo = 0, hi = segs_.size();
+    const SegVec& sg = *segs_;
+    size_t lo = 0, hi = sg.size();
     while (lo < hi) {  // first seg with e > b
         size_t mid = (lo + hi) / 2;
-        if (segs_[mid].e <= b) lo = mid + 1; else hi = mid;
+        if (sg[mid].e <= b) lo = mid + 1; else hi = mid;
     }
     return lo;
 }
 
 template <class F>
 void Tracker::query(uint64_t b, uint64_t e, F&& f) const {
-    for (size_t i = first_overlapping(b); i < segs_.size() && segs_[i].b < e; ++i) {
-        uint64_t lo = segs_[i].b > b ? segs_[i].b : b;
-        uint64_t hi = segs_[i].e < e ? segs_[i].e : e;
-        if (lo < hi) f(lo, hi, segs_[i].mask);
+    const SegVec& sg = *segs_;
+    for (size_t i = first_overlapping(b); i < sg.size() && sg[i].b < e; ++i) {
+        uint64_t lo = sg[i].b > b ? sg[i].b : b;
+        uint64_t hi = sg[i].e < e ? sg[i].e : e;
+        if (lo < hi) f(lo, hi, sg[i].mask);
     }
 }
 
 template <class F>
 void Tracker::apply(const RangeList& r, F&& f) {
     if (r.empty()) return;
-    std::vector<Seg> out;
-    out.reserve(segs_.size() + 2 * r.size() + 2);
+    SegVec out;
+    out.reserve(segs_->size() + 2 * r.size() + 2);
     auto push = [&out](uint64_t b, uint64_t e, uint64_t m) {
         if (b >= e) return;
         if (!out.empty() && out.back().e == b && out.back().mask == m) out.back().e = e;
         else out.push_back(Seg{b, e, m});
     };
     size_t ri = 0;
-    for (const Seg& s : segs_) {
+    for (const Seg& s : *segs_) {
         uint64_t cur = s.b;
         while (ri < r.size() && r[ri].e <= cur) ++ri;
         size_t rj = ri;
@@ -142,7 +161,8 @@ void Tracker::apply(const RangeList& r, F&& f) {
             if (r[rj].e <= s.e) ++rj;
         }
     }
-    segs_.swap(out);
+    segs_ = std::make_shared<const SegVec>(std::move(out));
+    fp_valid_ = false;
 }
 
 }  // namespace pk

@@ -210,8 +210,10 @@ uint64_t total_bytes(const RangeList& r) {
 
 void Tracker::init(uint64_t size, uint64_t mask) {
     size_ = size;
-    segs_.clear();
-    if (size) segs_.push_back(Seg{0, size, mask});
+    SegVec v;
+    if (size) v.push_back(Seg{0, size, mask});
+    segs_ = std::make_shared<const SegVec>(std::move(v));
+    fp_valid_ = false;
 }
 
 }  // namespace pk

@@ -47,6 +47,11 @@ extern const Builtin kBuiltinHeat3dTma;      // heat3d (TMA plane ring, default)
 extern const Builtin kBuiltinNbody;
 extern const Builtin kBuiltinSgemm;          // sgemm_tf32x3 (tcgen05 3xTF32)
 
+// Strided halo copy on the destination's SMs (kernels/halo_copy.cu): nslab slabs
+// (stride `slice`) of `rows` pieces (stride `pitch`) of `len` bytes, dst <- src.
+cudaError_t launch_strided_copy(char* dst, const char* src, uint64_t len, uint64_t pitch, uint64_t rows,
+                                uint64_t slice, uint64_t nslab, int sm_count, cudaStream_t stream);
+
 // Descriptor helpers used by the kernel files' describe() functions.
 inline pk_expr E(int64_t c0) {
     pk_expr e{};

@@ -123,6 +123,7 @@ struct Kernel {
     int nargs = 0;
     int32_t kinds[PK_MAX_ARGS] = {};
     int32_t partition_dim = -1;
+    int32_t tiles[3] = {0, 0, 0};  // (tx, ty, tz) tile partition; 0 = 1-D split
     std::vector<Tap> taps;
     LauncherFn launcher = nullptr;
     uint64_t version = 0;  // bumps when taps change (region cache key)
@@ -158,12 +159,14 @@ struct pk_ctx_s {
     uint32_t mode = 0;
     bool host_only = false;
     std::vector<int> dev, prank;
+    std::vector<int> sm_count;  // per partition's device (halo copy kernel grid)
     std::vector<cudaStream_t> stream;
     std::vector<cudaEvent_t> ev_kernel, ev_copy;
     std::vector<Buffer> bufs;
     std::vector<Kernel> kernels;
     pk_stats stats{};
-    std::vector<CopyOp> last_plan;
+    std::vector<CopyOp> last_plan;                               // built by the eager path
+    std::shared_ptr<const std::vector<CopyOp>> replay_plan;       // set by a graph replay
     std::unordered_map<std::string, std::shared_ptr<std::vector<Regions>>> region_cache;
     std::vector<TimedLaunch> pending_timing;
     std::vector<std::vector<cudaEvent_t>> event_pool;  // per partition (device-bound)
@@ -178,8 +181,9 @@ struct pk_ctx_s {
     struct Memo {
         int seen = 0;
         cudaGraphExec_t exec = nullptr;
-        std::vector<std::pair<int64_t, std::vector<Seg>>> post;  // tracker states after the launch
-        std::vector<CopyOp> plan;
+        struct Post { int64_t buf; SegState state; uint64_t fp; };
+        std::vector<Post> post;  // tracker states after the launch (shared, restored by pointer)
+        std::shared_ptr<const std::vector<CopyOp>> plan;
         pk_stats delta{};
     };
     std::unordered_map<std::string, Memo> memo;
@@ -203,6 +207,11 @@ namespace {
 
 bool valid_buf(pk_ctx c, pk_buf b) { return c && b >= 0 && b < (int64_t)c->bufs.size() && c->bufs[b].alive; }
 bool valid_kernel(pk_ctx c, pk_kernel k) { return c && k >= 0 && k < (int64_t)c->kernels.size(); }
+
+// cudaMemcpy2DAsync / cudaMemcpy3DPeerAsync pitch bound (beyond it: one copy per piece)
+constexpr uint64_t kMaxCopyPitch = 1ull << 30;
+// strided runs of pieces up to this size go through the SM halo-copy kernel
+constexpr uint64_t kNarrowPiece = 256;
 
 int choose_source(uint64_t mask, int p, int P) {
     // reading Q5: nearest holder, ties to the lower index
@@ -231,6 +240,25 @@ void partition_box(const int32_t grid[3], int P, int p, int w, int64_t box[6]) {
     box[0] = lo[2]; box[1] = hi[2];
     box[2] = lo[1]; box[3] = hi[1];
     box[4] = lo[0]; box[5] = hi[0];
+}
+
+// a1 with a tile shape (tx, ty, tz), tx*ty*tz == P: partition p is tile
+// (p % tx, (p / tx) % ty, p / (tx*ty)), each grid dim split like partition_box
+void tile_box(const int32_t grid[3], const int32_t tiles[3], int p, int64_t box[6]) {
+    const int idx[3] = {p % tiles[0], (p / tiles[0]) % tiles[1], p / (tiles[0] * tiles[1])};
+    int64_t lo[3], hi[3];
+    for (int d = 0; d < 3; ++d) {
+        lo[d] = (int64_t)idx[d] * grid[d] / tiles[d];
+        hi[d] = (int64_t)(idx[d] + 1) * grid[d] / tiles[d];
+    }
+    box[0] = lo[2]; box[1] = hi[2];
+    box[2] = lo[1]; box[3] = hi[1];
+    box[4] = lo[0]; box[5] = hi[0];
+}
+
+void kernel_box(const Kernel& K, const int32_t grid[3], int P, int p, int64_t box[6]) {
+    if (K.tiles[0] > 0) tile_box(grid, K.tiles, p, box);
+    else partition_box(grid, P, p, split_dim(grid, K.partition_dim), box);
 }
 
 bool box_empty(const int64_t box[6]) { return box[0] >= box[1] || box[2] >= box[3] || box[4] >= box[5]; }
@@ -362,9 +390,11 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
         c->ev_copy.resize(c->P);
         c->event_pool.resize(c->P);
         c->ev_join.assign(c->P, nullptr);
+        c->sm_count.assign(c->P, 148);
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
             PK_CUDA(cudaSetDevice(c->dev[p]));
+            PK_CUDA(cudaDeviceGetAttribute(&c->sm_count[p], cudaDevAttrMultiProcessorCount, c->dev[p]));
             PK_CUDA(cudaStreamCreateWithFlags(&c->stream[p], cudaStreamNonBlocking));
             PK_CUDA(cudaEventCreateWithFlags(&c->ev_kernel[p], cudaEventDisableTiming));
             PK_CUDA(cudaEventCreateWithFlags(&c->ev_copy[p], cudaEventDisableTiming));
@@ -677,13 +707,12 @@ int pk_copy_from_host_for(pk_ctx c, pk_buf b, const void* host, size_t bytes, pk
     const Kernel& K = c->kernels[k];
     if (arg < 0 || arg >= K.nargs || K.kinds[arg] != PK_ARG_BUFFER) return fail(PK_ERR_INVALID, "bad arg index");
     const int P = c->P;
-    const int w = split_dim(grid, K.partition_dim);
     EvalEnv env{scalars, ns, {block[0], block[1], block[2]}};
     std::vector<RangeList> U(P);
     RangeList covered;
     for (int p = 0; p < P; ++p) {
         int64_t box[6];
-        partition_box(grid, P, p, w, box);
+        kernel_box(K, grid, P, p, box);
         if (box_empty(box)) continue;
         Status st = arg_ranges(K, arg, PK_READ, box, B, env, &U[p]);
         if (!st.ok()) return fail(st);
@@ -852,10 +881,26 @@ int pk_builtin_kernel(pk_ctx c, const char* name, pk_kernel* out) {
     return b->describe(c, *out);
 }
 
+int pk_set_partition_shape(pk_ctx c, pk_kernel k, const int32_t tiles[3]) {
+    if (!valid_kernel(c, k)) return fail(PK_ERR_INVALID, "bad kernel");
+    Kernel& K = c->kernels[k];
+    if (!tiles || (tiles[0] == 0 && tiles[1] == 0 && tiles[2] == 0)) {
+        K.tiles[0] = K.tiles[1] = K.tiles[2] = 0;
+    } else {
+        if (tiles[0] < 1 || tiles[1] < 1 || tiles[2] < 1)
+            return fail(PK_ERR_INVALID, "tile counts must be >= 1 (or all 0 for the 1-D split)");
+        if ((int64_t)tiles[0] * tiles[1] * tiles[2] != c->P)
+            return fail(PK_ERR_INVALID, "tx*ty*tz must equal the number of partitions");
+        for (int d = 0; d < 3; ++d) K.tiles[d] = tiles[d];
+    }
+    K.version++;  // region cache + launch memo keys
+    return PK_OK;
+}
+
 int pk_partition_grid(pk_ctx c, pk_kernel k, const int32_t grid[3], int part, int64_t part_out[6]) {
     if (!valid_kernel(c, k) || !grid || !part_out || part < 0 || part >= c->P)
         return fail(PK_ERR_INVALID, "bad argument");
-    partition_box(grid, c->P, part, split_dim(grid, c->kernels[k].partition_dim), part_out);
+    kernel_box(c->kernels[k], grid, c->P, part, part_out);
     return PK_OK;
 }
 
@@ -881,7 +926,7 @@ int pk_tracker_dump(pk_ctx c, pk_buf b, pk_segment_cb cb, void* user) {
 
 int pk_last_plan(pk_ctx c, pk_copy_cb cb, void* user) {
     if (!c || !cb) return fail(PK_ERR_INVALID, "bad argument");
-    for (const CopyOp& o : c->last_plan) cb(user, o.buf, o.src, o.dst, o.b, o.e);
+    for (const CopyOp& o : c->replay_plan ? *c->replay_plan : c->last_plan) cb(user, o.buf, o.src, o.dst, o.b, o.e);
     return PK_OK;
 }
 
@@ -917,6 +962,8 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
     a.launches += sign * d.launches;
     a.kernel_launches += sign * d.kernel_launches;
     a.copies += sign * d.copies;
+    a.strided_copies += sign * d.strided_copies;
+    a.copy_kernels += sign * d.copy_kernels;
     a.stale_bytes += sign * d.stale_bytes;
     a.moved_bytes += sign * d.moved_bytes;
     for (int i = 0; i < 16; ++i)
@@ -971,8 +1018,8 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
         if (int r = enter_graph_mode(c)) return r;
         if (int r = c->set_device(c->dev[c->first_local])) return r;
         PK_CUDA(cudaGraphLaunch(m.exec, c->stream[c->first_local]));
-        for (auto& ps : m.post) c->bufs[ps.first].tracker.set_segments(ps.second);
-        c->last_plan = m.plan;
+        for (auto& ps : m.post) c->bufs[ps.buf].tracker.set_state(ps.state, ps.fp);
+        c->replay_plan = m.plan;
         add_stats(c->stats, m.delta, 1);
         c->stats.graph_replays += 1;
         c->launch_counter++;
@@ -1025,12 +1072,15 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
     }
     pk_ctx_s::Memo& m = c->memo[key];
     m.seen += 1;
-    m.plan = c->last_plan;
+    m.plan = std::make_shared<const std::vector<CopyOp>>(c->last_plan);
     m.delta = c->stats;
     add_stats(m.delta, before, -1);
     m.delta.graph_replays = m.delta.graph_captures = 0;
     m.post.clear();
-    for (int64_t b : bids) m.post.emplace_back(b, c->bufs[b].tracker.segments());
+    for (int64_t b : bids) {
+        const Tracker& T = c->bufs[b].tracker;
+        m.post.push_back({b, T.state(), T.fingerprint()});
+    }
     return PK_OK;
 }
 
@@ -1061,7 +1111,6 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     uint64_t t0 = now_ns();
 
     // ---- a1 + a2: partition boxes and regions (cached) ----
-    const int w = split_dim(grid, K.partition_dim);
     std::shared_ptr<std::vector<Regions>> regs;
     std::string key = region_key(K, k, grid, block, scalars, ns, P, bound);
     auto it = c->region_cache.find(key);
@@ -1073,7 +1122,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         EvalEnv env{scalars, ns, {block[0], block[1], block[2]}};
         for (int p = 0; p < P; ++p) {
             Regions& R = (*regs)[p];
-            partition_box(grid, P, p, w, R.box);
+            kernel_box(K, grid, P, p, R.box);
             R.empty = box_empty(R.box);
             R.args.resize(K.nargs);
             if (R.empty) continue;
@@ -1127,6 +1176,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
 
     // ---- a3: stale detection + transfer plan against the pre-launch state ----
     c->last_plan.clear();
+    c->replay_plan.reset();
     if (track) {
         for (int p = 0; p < P; ++p) {
             for (auto& bs : sets[p]) {
@@ -1158,6 +1208,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     // ---- a4 + a5: transfers, pulled on the destination stream ----
     if (!c->host_only) {
         if (transfer && !c->last_plan.empty()) {
+            std::vector<size_t> order;
             size_t i = 0;
             while (i < c->last_plan.size()) {
                 const int p = c->last_plan[i].dst;
@@ -1180,19 +1231,110 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                         waited_src |= bit;
                     }
                 }
-                for (size_t t = i; t < j; ++t) {
-                    const CopyOp& o = c->last_plan[t];
-                    if (!c->local(o.src)) continue;
+                // group by (buffer, source) in plan order; a run of equal-length pieces at a
+                // constant pitch (a tile partition's halo column, NEXT-2) is ONE 2-D copy
+                order.resize(j - i);
+                for (size_t t = i; t < j; ++t) order[t - i] = t;
+                std::stable_sort(order.begin(), order.end(), [&](size_t a, size_t b) {
+                    const CopyOp &x = c->last_plan[a], &y = c->last_plan[b];
+                    return x.buf != y.buf ? x.buf < y.buf : x.src < y.src;
+                });
+                // run2d(t): end of the constant-pitch run of equal pieces starting at order[t]
+                auto run2d = [&](size_t t, uint64_t* pitch) -> size_t {
+                    const CopyOp& o = c->last_plan[order[t]];
+                    const uint64_t len = o.e - o.b;
+                    auto same = [&](size_t v) {
+                        const CopyOp& x = c->last_plan[order[v]];
+                        return x.buf == o.buf && x.src == o.src && x.e - x.b == len;
+                    };
+                    *pitch = 0;
+                    size_t u = t + 1;
+                    if (u < order.size() && same(u)) *pitch = c->last_plan[order[u]].b - o.b;
+                    if (!*pitch || *pitch > kMaxCopyPitch) return t + 1;
+                    while (u < order.size() && same(u) &&
+                           c->last_plan[order[u]].b == c->last_plan[order[u - 1]].b + *pitch)
+                        ++u;
+                    return u;
+                };
+                for (size_t t = 0; t < order.size();) {
+                    const CopyOp& o = c->last_plan[order[t]];
+                    if (!c->local(o.src)) { ++t; continue; }
+                    const uint64_t len = o.e - o.b;
+                    uint64_t pitch = 0;
+                    size_t u = run2d(t, &pitch);
+                    const size_t rows = u - t;
+                    if (rows == 1) pitch = len;
+                    // slabs: equal 2-D runs at a constant slice stride (a 3-D tile's halo
+                    // column repeated per plane) become ONE 3-D copy
+                    size_t nslab = 1;
+                    uint64_t slice = 0, prev = o.b;
+                    while (rows > 1 && u < order.size()) {
+                        const CopyOp& q = c->last_plan[order[u]];
+                        if (q.buf != o.buf || q.src != o.src || q.e - q.b != len) break;
+                        uint64_t p2 = 0;
+                        const size_t w2 = run2d(u, &p2);
+                        if (w2 - u != rows || p2 != pitch) break;
+                        const uint64_t st = q.b - prev;
+                        if (nslab == 1) {
+                            if (st % pitch || st / pitch < rows || st > kMaxCopyPitch) break;
+                            slice = st;
+                        } else if (st != slice) {
+                            break;
+                        }
+                        prev = q.b;
+                        ++nslab;
+                        u = w2;
+                    }
                     Buffer& B = c->bufs[o.buf];
                     char* dst = (char*)B.inst[p] + o.b;
                     const char* src = (const char*)B.inst[o.src] + o.b;
-                    if (c->dev[o.src] == c->dev[p])
-                        PK_CUDA(cudaMemcpyAsync(dst, src, o.e - o.b, cudaMemcpyDeviceToDevice, c->stream[p]));
-                    else
-                        PK_CUDA(cudaMemcpyPeerAsync(dst, c->dev[p], src, c->dev[o.src], o.e - o.b, c->stream[p]));
+                    const bool same_dev = c->dev[o.src] == c->dev[p];
+                    if ((rows > 1 || nslab > 1) && len <= kNarrowPiece) {
+                        // narrow strided run (a halo column): pulled by the destination's SMs
+                        PK_CUDA(launch_strided_copy(dst, src, len, pitch, rows, slice, nslab, c->sm_count[p],
+                                                    c->stream[p]));
+                        c->stats.copy_kernels += 1;
+                    } else if (nslab > 1) {
+                        const size_t ysz = slice / pitch;
+                        if (same_dev) {
+                            cudaMemcpy3DParms pp = {};
+                            pp.srcPtr = make_cudaPitchedPtr((void*)src, pitch, len, ysz);
+                            pp.dstPtr = make_cudaPitchedPtr(dst, pitch, len, ysz);
+                            pp.extent = make_cudaExtent(len, rows, nslab);
+                            pp.kind = cudaMemcpyDeviceToDevice;
+                            PK_CUDA(cudaMemcpy3DAsync(&pp, c->stream[p]));
+                        } else {
+                            cudaMemcpy3DPeerParms pp = {};
+                            pp.srcPtr = make_cudaPitchedPtr((void*)src, pitch, len, ysz);
+                            pp.dstPtr = make_cudaPitchedPtr(dst, pitch, len, ysz);
+                            pp.srcDevice = c->dev[o.src];
+                            pp.dstDevice = c->dev[p];
+                            pp.extent = make_cudaExtent(len, rows, nslab);
+                            PK_CUDA(cudaMemcpy3DPeerAsync(&pp, c->stream[p]));
+                        }
+                    } else if (rows == 1) {
+                        if (same_dev)
+                            PK_CUDA(cudaMemcpyAsync(dst, src, len, cudaMemcpyDeviceToDevice, c->stream[p]));
+                        else
+                            PK_CUDA(cudaMemcpyPeerAsync(dst, c->dev[p], src, c->dev[o.src], len, c->stream[p]));
+                    } else if (same_dev) {
+                        PK_CUDA(cudaMemcpy2DAsync(dst, pitch, src, pitch, len, rows, cudaMemcpyDeviceToDevice,
+                                                  c->stream[p]));
+                    } else {
+                        cudaMemcpy3DPeerParms pp = {};
+                        pp.srcPtr = make_cudaPitchedPtr((void*)src, pitch, len, rows);
+                        pp.dstPtr = make_cudaPitchedPtr(dst, pitch, len, rows);
+                        pp.srcDevice = c->dev[o.src];
+                        pp.dstDevice = c->dev[p];
+                        pp.extent = make_cudaExtent(len, rows, 1);
+                        PK_CUDA(cudaMemcpy3DPeerAsync(&pp, c->stream[p]));
+                    }
+                    const uint64_t moved = len * rows * nslab;
                     c->stats.copies += 1;
-                    c->stats.moved_bytes += o.e - o.b;
-                    if (o.src < 16 && p < 16) c->stats.pair_bytes[o.src][p] += o.e - o.b;
+                    c->stats.strided_copies += rows > 1;
+                    c->stats.moved_bytes += moved;
+                    if (o.src < 16 && p < 16) c->stats.pair_bytes[o.src][p] += moved;
+                    t = u;
                 }
                 PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
                 for (size_t t = i; t < j; ++t) {

@@ -69,9 +69,11 @@ def sgemm_program(ctx, a_host, b_host, launches=1):
 class Problem:
     """A registered builtin kernel plus its ping-pong buffers on one context."""
 
-    def __init__(self, ctx, kernel_name):
+    def __init__(self, ctx, kernel_name, tiles=None):
         self.ctx = ctx
         self.k = abi.pk_builtin_kernel(ctx, kernel_name)
+        if tiles:   # NEXT-2 tile partitions (tx, ty, tz), tx*ty*tz == P
+            abi.pk_set_partition_shape(ctx, self.k, tiles)
         self.bufs = []
 
     def buffer(self, shape, elem_bytes=4, host=None, dev_ptrs=None):
@@ -83,11 +85,11 @@ class Problem:
         abi.pk_launch_partitioned(self.ctx, self.k, grid, block, args, scalars)
 
 
-def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK):
+def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None):
     """C1: both buffers carry the Dirichlet boundary (uploaded); returns the buffer id
     that holds the result after `iters` sweeps."""
     h, w = u_host.shape
-    pr = Problem(ctx, "jacobi2d")
+    pr = Problem(ctx, "jacobi2d", tiles)
     u0 = pr.buffer((h, w), 4, host=u_host)
     u1 = pr.buffer((h, w), 4, host=u_host)
     grid, blk, sc = jacobi2d_launch(h, w, block)
@@ -98,9 +100,9 @@ def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK):
 
 
 def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None,
-                    kernel="hotspot2d"):
+                    kernel="hotspot2d", tiles=None):
     h, w = temp_host.shape
-    pr = Problem(ctx, kernel)
+    pr = Problem(ctx, kernel, tiles)
     t0 = pr.buffer((h, w), 4, host=temp_host, dev_ptrs=dev_ptrs[0] if dev_ptrs else None)
     t1 = pr.buffer((h, w), 4, dev_ptrs=dev_ptrs[1] if dev_ptrs else None)   # undefined (reading Q3)
     pw = pr.buffer((h, w), 4, host=power_host, dev_ptrs=dev_ptrs[2] if dev_ptrs else None)
@@ -125,9 +127,9 @@ def hotspot2d_iterate(pr, iters, start=0):
     return t1 if ((start + iters) // k) % 2 == 1 else t0
 
 
-def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY, kernel="heat3d"):
+def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY, kernel="heat3d", tiles=None):
     d, h, w = u_host.shape
-    pr = Problem(ctx, kernel)
+    pr = Problem(ctx, kernel, tiles)
     u0 = pr.buffer((d, h, w), 4, host=u_host)
     u1 = pr.buffer((d, h, w), 4)
     pr.geom = heat3d_launch(d, h, w, zc, bdy)

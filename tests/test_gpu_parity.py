@@ -73,9 +73,9 @@ def test_no_transfers_negative_control_and_barrier_mode():
 
 
 # ------------------------------------------------------------------ C2 Hotspot
-def _hotspot(t, p, iters, P, ty=16, bdx=128, mode=0, kernel="hotspot2d"):
+def _hotspot(t, p, iters, P, ty=16, bdx=128, mode=0, kernel="hotspot2d", tiles=None):
     ctx = gpu_ctx(P, mode)
-    pr = K.hotspot2d_setup(ctx, t, p, ty, bdx, kernel=kernel)
+    pr = K.hotspot2d_setup(ctx, t, p, ty, bdx, kernel=kernel, tiles=tiles)
     out = K.hotspot2d_iterate(pr, iters)
     res = fetch(ctx, out, t.shape)
     st = abi.pk_get_stats(ctx)
@@ -132,9 +132,9 @@ def test_hotspot_uniform_closed_form_on_gpu():
 
 
 # ------------------------------------------------------------------ C3 Heat
-def _heat(u, iters, P, zc=8, bdy=8, kernel="heat3d"):
-    ctx = gpu_ctx(P)
-    pr = K.heat3d_setup(ctx, u, zc, bdy, kernel=kernel)
+def _heat(u, iters, P, zc=8, bdy=8, kernel="heat3d", tiles=None, mode=0):
+    ctx = gpu_ctx(P, mode)
+    pr = K.heat3d_setup(ctx, u, zc, bdy, kernel=kernel, tiles=tiles)
     out = K.heat3d_iterate(pr, iters)
     res = fetch(ctx, out, u.shape)
     st = abi.pk_get_stats(ctx)
@@ -369,3 +369,64 @@ def test_graph_mode_interleaved_with_eager_work():
     ref, _ = _hotspot(t, p, 20, 1)
     assert np.array_equal(g, ref)
     assert st["graph_replays"] > 0
+
+
+# ------------------------------------------------------------------ tile partitions (NEXT-2)
+@pytest.mark.parametrize("kernel,tiles,bdx", [("hotspot2d", (2, 2, 1), 128), ("hotspot2d", (3, 2, 1), 128),
+                                              ("hotspot2d_tb2", (2, 2, 1), 128), ("hotspot2d_tb2", (2, 4, 1), 128),
+                                              ("hotspot2d_regs", (4, 2, 1), 32)])
+def test_hotspot_tile_partitions_bitwise(kernel, tiles, bdx):
+    """px x py tiles: bit-identical to 1-way; halo columns moved as strided 2-D copies;
+    with graph replay and eagerly (NO_GRAPHS)."""
+    h, w = 300, 1800
+    t, p = synth.hotspot_grids(h, w)
+    iters = 12
+    g1, _ = _hotspot(t, p, iters, 1, 16, bdx, kernel=kernel)
+    assert rel_ok(g1, ok.hotspot2d(t, p, iters), 1e-5)[0]
+    P = tiles[0] * tiles[1]
+    for mode in (0, abi.PK_MODE_NO_GRAPHS):
+        gp, st = _hotspot(t, p, iters, P, 16, bdx, mode=mode, kernel=kernel, tiles=tiles)
+        assert np.array_equal(g1, gp), (tiles, mode)
+        assert st["moved_bytes"] == st["stale_bytes"] > 0
+        assert st["strided_copies"] > 0 and st["copy_kernels"] > 0
+
+
+def test_hotspot_tile_stale_closed_form_on_gpu():
+    h, w = 512, 2048
+    t, p = synth.hotspot_grids(h, w)
+    _, s2 = _hotspot(t, p, 2, 8, 64, tiles=(4, 2, 1))
+    _, s6 = _hotspot(t, p, 6, 8, 64, tiles=(4, 2, 1))
+    # launches 3..6 are steady state: every internal cut moves one row / column each way
+    assert s6["stale_bytes"] - s2["stale_bytes"] == 4 * cf.hotspot2d_tile_stale_per_iter(h, w, 4, 2)
+    assert s6["moved_bytes"] == s6["stale_bytes"]
+
+
+def test_jacobi_tile_partitions_bitwise():
+    u = synth.jacobi_grid(200, 300)
+    ctx = gpu_ctx(1)
+    _, o1 = K.jacobi2d_program(ctx, u, 9)
+    g1 = fetch(ctx, o1, u.shape)
+    abi.pk_finalize(ctx)
+    assert rel_ok(g1, ok.jacobi2d(u, 9), 1e-5)[0]
+    for tiles in ((2, 2, 1), (5, 1, 1), (3, 3, 1)):
+        ctx = gpu_ctx(tiles[0] * tiles[1])
+        _, o = K.jacobi2d_program(ctx, u, 9, tiles=tiles)
+        g = fetch(ctx, o, u.shape)
+        st = abi.pk_get_stats(ctx)
+        abi.pk_finalize(ctx)
+        assert np.array_equal(g, g1), tiles
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+@pytest.mark.parametrize("kernel", ["heat3d", "heat3d_regs"])
+def test_heat_tile_partitions_bitwise(kernel):
+    d, h, w = 24, 40, 260
+    u = synth.heat_grid(d, h, w)
+    iters = 6
+    g1, _ = _heat(u, iters, 1, 4, 8, kernel)
+    assert rel_ok(g1, ok.heat3d(u, iters), 1e-5)[0]
+    for tiles in ((1, 2, 2), (3, 1, 2), (2, 2, 1)):
+        for mode in (0, abi.PK_MODE_NO_GRAPHS):
+            gp, st = _heat(u, iters, tiles[0] * tiles[1] * tiles[2], 4, 8, kernel, tiles=tiles, mode=mode)
+            assert np.array_equal(g1, gp), (tiles, mode)
+            assert st["moved_bytes"] == st["stale_bytes"] > 0

@@ -217,12 +217,14 @@ def _norm_plan(plan, names):
     return res
 
 
-def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0):
+def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0, tiles=None):
     """specs: {name: (shape, eb, uploaded)}; launches: list of [arg binding names or None];
-    thread_prog(box) -> oracle access dict keyed by (arg, 'r'/'w')."""
+    thread_prog(box) -> oracle access dict keyed by (arg, 'r'/'w'); tiles: NEXT-2 tile shape."""
     ctx = host_ctx(P, mode)
     sh = shadow.Shadow(P, single_owner=bool(mode & abi.PK_MODE_SINGLE_OWNER))
     k = abi.pk_builtin_kernel(ctx, kernel)
+    if tiles:
+        abi.pk_set_partition_shape(ctx, k, tiles)
     ids, names = {}, {}
     for name, (shape, eb, up) in specs.items():
         host = np.zeros(int(np.prod(shape)) * eb // 4, dtype=np.float32) if up else None
@@ -236,7 +238,8 @@ def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0):
         abi.pk_launch_partitioned(ctx, k, grid, blk, args, sc)
         per = []
         for p in range(P):
-            box = og.partition_box(grid, P, p)
+            box = og.tile_box(grid, tiles, p) if tiles else og.partition_box(grid, P, p)
+            assert abi.pk_partition_grid(ctx, k, grid, p) == box
             if og.box_empty(box):
                 per.append(None)
                 continue
@@ -325,6 +328,73 @@ def test_nbody_sequence(mode):
     st_, _ = _run_pair(P, "nbody", {"p0": ((n,), 16, True), "p1": ((n,), 16, False), "v": ((n,), 16, True)},
                        launches, geom, lambda box: regions.nbody(box, geom[1], n, K.NBODY_PER_THREAD), mode)
     assert st_["stale_bytes"] == 3 * cf.nbody_stale_per_step(n, P)
+
+
+# ------------------------------------------------------------ tile partitions (NEXT-2)
+@pytest.mark.parametrize("tiles", [(2, 2, 1), (4, 2, 1), (3, 1, 1), (1, 1, 1)])
+def test_jacobi_tile_sequence(tiles):
+    n = 64
+    P = tiles[0] * tiles[1] * tiles[2]
+    geom = K.jacobi2d_launch(n, n)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), n, n] for t in range(5)]
+    st_, _ = _run_pair(P, "jacobi2d", {"u0": ((n, n), 4, True), "u1": ((n, n), 4, True)}, launches, geom,
+                       lambda box: regions.jacobi2d(box, geom[1], n, n), tiles=tiles)
+    assert st_["launches"] == 5
+
+
+@pytest.mark.parametrize("kernel,tiles", [("hotspot2d", (2, 2, 1)), ("hotspot2d_regs", (4, 2, 1)),
+                                          ("hotspot2d_tb2", (2, 3, 1)), ("hotspot2d_tb2", (3, 2, 1))])
+def test_hotspot_tile_sequence(kernel, tiles):
+    h, w = 48, 1600
+    P = tiles[0] * tiles[1]
+    prog = regions.hotspot2d_tb2 if kernel == "hotspot2d_tb2" else regions.hotspot2d
+    bdx = 32 if kernel == "hotspot2d_regs" else 128
+    geom = K.hotspot2d_launch(h, w, 4, bdx)
+    launches = [[("t0" if t % 2 == 0 else "t1"), "pw", ("t1" if t % 2 == 0 else "t0"), h, w, 4] for t in range(4)]
+    _run_pair(P, kernel, {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False), "pw": ((h, w), 4, True)},
+              launches, geom, lambda box: prog(box, geom[1], h, w, 4), tiles=tiles)
+
+
+def test_heat_tile_sequence():
+    d, h, w = 12, 16, 64
+    tiles = (1, 2, 2)
+    geom = K.heat3d_launch(d, h, w, 2, 4)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), d, h, w, 2] for t in range(4)]
+    _run_pair(4, "heat3d", {"u0": ((d, h, w), 4, True), "u1": ((d, h, w), 4, False)}, launches, geom,
+              lambda box: regions.heat3d(box, geom[1], d, h, w, 2), tiles=tiles)
+
+
+def test_tile_shape_validation_and_reset():
+    ctx = host_ctx(4)
+    k = abi.pk_builtin_kernel(ctx, "jacobi2d")
+    for bad in ((2, 1, 1), (0, 4, 1), (2, 2, 2), (-2, -2, 1)):
+        with pytest.raises(abi.PkError):
+            abi.pk_set_partition_shape(ctx, k, bad)
+    abi.pk_set_partition_shape(ctx, k, (2, 2, 1))
+    assert abi.pk_partition_grid(ctx, k, (16, 64, 1), 3) == (0, 1, 32, 64, 8, 16)
+    abi.pk_set_partition_shape(ctx, k, None)
+    assert abi.pk_partition_grid(ctx, k, (16, 64, 1), 3) == og.partition_box((16, 64, 1), 4, 3)
+    abi.pk_finalize(ctx)
+
+
+def test_hotspot_tile_closed_form_through_library():
+    h, w = 64, 2048
+    tiles = (4, 2, 1)
+    geom = K.hotspot2d_launch(h, w, 4, 128)
+    ctx = host_ctx(8)
+    k = abi.pk_builtin_kernel(ctx, "hotspot2d")
+    abi.pk_set_partition_shape(ctx, k, tiles)
+    t0 = abi.pk_register_buffer(ctx, (h, w), 4, host_init=np.zeros(h * w, np.float32))
+    t1 = abi.pk_register_buffer(ctx, (h, w), 4)
+    pw = abi.pk_register_buffer(ctx, (h, w), 4, host_init=np.zeros(h * w, np.float32))
+    per = []
+    for t in range(6):
+        a, b = (t0, t1) if t % 2 == 0 else (t1, t0)
+        s0 = abi.pk_get_stats(ctx)["stale_bytes"]
+        abi.pk_launch_partitioned(ctx, k, geom[0], geom[1], [a, pw, b, h, w, 4], geom[2])
+        per.append(abi.pk_get_stats(ctx)["stale_bytes"] - s0)
+    assert per[2:] == [cf.hotspot2d_tile_stale_per_iter(h, w, 4, 2)] * 4
+    abi.pk_finalize(ctx)
 
 
 # ------------------------------------------------------------ error paths / modes

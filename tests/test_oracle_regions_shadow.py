@@ -34,6 +34,26 @@ def test_partition_rule():
     assert covered == _rng(0, 100)
 
 
+def test_tile_rule():
+    # NEXT-2 tile partitions (reading Q24): x fastest, each dim split by the floor rule
+    assert [grid.tile_box((16, 64, 1), (2, 2, 1), p) for p in range(4)] == [
+        (0, 1, 0, 32, 0, 8), (0, 1, 0, 32, 8, 16), (0, 1, 32, 64, 0, 8), (0, 1, 32, 64, 8, 16)]
+    # (1, P, 1) tiles of a 2-D grid are the 1-D row slabs
+    for p in range(3):
+        assert grid.tile_box((5, 100, 1), (1, 3, 1), p) == grid.partition_box((5, 100, 1), 3, p)
+    # every block of the grid lies in exactly one tile (brute force, ragged sizes)
+    for g, t in (((7, 5, 3), (2, 2, 2)), ((3, 9, 1), (3, 2, 1)), ((1, 4, 6), (1, 2, 3)), ((2, 2, 2), (3, 1, 1))):
+        seen = {}
+        for p in range(t[0] * t[1] * t[2]):
+            z0, z1, y0, y1, x0, x1 = grid.tile_box(g, t, p)
+            for z in range(z0, z1):
+                for y in range(y0, y1):
+                    for x in range(x0, x1):
+                        assert (x, y, z) not in seen
+                        seen[(x, y, z)] = p
+        assert len(seen) == g[0] * g[1] * g[2]
+
+
 # ----------------------- C1 worked example (hand derived) -----------------------
 def test_c1_partition0_read_and_write_sets():
     n = 512
@@ -135,6 +155,43 @@ def test_hotspot_steady_state_matches_closed_form(nparts):
     # fragmentation: bounded segment count per buffer
     for name in ("t0", "t1"):
         assert len(sh.buffers[name].rle()) <= 2 * nparts - 1
+
+
+@pytest.mark.parametrize("tiles", [(2, 2, 1), (4, 2, 1), (2, 3, 1)])
+def test_tile_partition_steady_state_matches_closed_form(tiles):
+    """NEXT-2: with tx x ty tiles every internal cut moves one row / column each way."""
+    h, w = 48, 96
+    ty, bdx = 4, 4                                      # block = 16 columns x 4 rows
+    g = ((w + 4 * bdx - 1) // (4 * bdx), (h + ty - 1) // ty, 1)
+    nparts = tiles[0] * tiles[1]
+    sh = shadow.Shadow(nparts)
+    for name, up in (("t0", True), ("t1", False), ("pw", True)):
+        sh.register(name, h * w, 4, up)
+    stale = []
+    for it in range(4):
+        a, b = ("t0", "t1") if it % 2 == 0 else ("t1", "t0")
+        per = []
+        for p in range(nparts):
+            acc = regions.hotspot2d(grid.tile_box(g, tiles, p), (bdx,), h, w, ty)
+            per.append({a: (acc[(0, "r")], None), "pw": (acc[(1, "r")], None), b: (None, acc[(2, "w")])})
+        stale.append(sum(sh.launch(per)["stale"]))
+    assert stale[2:] == [cf.hotspot2d_tile_stale_per_iter(h, w, tiles[0], tiles[1])] * 2
+    # Jacobi (Dirichlet): interior cells only cross the cuts
+    n = 64
+    sj = shadow.Shadow(nparts)
+    sj.register("u0", n * n, 4, True)
+    sj.register("u1", n * n, 4, True)
+    gj = (n // 32 + (n % 32 > 0), n // 8, 1)
+    per_it = []
+    for it in range(4):
+        a, b = ("u0", "u1") if it % 2 == 0 else ("u1", "u0")
+        per = []
+        for p in range(nparts):
+            acc = regions.jacobi2d(grid.tile_box(gj, tiles, p), (32, 8), n, n)
+            per.append({a: (acc[(0, "r")], None), b: (None, acc[(1, "w")])})
+        per_it.append(sum(sj.launch(per)["stale"]))
+    if gj[0] % tiles[0] == 0:
+        assert per_it[2:] == [cf.jacobi2d_tile_stale_per_iter(n, n, tiles[0], tiles[1])] * 2
 
 
 def test_nbody_allgather_and_validity_vs_single_owner():
