@@ -359,6 +359,8 @@ def main():
     ap.add_argument("--tile", type=int, default=0, help="rows per block (hotspot2d TY) / planes per block (heat3d ZC)")
     ap.add_argument("--tiles", default=None,
                     help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")
+    ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
+                    help="SPMD (torchrun, N > 1) cross-rank transport: CUDA IPC peer memory or NCCL send/recv")
     ap.add_argument("--abg", action="store_true",
                     help="also run the paper's alpha/beta/gamma overhead decomposition (P:L1164-1181)")
     args = ap.parse_args()
@@ -392,16 +394,26 @@ def main():
     ngpu = max(1, args.gpus)
     result = {}
     if world > 1:
-        # SPMD: one process per GPU, one partition per rank; the
-        # replicated plan's cross-rank copies are NCCL send/recv pairs.
+        # SPMD: one process per GPU, one partition per rank.  Default
+        # transport: peer memory (CUDA IPC instances + device epoch flags, each rank pulls
+        # its stale ranges over NVLink); --transport nccl: NCCL send/recv pairs.
         P = world
         local_rank = env_int("LOCAL_RANK", rank)
-        torch.cuda.set_device(local_rank)
-        nid = [abi.pk_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(nid, src=0)
-        ctx = abi.pk_init_spmd(P, rank, world, list(range(world)), part_device=[local_rank] * P, nccl_id=nid[0])
-        devices = list(range(ngpu))
-        process_model = "SPMD: one process per GPU, replicated tracker, NCCL send/recv for cross-rank copies"
+        ndev = torch.cuda.device_count()
+        dev = local_rank % max(1, ndev)          # ranks share a GPU only on boxes with fewer GPUs
+        torch.cuda.set_device(dev)
+        if args.transport == "nccl":
+            nid = [abi.pk_nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(nid, src=0)
+            ctx = abi.pk_init_spmd(P, rank, world, list(range(world)), part_device=[dev] * P, nccl_id=nid[0])
+            process_model = "SPMD: one process per GPU, replicated tracker, NCCL send/recv for cross-rank copies"
+        else:
+            from paper_conf_icppw_matzdf20_b200 import spmd
+            ctx = abi.pk_init_spmd_ipc(P, rank, world, list(range(world)), spmd.dist_allgather(),
+                                       part_device=[dev] * P)
+            process_model = ("SPMD: one process per GPU, replicated tracker, pull copies from CUDA-IPC-mapped "
+                             "peer instances ordered by device epoch flags")
+        devices = list(range(min(ngpu, max(1, ndev))))
     else:
         P = args.parts or ngpu
         ndev = torch.cuda.device_count()
@@ -417,7 +429,7 @@ def main():
     abi.pk_reset_stats(ctx)
     if dist:
         dist.barrier()
-    sampler = ClockSampler(range(ngpu)) if rank == 0 else None
+    sampler = ClockSampler(range(min(ngpu, torch.cuda.device_count()))) if rank == 0 else None
     if sampler:
         sampler.start()
         time.sleep(0.3)

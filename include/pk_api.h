@@ -107,6 +107,36 @@ int pk_finalize(pk_ctx ctx);
 int pk_nccl_unique_id(void* out, size_t bytes);
 int pk_init_spmd(const pk_init_params* params, const void* nccl_unique_id, pk_ctx* out);
 
+/* ---- multi-process SPMD over peer memory (CUDA IPC; no NCCL on the data path) ----
+ * Same replicated model as pk_init_spmd, but every rank maps every other rank's
+ * buffer instances into its own address space (cudaIpcGetMemHandle /
+ * cudaIpcOpenMemHandle, exchanged at pk_register_buffer) and PULLS its stale
+ * ranges itself, straight out of the holder's instance over NVLink/NVSwitch
+ * (copy engine, or the SM halo-copy kernel for narrow strided runs) -- the
+ * paper's "copy from the GPU it was most recently written to",
+ * one process per GPU.  Ordering across processes replaces the global barrier
+ * of Fig. 4 l. 8 by device-side epoch flags in peer memory: every rank
+ * owns two monotone 64-bit words (incoming copies of launch E done / kernel of
+ * launch E done) written by cuStreamWriteValue64 on its stream; a reader waits
+ * (cuStreamWaitValue64, GEQ) for the holder's word before copying (RAW), a
+ * writer waits for the readers' words before overwriting what they read (WAR).
+ * The host thread never blocks on another rank inside pk_launch_partitioned.
+ *
+ * `allgather` is the caller's host all-gather (e.g. torch.distributed over gloo):
+ * every rank passes `bytes` bytes at `send`; on return `recv` holds world_size *
+ * bytes, rank r's contribution at offset r * bytes; it returns 0 on success.  The
+ * library calls it (identically on every rank) inside pk_init_spmd_ipc,
+ * pk_register_buffer, pk_unregister_buffer, pk_copy_from_host(_for),
+ * pk_sync_to_host and pk_finalize, which are therefore collective in this mode.
+ * `user` is passed back unchanged; callback and user must outlive the context.
+ * Execution requires exactly one partition per rank; ranks may share a GPU
+ * (functional testing on one device).  Caller-owned instances must come from
+ * cudaMalloc'd allocations (IPC handles cover whole allocations; the offset is
+ * exchanged too).  Errors: PK_ERR_STATE, PK_ERR_CUDA, PK_ERR_INVALID (callback
+ * failed or missing). */
+typedef int (*pk_host_allgather_fn)(void* user, const void* send, void* recv, size_t bytes);
+int pk_init_spmd_ipc(const pk_init_params* params, pk_host_allgather_fn allgather, void* user, pk_ctx* out);
+
 /* ---------------------------------------------------------------- buffers */
 /* Virtual buffer = one full-size device instance per partition + a tracker
  * (§8.1; full-size instances keep the kernels' global indices, reading

@@ -77,6 +77,8 @@ class pk_stats(C.Structure):
 RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)
 SEGMENT_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64, C.c_uint64)
 COPY_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_int64, C.c_int, C.c_int, C.c_uint64, C.c_uint64)
+ALLGATHER_CB = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_size_t)
+_keepalive = {}   # ctx address -> ctypes callback of pk_init_spmd_ipc (must outlive the context)
 
 _lib = None
 _I64P = C.POINTER(C.c_int64)
@@ -106,6 +108,7 @@ def lib():
         "pk_init": [C.POINTER(pk_init_params), C.POINTER(C.c_void_p)],
         "pk_init_spmd": [C.POINTER(pk_init_params), C.c_void_p, C.POINTER(C.c_void_p)],
         "pk_nccl_unique_id": [C.c_void_p, C.c_size_t],
+        "pk_init_spmd_ipc": [C.POINTER(pk_init_params), ALLGATHER_CB, C.c_void_p, C.POINTER(C.c_void_p)],
         "pk_finalize": [C.c_void_p],
         "pk_register_buffer": [C.c_void_p, C.c_int, _I64P, C.c_int, C.POINTER(C.c_void_p), C.c_void_p, _I64P],
         "pk_copy_from_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
@@ -212,8 +215,33 @@ def pk_init_spmd(nparts, my_rank, world_size, part_rank, part_device=None, nccl_
     return ctx
 
 
+def pk_init_spmd_ipc(nparts, my_rank, world_size, part_rank, allgather, part_device=None, flags=0):
+    """Multi-process SPMD context over peer memory (CUDA IPC, device epoch flags).
+    `allgather(data: bytes) -> bytes` must return the concatenation of every rank's
+    `data` in rank order (e.g. ``spmd.dist_allgather()``); it is called collectively."""
+    def _cb(_user, send, recv, n):
+        try:
+            out = allgather(C.string_at(send, n))
+            if len(out) != n * world_size:
+                return -1
+            C.memmove(recv, out, len(out))
+            return 0
+        except Exception:
+            return -1
+    cb = ALLGATHER_CB(_cb)
+    p = pk_init_params(nparts, my_rank, world_size, flags,
+                       _i32(part_device) if part_device is not None else None, _i32(part_rank))
+    ctx = C.c_void_p()
+    _check(lib().pk_init_spmd_ipc(C.byref(p), cb, None, C.byref(ctx)), "pk_init_spmd_ipc")
+    _keepalive[ctx.value] = cb
+    return ctx
+
+
 def pk_finalize(ctx):
-    _check(lib().pk_finalize(ctx), "pk_finalize")
+    try:
+        _check(lib().pk_finalize(ctx), "pk_finalize")
+    finally:
+        _keepalive.pop(ctx.value, None)
 
 
 def pk_register_buffer(ctx, shape, elem_bytes, dev_ptrs=None, host_init=None, nparts=None):

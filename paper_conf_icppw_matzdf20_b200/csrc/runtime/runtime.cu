@@ -13,6 +13,7 @@
 //   WAR  any write into (b,p) -- kernel or incoming copy -- waits for the copies
 //        that read (b,p) since its last write ("readers").
 // PK_MODE_GLOBAL_BARRIER restores the literal host-side barrier.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 
@@ -109,6 +110,11 @@ struct Buffer {
     Tracker tracker;
     std::vector<uint8_t> last_writer;  // per partition
     std::vector<uint64_t> readers;     // per partition: mask of partitions whose ev_copy must precede a write
+    // SPMD over peer memory (pk_init_spmd_ipc): replicated epoch bookkeeping
+    std::vector<uint64_t> ep_mod;      // [q]: epoch of the last device write of (b,q); 0 = settled
+    std::vector<uint8_t> ep_kind;      // [q]: W_KERNEL / W_COPY (which flag word signals it)
+    std::vector<uint64_t> ep_read;     // [q*P + r]: epoch at which r last copied out of (b,q); 0 = none
+    std::vector<void*> ipc_base;       // [q]: mapped base of a remote instance (cudaIpcCloseMemHandle)
 };
 
 struct Tap {
@@ -177,6 +183,15 @@ struct pk_ctx_s {
     int first_local = -1;    // lowest partition owned by this rank
     int nlocal = 0;          // partitions owned by this rank
     void* comm = nullptr;    // ncclComm_t (SPMD only)
+    // SPMD over peer memory (pk_init_spmd_ipc)
+    bool ipc = false;
+    pk_host_allgather_fn allgather = nullptr;
+    void* ag_user = nullptr;
+    uint64_t* flag_local = nullptr;      // device words [kFlagCopied, kFlagDone] of this rank
+    std::vector<uint64_t*> flag;         // [p]: flag words of partition p's rank (mapped)
+    std::vector<void*> flag_mapped;      // [p]: mapped bases to close
+    uint64_t epoch = 0;                  // replicated launch epoch (flags are compared GEQ)
+    std::unordered_map<std::string, std::pair<void*, int>> ipc_maps;  // handle -> (mapped base, refs)
     // steady-state graph replay (pk_api.h, PK_MODE_NO_GRAPHS)
     struct Memo {
         int seen = 0;
@@ -207,6 +222,119 @@ namespace {
 
 bool valid_buf(pk_ctx c, pk_buf b) { return c && b >= 0 && b < (int64_t)c->bufs.size() && c->bufs[b].alive; }
 bool valid_kernel(pk_ctx c, pk_kernel k) { return c && k >= 0 && k < (int64_t)c->kernels.size(); }
+
+// ---- SPMD over peer memory (pk_init_spmd_ipc) ----
+constexpr int kFlagCopied = 0;  // incoming copies of epoch E complete
+constexpr int kFlagDone = 1;    // partition kernel of epoch E complete
+
+// Driver entry points, resolved through the runtime at first use (the library does
+// not link libcuda, so host-only contexts load on machines without a driver).
+struct DriverApi {
+    bool ok = false;
+    CUresult (*WaitValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned) = nullptr;
+    CUresult (*WriteValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned) = nullptr;
+    CUresult (*GetAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr) = nullptr;
+    CUresult (*GetErrorName)(CUresult, const char**) = nullptr;
+};
+const DriverApi& drv() {
+    static DriverApi d;
+    static bool tried = false;
+    if (tried) return d;
+    tried = true;
+    auto get = [](const char* name, void** fn) {
+        cudaDriverEntryPointQueryResult q;
+        return cudaGetDriverEntryPointByVersion(name, fn, CUDART_VERSION, cudaEnableDefault, &q) == cudaSuccess &&
+               q == cudaDriverEntryPointSuccess && *fn;
+    };
+    d.ok = get("cuStreamWaitValue64", (void**)&d.WaitValue64) && get("cuStreamWriteValue64", (void**)&d.WriteValue64) &&
+           get("cuMemGetAddressRange", (void**)&d.GetAddressRange) && get("cuGetErrorName", (void**)&d.GetErrorName);
+    return d;
+}
+
+#define PK_CU(call)                                                                        \
+    do {                                                                                   \
+        if (!drv().ok) return fail(PK_ERR_CUDA, "CUDA driver entry points unavailable");  \
+        CUresult e_ = drv().call;                                                          \
+        if (e_ != CUDA_SUCCESS) {                                                          \
+            const char* s_ = nullptr;                                                      \
+            drv().GetErrorName(e_, &s_);                                                   \
+            return fail(PK_ERR_CUDA, std::string(#call) + ": " + (s_ ? s_ : "CUresult")); \
+        }                                                                                  \
+    } while (0)
+
+int host_allgather(pk_ctx c, const void* send, void* recv, size_t n) {
+    if (!c->allgather || c->allgather(c->ag_user, send, recv, n) != 0)
+        return fail(PK_ERR_INVALID, "host all-gather callback failed");
+    return PK_OK;
+}
+
+// Every rank's enqueued work is complete when this returns (local drain + host barrier).
+int ipc_barrier(pk_ctx c) {
+    for (int p = 0; p < c->P; ++p) {
+        if (!c->local(p)) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        PK_CUDA(cudaStreamSynchronize(c->stream[p]));
+    }
+    char s = 0;
+    std::vector<char> all(c->world);
+    return host_allgather(c, &s, all.data(), 1);
+}
+
+// After a barrier nothing is in flight anywhere: no epoch needs waiting for.
+void ipc_settle(pk_ctx c) {
+    for (Buffer& B : c->bufs)
+        if (B.alive) {
+            std::fill(B.ep_mod.begin(), B.ep_mod.end(), 0ull);
+            std::fill(B.ep_read.begin(), B.ep_read.end(), 0ull);
+        }
+}
+
+// Map a remote allocation (the same handle may back several buffers: reference counted).
+int ipc_open(pk_ctx c, const cudaIpcMemHandle_t& h, void** out) {
+    std::string key((const char*)&h, sizeof h);
+    auto it = c->ipc_maps.find(key);
+    if (it != c->ipc_maps.end()) {
+        it->second.second += 1;
+        *out = it->second.first;
+        return PK_OK;
+    }
+    void* m = nullptr;
+    PK_CUDA(cudaIpcOpenMemHandle(&m, h, cudaIpcMemLazyEnablePeerAccess));
+    c->ipc_maps[key] = {m, 1};
+    *out = m;
+    return PK_OK;
+}
+
+void ipc_close(pk_ctx c, void* base) {
+    for (auto it = c->ipc_maps.begin(); it != c->ipc_maps.end(); ++it)
+        if (it->second.first == base) {
+            if (--it->second.second == 0) {
+                cudaIpcCloseMemHandle(base);
+                c->ipc_maps.erase(it);
+            }
+            return;
+        }
+}
+
+// Per-stream wait list: the max epoch needed from each partition's two flag words.
+struct FlagWaits {
+    std::vector<uint64_t> need;  // [q*2 + word]
+    explicit FlagWaits(int P) : need(2 * P, 0) {}
+    void add(int q, int word, uint64_t e) { need[2 * q + word] = std::max(need[2 * q + word], e); }
+    int issue(pk_ctx c, cudaStream_t s) {
+        for (size_t i = 0; i < need.size(); ++i)
+            if (need[i])
+                PK_CU(WaitValue64((CUstream)s, (CUdeviceptr)(c->flag[i / 2] + (i % 2)), need[i],
+                                          CU_STREAM_WAIT_VALUE_GEQ));
+        return PK_OK;
+    }
+};
+
+int ipc_signal(pk_ctx c, int p, int word, uint64_t e) {
+    PK_CU(WriteValue64((CUstream)c->stream[p], (CUdeviceptr)(c->flag_local + word), e,
+                               CU_STREAM_WRITE_VALUE_DEFAULT));
+    return PK_OK;
+}
 
 // cudaMemcpy2DAsync / cudaMemcpy3DPeerAsync pitch bound (beyond it: one copy per piece)
 constexpr uint64_t kMaxCopyPitch = 1ull << 30;
@@ -321,12 +449,20 @@ int pk_nccl_unique_id(void* out, size_t bytes) {
     return PK_OK;
 }
 
-static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out);
+static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_allgather_fn ag, void* ag_user,
+                     pk_ctx* out);
 
-int pk_init(const pk_init_params* prm, pk_ctx* out) { return init_impl(prm, nullptr, out); }
-int pk_init_spmd(const pk_init_params* prm, const void* nccl_id, pk_ctx* out) { return init_impl(prm, nccl_id, out); }
+int pk_init(const pk_init_params* prm, pk_ctx* out) { return init_impl(prm, nullptr, nullptr, nullptr, out); }
+int pk_init_spmd(const pk_init_params* prm, const void* nccl_id, pk_ctx* out) {
+    return init_impl(prm, nccl_id, nullptr, nullptr, out);
+}
+int pk_init_spmd_ipc(const pk_init_params* prm, pk_host_allgather_fn ag, void* user, pk_ctx* out) {
+    if (!ag) return fail(PK_ERR_INVALID, "pk_init_spmd_ipc needs a host all-gather callback");
+    return init_impl(prm, nullptr, ag, user, out);
+}
 
-static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out) {
+static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_allgather_fn ag, void* ag_user,
+                     pk_ctx* out) {
     if (!prm || !out) return fail(PK_ERR_INVALID, "null argument");
     if (prm->nparts < 1 || prm->nparts > PK_MAX_PARTS)
         return fail(PK_ERR_INVALID, "nparts must be in [1, 64]");
@@ -338,6 +474,9 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
     c->world = prm->world_size;
     c->init_flags = prm->flags;
     c->host_only = prm->flags & PK_INIT_HOST_ONLY;
+    c->ipc = ag != nullptr && c->world > 1;
+    c->allgather = ag;
+    c->ag_user = ag_user;
     c->dev.assign(c->P, 0);
     c->prank.assign(c->P, 0);
     for (int p = 0; p < c->P; ++p) {
@@ -353,12 +492,24 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
             if (c->first_local < 0) c->first_local = p;
             c->nlocal++;
         }
+    if (c->ipc) {
+        // collective handshake: every rank must describe the same partition -> rank map
+        struct Cfg { int64_t P, world, map_hash, host_only; } mine{c->P, c->world, 1469598103934665603ll,
+                                                                   (int64_t)c->host_only};
+        for (int p = 0; p < c->P; ++p) mine.map_hash = (mine.map_hash ^ c->prank[p]) * 1099511628211ll;
+        std::vector<Cfg> all(c->world);
+        if (int r = host_allgather(c.get(), &mine, all.data(), sizeof mine)) return r;
+        for (const Cfg& x : all)
+            if (std::memcmp(&x, &mine, sizeof mine) != 0)
+                return fail(PK_ERR_INVALID, "ranks disagree on nparts / world_size / part_rank / host-only");
+    }
     if (!c->host_only) {
         int nlocal = 0;
         for (int p = 0; p < c->P; ++p) nlocal += c->local(p);
         if (c->world > 1 && nlocal != 1)
             return fail(PK_ERR_STATE, "SPMD execution needs exactly one partition per rank");
-        if (c->world > 1 && !nccl_id) return fail(PK_ERR_INVALID, "SPMD execution needs an NCCL unique id");
+        if (c->world > 1 && !nccl_id && !c->ipc)
+            return fail(PK_ERR_INVALID, "SPMD execution needs an NCCL unique id (or pk_init_spmd_ipc)");
         int ndev = 0;
         PK_CUDA(cudaGetDeviceCount(&ndev));
         if (ndev < 1) return fail(PK_ERR_CUDA, "no CUDA device");
@@ -404,7 +555,26 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_ctx* out
         PK_CUDA(cudaSetDevice(c->dev[c->first_local]));
         PK_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
         c->cur_device = c->dev[c->first_local];
-        if (c->world > 1) {
+        if (c->ipc) {
+            // epoch flag words of this rank, mapped by every other rank
+            if (int r = c->set_device(c->dev[c->first_local])) return r;
+            PK_CUDA(cudaMalloc((void**)&c->flag_local, 256));
+            PK_CUDA(cudaMemset(c->flag_local, 0, 256));
+            PK_CUDA(cudaDeviceSynchronize());
+            cudaIpcMemHandle_t h;
+            PK_CUDA(cudaIpcGetMemHandle(&h, c->flag_local));
+            std::vector<cudaIpcMemHandle_t> all(c->world);
+            if (int r = host_allgather(c.get(), &h, all.data(), sizeof h)) return r;
+            c->flag.assign(c->P, nullptr);
+            c->flag_mapped.assign(c->P, nullptr);
+            for (int p = 0; p < c->P; ++p) {
+                if (c->local(p)) { c->flag[p] = c->flag_local; continue; }
+                void* m = nullptr;
+                if (int r = ipc_open(c.get(), all[c->prank[p]], &m)) return r;
+                c->flag[p] = (uint64_t*)m;
+                c->flag_mapped[p] = m;
+            }
+        } else if (c->world > 1) {
             const NcclApi& n = nccl();
             if (!n.ok) return fail(PK_ERR_NCCL, "libnccl.so.2 could not be loaded (set PK_NCCL_LIB)");
             if (int r = c->set_device(c->dev[c->first_local])) return r;
@@ -551,11 +721,23 @@ int pk_finalize(pk_ctx c) {
     if (!c->host_only) {
         pk_synchronize(c);
         drain_timing(c);
+        if (c->ipc) {
+            // nobody may still read our instances / flags; unmap theirs before they free them
+            ipc_barrier(c);
+            for (Buffer& B : c->bufs)
+                if (B.alive)
+                    for (int p = 0; p < c->P; ++p)
+                        if (B.ipc_base[p]) { ipc_close(c, B.ipc_base[p]); B.ipc_base[p] = nullptr; B.inst[p] = nullptr; }
+            for (void* m : c->flag_mapped)
+                if (m) ipc_close(c, m);
+            ipc_barrier(c);
+            if (c->flag_local) { cudaSetDevice(c->dev[c->first_local]); cudaFree(c->flag_local); }
+        }
         for (size_t b = 0; b < c->bufs.size(); ++b) {
             Buffer& B = c->bufs[b];
             if (B.alive && B.owned)
                 for (int p = 0; p < c->P; ++p)
-                    if (B.inst[p]) { cudaSetDevice(c->dev[p]); cudaFree(B.inst[p]); }
+                    if (B.inst[p] && c->local(p)) { cudaSetDevice(c->dev[p]); cudaFree(B.inst[p]); }
         }
         clear_memo(c);
         for (int p = 0; p < c->P; ++p) {
@@ -598,6 +780,10 @@ int pk_register_buffer(pk_ctx c, int ndim, const int64_t* shape, int elem_bytes,
     B.inst.assign(c->P, nullptr);
     B.last_writer.assign(c->P, W_NONE);
     B.readers.assign(c->P, 0);
+    B.ep_mod.assign(c->P, 0);
+    B.ep_kind.assign(c->P, W_NONE);
+    B.ep_read.assign((size_t)c->P * c->P, 0);
+    B.ipc_base.assign(c->P, nullptr);
     const uint64_t all = c->P == 64 ? ~0ull : ((1ull << c->P) - 1);
     B.tracker.init(B.bytes, all);  // reading Q3: undefined contents are valid everywhere
     if (!c->host_only) {
@@ -624,6 +810,35 @@ int pk_register_buffer(pk_ctx c, int ndim, const int64_t* shape, int elem_bytes,
             }
         }
     }
+    if (c->ipc && !c->host_only) {
+        // collective: export this rank's instance, map every other rank's (pulled from later)
+        struct Exp {
+            cudaIpcMemHandle_t h;
+            uint64_t off;
+            int64_t valid;
+        } mine{};
+        const int p0 = c->first_local;
+        if (B.bytes) {
+            CUdeviceptr base = 0;
+            size_t sz = 0;
+            if (int r = c->set_device(c->dev[p0])) return r;
+            PK_CU(GetAddressRange(&base, &sz, (CUdeviceptr)B.inst[p0]));
+            PK_CUDA(cudaIpcGetMemHandle(&mine.h, (void*)base));
+            mine.off = (uint64_t)((CUdeviceptr)B.inst[p0] - base);
+            mine.valid = 1;
+        }
+        std::vector<Exp> all(c->world);
+        if (int r = host_allgather(c, &mine, all.data(), sizeof mine)) return r;
+        for (int q = 0; q < c->P; ++q) {
+            if (c->local(q)) continue;
+            const Exp& x = all[c->prank[q]];
+            if (!x.valid) continue;
+            void* m = nullptr;
+            if (int r = ipc_open(c, x.h, &m)) return r;
+            B.ipc_base[q] = m;
+            B.inst[q] = (char*)m + x.off;
+        }
+    }
     B.alive = true;
     c->bufs.push_back(std::move(B));
     *out = (pk_buf)(c->bufs.size() - 1);
@@ -647,9 +862,16 @@ int pk_unregister_buffer(pk_ctx c, pk_buf b) {
         if (int r = pk_synchronize(c)) return r;
         clear_memo(c);  // replay graphs may reference the instances
     }
+    if (c->ipc && !c->host_only) {
+        // collective: every rank unmaps before any rank frees
+        if (int r = ipc_barrier(c)) return r;
+        for (int q = 0; q < c->P; ++q)
+            if (B.ipc_base[q]) { ipc_close(c, B.ipc_base[q]); B.ipc_base[q] = nullptr; B.inst[q] = nullptr; }
+        if (int r = ipc_barrier(c)) return r;
+    }
     if (!c->host_only && B.owned) {
         for (int p = 0; p < c->P; ++p)
-            if (B.inst[p]) {
+            if (B.inst[p] && c->local(p)) {
                 if (int r = c->set_device(c->dev[p])) return r;
                 PK_CUDA(cudaFree(B.inst[p]));
             }
@@ -677,6 +899,8 @@ int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
     uint64_t t0 = now_ns();
     if (!c->host_only) {
         if (int r = pk_synchronize(c)) return r;  // WAR against everything in flight
+        if (c->ipc)                               // ... on every rank (peers may read our slab)
+            if (int r = ipc_barrier(c)) return r;
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
             uint64_t lo = (uint64_t)p * n / c->P * B.eb, hi = (uint64_t)(p + 1) * n / c->P * B.eb;
@@ -686,6 +910,10 @@ int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
                                     cudaMemcpyHostToDevice, c->stream[p]));
         }
         if (int r = pk_synchronize(c)) return r;
+        if (c->ipc) {  // every slab is in place before any rank pulls from it
+            if (int r = ipc_barrier(c)) return r;
+            ipc_settle(c);
+        }
         for (int p = 0; p < c->P; ++p) { B.last_writer[p] = W_NONE; B.readers[p] = 0; }
     }
     // linear distribution; tracker says slab p lives on p (reading Q2)
@@ -736,6 +964,8 @@ int pk_copy_from_host_for(pk_ctx c, pk_buf b, const void* host, size_t bytes, pk
     }
     if (!c->host_only) {
         if (int r = pk_synchronize(c)) return r;
+        if (c->ipc)
+            if (int r = ipc_barrier(c)) return r;
         for (int p = 0; p < P; ++p) {
             if (!c->local(p)) continue;
             if (int r = c->set_device(c->dev[p])) return r;
@@ -744,6 +974,10 @@ int pk_copy_from_host_for(pk_ctx c, pk_buf b, const void* host, size_t bytes, pk
                                         cudaMemcpyHostToDevice, c->stream[p]));
         }
         if (int r = pk_synchronize(c)) return r;
+        if (c->ipc) {
+            if (int r = ipc_barrier(c)) return r;
+            ipc_settle(c);
+        }
         for (int p = 0; p < P; ++p) { B.last_writer[p] = W_NONE; B.readers[p] = 0; }
     }
     B.tracker.init(B.bytes, 0);
@@ -797,13 +1031,55 @@ static int sync_to_host_spmd(pk_ctx c, Buffer& B, void* host) {
     return PK_OK;
 }
 
+static int sync_to_host_ipc(pk_ctx c, Buffer& B, void* host) {
+    // collective n:1 gather to rank 0 over peer memory: rank 0 pulls every segment its
+    // partition lacks from the lowest holder's mapped instance into its own instance
+    // (same tracker semantics as the NCCL variant), then copies the whole buffer down
+    int r0 = -1;
+    for (int p = 0; p < c->P; ++p)
+        if (c->prank[p] == 0) { r0 = p; break; }
+    if (r0 < 0) return fail(PK_ERR_STATE, "rank 0 owns no partition");
+    if (int r = ipc_barrier(c)) return r;  // every rank's writes are complete
+    RangeList received;
+    struct Piece { uint64_t b, e; int src; };
+    std::vector<Piece> pieces;
+    for (const Seg& s : B.tracker.segments()) {
+        int src = ((s.mask >> r0) & 1) ? r0 : -1;
+        for (int q = 0; q < c->P && src < 0; ++q)
+            if ((s.mask >> q) & 1) src = q;
+        if (src < 0) return fail(PK_ERR_STATE, "segment held by no partition");
+        if (!pieces.empty() && pieces.back().src == src && pieces.back().e == s.b) pieces.back().e = s.e;
+        else pieces.push_back({s.b, s.e, src});
+    }
+    for (const Piece& pc : pieces) {
+        if (pc.src == r0) continue;
+        received.push_back(Range{pc.b, pc.e});
+        if (c->rank != 0) continue;
+        if (int r = c->set_device(c->dev[r0])) return r;
+        PK_CUDA(cudaMemcpyAsync((char*)B.inst[r0] + pc.b, (const char*)B.inst[pc.src] + pc.b, pc.e - pc.b,
+                                cudaMemcpyDefault, c->stream[r0]));
+    }
+    if (c->rank == 0) {
+        if (int r = c->set_device(c->dev[r0])) return r;
+        PK_CUDA(cudaMemcpyAsync(host, B.inst[r0], B.bytes, cudaMemcpyDeviceToHost, c->stream[r0]));
+    }
+    if (int r = ipc_barrier(c)) return r;  // nobody overwrites what rank 0 read
+    ipc_settle(c);
+    if (!(c->mode & PK_MODE_SINGLE_OWNER)) {
+        canonicalize(&received);
+        B.tracker.add_bit(received, r0);
+    }
+    c->stats.d2h_bytes += c->rank == 0 ? B.bytes : 0;
+    return PK_OK;
+}
+
 int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
     if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "bad argument");
     Buffer& B = c->bufs[b];
     if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (D2H gathers the whole virtual buffer)");
     if (c->host_only) return fail(PK_ERR_STATE, "host-only context holds no data");
     if (!host && (c->world == 1 || c->rank == 0)) return fail(PK_ERR_INVALID, "null host buffer");
-    if (c->world > 1) return sync_to_host_spmd(c, B, host);
+    if (c->world > 1) return c->ipc ? sync_to_host_ipc(c, B, host) : sync_to_host_spmd(c, B, host);
     // replay graphs run on stream[p0]: fork the other streams from its tail first
     if (int r = exit_graph_mode(c)) return r;
     // query all segments, copy each from a partition that holds it.
@@ -1204,6 +1480,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     c->stats.host_ns_plan += t3 - t2;
     c->stats.launches += 1;
     const uint64_t launch_id = c->launch_counter++;
+    const uint64_t E = c->ipc ? ++c->epoch : 0;  // replicated: identical on every rank
 
     // ---- a4 + a5: transfers, pulled on the destination stream ----
     if (!c->host_only) {
@@ -1214,8 +1491,22 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 const int p = c->last_plan[i].dst;
                 size_t j = i;
                 while (j < c->last_plan.size() && c->last_plan[j].dst == p) ++j;
-                if (!c->local(p)) { i = j; continue; }  // another rank pulls (NCCL pass below)
+                if (!c->local(p)) { i = j; continue; }  // another rank pulls (NCCL / its own IPC pass)
                 if (int r = c->set_device(c->dev[p])) return r;
+                if (c->ipc) {
+                    // peer memory: RAW on the holder's flag word of its last write of (b,q);
+                    // WAR on (b,p): readers of earlier launches must have finished copying it
+                    FlagWaits fw(P);
+                    for (size_t t = i; t < j; ++t) {
+                        const CopyOp& o = c->last_plan[t];
+                        const Buffer& B = c->bufs[o.buf];
+                        if (B.ep_mod[o.src])
+                            fw.add(o.src, B.ep_kind[o.src] == W_COPY ? kFlagCopied : kFlagDone, B.ep_mod[o.src]);
+                        for (int r = 0; r < P; ++r)
+                            if (B.ep_read[(size_t)p * P + r]) fw.add(r, kFlagCopied, B.ep_read[(size_t)p * P + r]);
+                    }
+                    if (int r = fw.issue(c, c->stream[p])) return r;
+                }
                 // WAR on the destination instances + RAW on each source's last writer
                 uint64_t waited_src = 0;
                 for (size_t t = i; t < j; ++t) {
@@ -1258,7 +1549,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 };
                 for (size_t t = 0; t < order.size();) {
                     const CopyOp& o = c->last_plan[order[t]];
-                    if (!c->local(o.src)) { ++t; continue; }
+                    if (!c->local(o.src) && !c->ipc) { ++t; continue; }
                     const uint64_t len = o.e - o.b;
                     uint64_t pitch = 0;
                     size_t u = run2d(t, &pitch);
@@ -1288,7 +1579,9 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     Buffer& B = c->bufs[o.buf];
                     char* dst = (char*)B.inst[p] + o.b;
                     const char* src = (const char*)B.inst[o.src] + o.b;
-                    const bool same_dev = c->dev[o.src] == c->dev[p];
+                    // IPC-mapped peer instances are addressed through UVA (cudaMemcpyDefault)
+                    const bool same_dev = c->ipc || c->dev[o.src] == c->dev[p];
+                    const cudaMemcpyKind dkind = c->ipc ? cudaMemcpyDefault : cudaMemcpyDeviceToDevice;
                     if ((rows > 1 || nslab > 1) && len <= kNarrowPiece) {
                         // narrow strided run (a halo column): pulled by the destination's SMs
                         PK_CUDA(launch_strided_copy(dst, src, len, pitch, rows, slice, nslab, c->sm_count[p],
@@ -1301,7 +1594,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                             pp.srcPtr = make_cudaPitchedPtr((void*)src, pitch, len, ysz);
                             pp.dstPtr = make_cudaPitchedPtr(dst, pitch, len, ysz);
                             pp.extent = make_cudaExtent(len, rows, nslab);
-                            pp.kind = cudaMemcpyDeviceToDevice;
+                            pp.kind = dkind;
                             PK_CUDA(cudaMemcpy3DAsync(&pp, c->stream[p]));
                         } else {
                             cudaMemcpy3DPeerParms pp = {};
@@ -1314,12 +1607,11 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                         }
                     } else if (rows == 1) {
                         if (same_dev)
-                            PK_CUDA(cudaMemcpyAsync(dst, src, len, cudaMemcpyDeviceToDevice, c->stream[p]));
+                            PK_CUDA(cudaMemcpyAsync(dst, src, len, dkind, c->stream[p]));
                         else
                             PK_CUDA(cudaMemcpyPeerAsync(dst, c->dev[p], src, c->dev[o.src], len, c->stream[p]));
                     } else if (same_dev) {
-                        PK_CUDA(cudaMemcpy2DAsync(dst, pitch, src, pitch, len, rows, cudaMemcpyDeviceToDevice,
-                                                  c->stream[p]));
+                        PK_CUDA(cudaMemcpy2DAsync(dst, pitch, src, pitch, len, rows, dkind, c->stream[p]));
                     } else {
                         cudaMemcpy3DPeerParms pp = {};
                         pp.srcPtr = make_cudaPitchedPtr((void*)src, pitch, len, rows);
@@ -1337,6 +1629,8 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     t = u;
                 }
                 PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
+                if (c->ipc)
+                    if (int r = ipc_signal(c, p, kFlagCopied, E)) return r;
                 for (size_t t = i; t < j; ++t) {
                     const CopyOp& o = c->last_plan[t];
                     if (!c->local(o.src)) continue;
@@ -1349,7 +1643,20 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             // SPMD: copies between ranks are NCCL send/recv pairs issued in the
             // global plan order on both sides (one partition per rank, so stream
             // order on that partition covers RAW and both WARs).
-            if (c->world > 1) {
+            if (c->ipc) {
+                // replicated bookkeeping (every rank, every partition): WAR entries of the
+                // destinations are consumed, then this launch's reads and copy-writes recorded
+                for (const CopyOp& o : c->last_plan) {
+                    Buffer& B = c->bufs[o.buf];
+                    std::fill(B.ep_read.begin() + (size_t)o.dst * P, B.ep_read.begin() + (size_t)(o.dst + 1) * P, 0ull);
+                }
+                for (const CopyOp& o : c->last_plan) {
+                    Buffer& B = c->bufs[o.buf];
+                    B.ep_read[(size_t)o.src * P + o.dst] = E;
+                    B.ep_mod[o.dst] = E;
+                    B.ep_kind[o.dst] = W_COPY;
+                }
+            } else if (c->world > 1) {
                 const NcclApi& n = nccl();
                 bool open = false;
                 for (const CopyOp& o : c->last_plan) {
@@ -1381,12 +1688,21 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 }
             }
         }
-        if (mode & PK_MODE_GLOBAL_BARRIER)  // Fig. 4 line 8, literally
+        if (mode & PK_MODE_GLOBAL_BARRIER) {  // Fig. 4 line 8, literally
             if (int r = pk_synchronize(c)) return r;
+            if (c->ipc) {
+                if (int r = ipc_barrier(c)) return r;
+                ipc_settle(c);
+            }
+        }
     }
     uint64_t t4 = now_ns();
 
     // ---- a6: partitioned launches (Eq. 8-10) ----
+    bool writes_arg[PK_MAX_ARGS] = {};
+    for (int a = 0; a < K.nargs; ++a)
+        for (const Tap& t : K.taps)
+            if (t.arg == a && t.mode != PK_READ) writes_arg[a] = true;
     if (!c->host_only) {
         void* inst[PK_MAX_ARGS];
         void* argv[PK_MAX_ARGS + 1];
@@ -1394,6 +1710,18 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             const Regions& R = (*regs)[p];
             if (R.empty || !c->local(p)) continue;
             if (int r = c->set_device(c->dev[p])) return r;
+            if (c->ipc) {
+                // WAR across ranks: readers of (b,p) -- this launch's included -- must have
+                // finished their copies before p's kernel overwrites b
+                FlagWaits fw(P);
+                for (int a = 0; a < K.nargs; ++a) {
+                    if (!bound[a] || !(writes_arg[a] || !track)) continue;
+                    const Buffer& B = c->bufs[bid[a]];
+                    for (int r = 0; r < P; ++r)
+                        if (B.ep_read[(size_t)p * P + r]) fw.add(r, kFlagCopied, B.ep_read[(size_t)p * P + r]);
+                }
+                if (int r = fw.issue(c, c->stream[p])) return r;
+            }
             // WAR: writes into (b,p) wait for copies that read (b,p)
             if (track) {
                 for (auto& bs : sets[p])
@@ -1440,6 +1768,8 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 c->pending_timing.push_back(TimedLaunch{e0, e1, p, launch_id});
             }
             if (P > 1) PK_CUDA(cudaEventRecord(c->ev_kernel[p], c->stream[p]));
+            if (c->ipc)
+                if (int r = ipc_signal(c, p, kFlagDone, E)) return r;
             c->stats.kernel_launches += 1;
             for (int a = 0; a < K.nargs; ++a)
                 if (bound[a]) {
@@ -1452,6 +1782,19 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     } else {
         for (int p = 0; p < P; ++p)
             if (!(*regs)[p].empty && c->local(p)) c->stats.kernel_launches += 1;
+    }
+    if (c->ipc) {
+        // replicated: the kernels' writes consume the WAR entries and become the last writes
+        for (int p = 0; p < P; ++p) {
+            if ((*regs)[p].empty) continue;
+            for (int a = 0; a < K.nargs; ++a) {
+                if (!bound[a] || !(writes_arg[a] || !track)) continue;
+                Buffer& B = c->bufs[bid[a]];
+                std::fill(B.ep_read.begin() + (size_t)p * P, B.ep_read.begin() + (size_t)(p + 1) * P, 0ull);
+                B.ep_mod[p] = E;
+                B.ep_kind[p] = W_KERNEL;
+            }
+        }
     }
     uint64_t t5 = now_ns();
     c->stats.host_ns_issue += (t4 - t3) + (t5 - t4);

@@ -60,14 +60,19 @@ def _sequence(abi, K, ctx, kernel, world):
     return out
 
 
-def _worker(rank, world, port, kernel, qdir):
+def _worker(rank, world, port, kernel, qdir, transport="nccl"):
     import sys
     sys.path.insert(0, ROOT)
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_icppw_matzdf20_b200 import abi
     from paper_conf_icppw_matzdf20_b200 import kernels as K
-    ctx = abi.pk_init_spmd(world, rank, world, list(range(world)), flags=abi.PK_INIT_HOST_ONLY)
+    if transport == "ipc":   # peer-memory transport: the host all-gather callback runs (handshake)
+        from paper_conf_icppw_matzdf20_b200 import spmd
+        ctx = abi.pk_init_spmd_ipc(world, rank, world, list(range(world)), spmd.dist_allgather(),
+                                   flags=abi.PK_INIT_HOST_ONLY)
+    else:
+        ctx = abi.pk_init_spmd(world, rank, world, list(range(world)), flags=abi.PK_INIT_HOST_ONLY)
     seq = _sequence(abi, K, ctx, kernel, world)
     launches = abi.pk_get_stats(ctx)["kernel_launches"]
     abi.pk_finalize(ctx)
@@ -81,10 +86,11 @@ def _worker(rank, world, port, kernel, qdir):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("kernel", ["jacobi2d", "hotspot2d", "nbody"])
-def test_spmd_two_ranks_replicated_plan_and_matched_transfers(kernel, tmp_path):
+@pytest.mark.parametrize("kernel,transport", [("jacobi2d", "nccl"), ("hotspot2d", "nccl"), ("nbody", "nccl"),
+                                              ("hotspot2d", "ipc")])
+def test_spmd_two_ranks_replicated_plan_and_matched_transfers(kernel, transport, tmp_path):
     world = 2
-    mp.spawn(_worker, args=(world, _free_port(), kernel, str(tmp_path)), nprocs=world, join=True)
+    mp.spawn(_worker, args=(world, _free_port(), kernel, str(tmp_path), transport), nprocs=world, join=True)
     import pickle
     allseq = pickle.load(open(tmp_path / "res.pkl", "rb"))
     (seq0, l0), (seq1, l1) = allseq
@@ -112,3 +118,28 @@ def test_spmd_two_ranks_replicated_plan_and_matched_transfers(kernel, tmp_path):
                 assert sends == recvs
                 moved += sum(hi - lo for (_, lo, hi) in sends)
     assert moved == seq0[-1][1] > 0          # all stale bytes cross ranks (one partition per rank)
+
+
+def _mismatch_worker(rank, world, port, qdir):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icppw_matzdf20_b200 import abi, spmd
+    part_rank = [0, 1] if rank == 0 else [1, 0]      # the ranks disagree on the partition map
+    err = None
+    try:
+        ctx = abi.pk_init_spmd_ipc(2, rank, world, part_rank, spmd.dist_allgather(), flags=abi.PK_INIT_HOST_ONLY)
+        abi.pk_finalize(ctx)
+    except abi.PkError as e:
+        err = e.name
+    with open(os.path.join(qdir, f"r{rank}.txt"), "w") as f:
+        f.write(str(err))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_spmd_ipc_handshake_rejects_inconsistent_ranks(tmp_path):
+    """pk_init_spmd_ipc's collective handshake: every rank fails PK_ERR_INVALID."""
+    mp.spawn(_mismatch_worker, args=(2, _free_port(), str(tmp_path)), nprocs=2, join=True)
+    assert [(tmp_path / f"r{r}.txt").read_text() for r in range(2)] == ["PK_ERR_INVALID"] * 2
