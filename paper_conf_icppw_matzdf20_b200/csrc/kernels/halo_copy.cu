@@ -28,7 +28,51 @@ __global__ void __launch_bounds__(256) k_strided_copy(char* __restrict__ dst, co
     }
 }
 
+// Epoch flags of the peer-memory SPMD transport, SM variant (used when the driver
+// refuses stream memory operations on a mapped peer address): one thread spins
+// with system-scope acquire loads until every flag reaches its target / stores a
+// flag with system-scope release after the stream's earlier work.
+struct FlagWaitList {
+    const unsigned long long* flag[8];
+    unsigned long long target[8];
+    int n;
+};
+
+__global__ void k_flag_wait(FlagWaitList w) {
+    for (int i = 0; i < w.n; ++i) {
+        unsigned long long v;
+        do {
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(w.flag[i]) : "memory");
+            if (v >= w.target[i]) break;
+            __nanosleep(256);
+        } while (true);
+    }
+}
+
+__global__ void k_flag_write(unsigned long long* flag, unsigned long long v) {
+    __threadfence_system();
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(flag), "l"(v) : "memory");
+}
+
 }  // namespace
+
+cudaError_t launch_flag_wait(const uint64_t* const* flags, const uint64_t* targets, int n, cudaStream_t stream) {
+    for (int i0 = 0; i0 < n; i0 += 8) {
+        FlagWaitList w{};
+        w.n = n - i0 < 8 ? n - i0 : 8;
+        for (int i = 0; i < w.n; ++i) {
+            w.flag[i] = reinterpret_cast<const unsigned long long*>(flags[i0 + i]);
+            w.target[i] = targets[i0 + i];
+        }
+        k_flag_wait<<<1, 1, 0, stream>>>(w);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_flag_write(uint64_t* flag, uint64_t v, cudaStream_t stream) {
+    k_flag_write<<<1, 1, 0, stream>>>(reinterpret_cast<unsigned long long*>(flag), v);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_strided_copy(char* dst, const char* src, uint64_t len, uint64_t pitch, uint64_t rows,
                                 uint64_t slice, uint64_t nslab, int sm_count, cudaStream_t stream) {

@@ -52,6 +52,11 @@ extern const Builtin kBuiltinSgemm;          // sgemm_tf32x3 (tcgen05 3xTF32)
 cudaError_t launch_strided_copy(char* dst, const char* src, uint64_t len, uint64_t pitch, uint64_t rows,
                                 uint64_t slice, uint64_t nslab, int sm_count, cudaStream_t stream);
 
+// Epoch flags of the peer-memory SPMD transport on the SMs (fallback of the stream
+// memory operations): wait until *flags[i] >= targets[i] for all i; store *flag = v.
+cudaError_t launch_flag_wait(const uint64_t* const* flags, const uint64_t* targets, int n, cudaStream_t stream);
+cudaError_t launch_flag_write(uint64_t* flag, uint64_t v, cudaStream_t stream);
+
 // Descriptor helpers used by the kernel files' describe() functions.
 inline pk_expr E(int64_t c0) {
     pk_expr e{};

@@ -191,6 +191,7 @@ struct pk_ctx_s {
     std::vector<uint64_t*> flag;         // [p]: flag words of partition p's rank (mapped)
     std::vector<void*> flag_mapped;      // [p]: mapped bases to close
     uint64_t epoch = 0;                  // replicated launch epoch (flags are compared GEQ)
+    bool flags_on_sm = false;            // epoch flags by SM kernels instead of stream memory operations
     std::unordered_map<std::string, std::pair<void*, int>> ipc_maps;  // handle -> (mapped base, refs)
     // steady-state graph replay (pk_api.h, PK_MODE_NO_GRAPHS)
     struct Memo {
@@ -317,22 +318,44 @@ void ipc_close(pk_ctx c, void* base) {
 }
 
 // Per-stream wait list: the max epoch needed from each partition's two flag words.
+// Issued as stream memory operations (cuStreamWaitValue64, processed by the stream
+// front end, no SM); if the driver refuses them for a mapped peer address the
+// context switches to the SM spin-wait kernels for good (PK_FLAGS_SM env forces it).
 struct FlagWaits {
     std::vector<uint64_t> need;  // [q*2 + word]
     explicit FlagWaits(int P) : need(2 * P, 0) {}
     void add(int q, int word, uint64_t e) { need[2 * q + word] = std::max(need[2 * q + word], e); }
     int issue(pk_ctx c, cudaStream_t s) {
+        std::vector<const uint64_t*> fl;
+        std::vector<uint64_t> tg;
         for (size_t i = 0; i < need.size(); ++i)
-            if (need[i])
-                PK_CU(WaitValue64((CUstream)s, (CUdeviceptr)(c->flag[i / 2] + (i % 2)), need[i],
-                                          CU_STREAM_WAIT_VALUE_GEQ));
+            if (need[i]) {
+                const uint64_t* f = c->flag[i / 2] + (i % 2);
+                if (!c->flags_on_sm) {
+                    CUresult e = drv().ok ? drv().WaitValue64((CUstream)s, (CUdeviceptr)f, need[i],
+                                                              CU_STREAM_WAIT_VALUE_GEQ)
+                                          : CUDA_ERROR_NOT_SUPPORTED;
+                    if (e == CUDA_SUCCESS) continue;
+                    c->flags_on_sm = true;
+                }
+                fl.push_back(f);
+                tg.push_back(need[i]);
+            }
+        if (!fl.empty()) PK_CUDA(launch_flag_wait(fl.data(), tg.data(), (int)fl.size(), s));
         return PK_OK;
     }
 };
 
 int ipc_signal(pk_ctx c, int p, int word, uint64_t e) {
-    PK_CU(WriteValue64((CUstream)c->stream[p], (CUdeviceptr)(c->flag_local + word), e,
-                               CU_STREAM_WRITE_VALUE_DEFAULT));
+    uint64_t* f = c->flag_local + word;
+    if (!c->flags_on_sm) {
+        CUresult r = drv().ok ? drv().WriteValue64((CUstream)c->stream[p], (CUdeviceptr)f, e,
+                                                   CU_STREAM_WRITE_VALUE_DEFAULT)
+                              : CUDA_ERROR_NOT_SUPPORTED;
+        if (r == CUDA_SUCCESS) return PK_OK;
+        c->flags_on_sm = true;
+    }
+    PK_CUDA(launch_flag_write(f, e, c->stream[p]));
     return PK_OK;
 }
 
@@ -556,6 +579,7 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
         PK_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
         c->cur_device = c->dev[c->first_local];
         if (c->ipc) {
+            c->flags_on_sm = getenv("PK_FLAGS_SM") != nullptr;
             // epoch flag words of this rank, mapped by every other rank
             if (int r = c->set_device(c->dev[c->first_local])) return r;
             PK_CUDA(cudaMalloc((void**)&c->flag_local, 256));

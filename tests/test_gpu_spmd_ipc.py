@@ -28,13 +28,17 @@ def _free_port():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("world", [2, 3])
-def test_spmd_ipc_processes_match_one_way(world, tmp_path):
+@pytest.mark.parametrize("world,flags_on_sm", [(2, False), (3, False), (2, True)])
+def test_spmd_ipc_processes_match_one_way(world, flags_on_sm, tmp_path):
+    """flags_on_sm: epoch flags by the SM spin/store kernels instead of stream memory operations."""
     out = tmp_path / "report.json"
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr=127.0.0.1", f"--master-port={_free_port()}",
            os.path.join(ROOT, "tests", "spmd_ipc_worker.py"), str(out)]
     env = dict(os.environ, OMP_NUM_THREADS="1")
+    env.pop("PK_FLAGS_SM", None)
+    if flags_on_sm:
+        env["PK_FLAGS_SM"] = "1"
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
     assert r.returncode == 0, (r.stdout[-4000:], r.stderr[-4000:])
     rep = json.loads(out.read_text())
