@@ -12,10 +12,15 @@
 // per lattice update halves (6 B/LU instead of 12 B/LU).
 //
 // Design = hotspot_tma.cu's TMA bulk ring (persistent CTAs, producer thread,
-// mbarrier full/empty, alternating march direction) plus a 4-row shared-memory
-// ring for the intermediate sweep: at input row q the 4 consumer warps compute
-// sweep-1 row q-1 (columns c0-1 .. c0+512, edge lanes add the two halo columns),
-// sync on a named barrier, then compute sweep-2 row q-2 and store it.
+// mbarrier full/empty, alternating march direction); the consumers keep both
+// sweeps in registers: a thread owns 4 columns for the whole tile and carries
+// 3-row windows of the input and of sweep 1, so per input row q it loads one new
+// input row (+ power), computes sweep-1 row q-1 and sweep-2 row q-2 and stores
+// it.  W/E neighbours come from warp shuffles; the warp's edge lanes also compute
+// sweep 1 on the column just outside the warp (redundantly, bit-identically), so
+// the 4 consumer warps never synchronise with each other -- only with the ring.
+// (v1 staged sweep 1 through a shared-memory row ring with a named barrier per
+// row: 521 M issued instructions per launch at C2, issue-bound at 76 % of HBM.)
 #include <cuda_runtime.h>
 
 #include "../runtime/builtins.h"
@@ -35,16 +40,13 @@ constexpr int kRowF = kTC + 2 * kHalo;    // 520 floats per row segment
 constexpr int kStageFloats = 2 * kRowF;   // temp row + power row
 constexpr int kStageBytes = kStageFloats * 4;
 constexpr int kNS = 8;                    // input ring depth
-constexpr int kS1 = 4;                    // sweep-1 row ring
 constexpr int kConsumers = 128;
 constexpr int kThreads = kConsumers + 32;
-constexpr size_t kSmem = (size_t)kNS * kStageBytes + (size_t)kS1 * kRowF * 4 + 2 * kNS * sizeof(uint64_t);
+constexpr size_t kSmem = (size_t)kNS * kStageBytes + 2 * kNS * sizeof(uint64_t);
 
 __device__ __forceinline__ float hs(float c, float n, float s, float e, float w, float p) {
     return c + kCap * (p + (s + n - 2.0f * c) * kRy1 + (e + w - 2.0f * c) * kRx1 + (kAmb - c) * kRz1);
 }
-
-__device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 
 __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restrict__ tin,
                                                             const float* __restrict__ pw,
@@ -52,8 +54,7 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
                                                             int64_t TY, pk_partition part) {
     extern __shared__ __align__(128) unsigned char smem[];
     float* ring = reinterpret_cast<float*>(smem);
-    float* s1 = ring + (size_t)kNS * kStageFloats;  // [kS1][kRowF]
-    uint64_t* full = reinterpret_cast<uint64_t*>(s1 + (size_t)kS1 * kRowF);
+    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)kNS * kStageFloats);
     uint64_t* empty = full + kNS;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
@@ -91,105 +92,102 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
         return;
     }
 
-    // ---------------- consumers: thread owns columns c0 + 4*tc .. +3
+    // ---------------- consumers: thread owns columns j0 = c0 + 4*tc .. j0+3 for every row.
+    // Everything a thread needs vertically stays in registers (3-row windows of the
+    // input and of sweep 1); horizontal neighbours come from warp shuffles.  Each warp
+    // is independent: its two edge lanes also compute sweep 1 at the column just
+    // outside the warp (lane 0: w0-1, lane 31: w0+128) -- the warp's own halo,
+    // recomputed redundantly with identical inputs and operation order -- so no
+    // barrier among consumers is needed and warps drift freely through the ring.
     const int tc = threadIdx.x;
+    const bool left = lane == 0;          // edge lane: extra column w0-1 (left) or w0+128 (right)
     uint32_t g = 0;
     for (int64_t T = blockIdx.x; T < ntiles; T += gridDim.x) {
         const int64_t bx = part.min[0] + T % gx, by = part.min[1] + T / gx;
         const int64_t c0 = bx * kTC, r0 = by * TY, rend = min(r0 + TY, H), nr = rend - r0;
         const bool down = (by & 1) == 0;
-        const int64_t dir = down ? 1 : -1;
-        const int64_t rstart = down ? r0 - 2 : rend + 1;  // input row of sequence index 0
+        const int dir = down ? 1 : -1;
         const int64_t j0 = c0 + 4 * tc;
         const bool active = j0 < W;
         const int cx = kHalo + 4 * tc;  // smem column of j0
-        // clamped smem columns of the west/east neighbours of j0 and j0+3
-        const int cw = j0 == 0 ? cx : cx - 1;
-        const int ce = j0 + 4 >= W ? cx + 3 : cx + 4;
-        ptx::mbar_wait(&full[g % kNS], (g / kNS) & 1u);
-        ptx::mbar_wait(&full[(g + 1) % kNS], ((g + 1) / kNS) & 1u);
-        static_assert((kNS & (kNS - 1)) == 0 && (kS1 & (kS1 - 1)) == 0, "rings are powers of two");
+        const bool wclamp = j0 == 0;            // west neighbour of j0 is j0 itself (grid border)
+        const bool eclamp = j0 + 4 >= W;        // east neighbour of j0+3 is j0+3 itself
+        // extra column of the edge lanes (other lanes evaluate a harmless copy of their own)
+        const int64_t xe = left ? j0 - 1 : j0 + 4;
+        const bool xneed = (lane == 0 || lane == 31) && xe >= 0 && xe < W;
+        const int xc = xneed ? (left ? cx - 1 : cx + 4) : cx;          // smem column of xe
+        const int xf = xneed ? (left ? cx - 2 : (xe + 1 < W ? cx + 5 : cx + 4)) : cx;  // far neighbour
+        // W/E neighbours the edge lanes take from the extra column instead of a shuffle
+        const bool use_xw = lane == 0 && xneed, use_xe = lane == 31 && xneed;
+        const float* st = ring + (size_t)(g & (kNS - 1)) * kStageFloats;
+        ptx::mbar_wait(&full[g & (kNS - 1)], (g / kNS) & 1u);
+        const float4 in0 = *reinterpret_cast<const float4*>(st + cx);
+        const float x0 = st[xc];
+        st = ring + (size_t)((g + 1) & (kNS - 1)) * kStageFloats;
+        ptx::mbar_wait(&full[(g + 1) & (kNS - 1)], ((g + 1) / kNS) & 1u);
+        float4 inA = in0, inB = *reinterpret_cast<const float4*>(st + cx);  // input rows seq t-2, t-1
+        float xA = x0, xB = st[xc];
+        float4 s1A = make_float4(0.f, 0.f, 0.f, 0.f), s1B = s1A;         // sweep-1 rows seq t-3, t-2
+        float eB = 0.f;                                                  // extra column, sweep 1, seq t-2
+        float4 pA = s1A;                                                  // power, seq t-2
         const int nt = (int)nr + 4;
-        int row1 = (int)(rstart + dir);              // sweep-1 row of iteration t = 2
-        float* outp = tout + (rstart + 2 * dir) * W + j0;  // sweep-2 row of iteration t = 4
+        int row1 = (int)((down ? r0 - 2 : rend + 1) + dir);  // grid row of sweep-1 seq t-1 (t = 2)
+        const int Hi = (int)H;
+        float* outp = tout + ((down ? r0 - 2 : rend + 1) + 2 * dir) * W + j0;  // sweep-2 row, t = 4
         const int64_t dW = dir * W;
-        for (int t = 2; t < nt; ++t, row1 += (int)dir) {
-            // input rows (sequence) t-2, t-1, t are in the ring; compute sweep-1 of
-            // the row at sequence t-1 (rows r0-1 .. rend in march order), then sweep-2
-            // of the row at sequence t-2 (rows r0 .. rend-1).
+        for (int t = 2; t < nt; ++t, row1 += dir) {
             const uint32_t gq = g + (uint32_t)t;
             ptx::mbar_wait(&full[gq & (kNS - 1)], (gq / kNS) & 1u);
-            const float* sa = ring + ((gq - 2) & (kNS - 1)) * kStageFloats;  // seq t-2
-            const float* sb = ring + ((gq - 1) & (kNS - 1)) * kStageFloats;  // seq t-1
-            const float* sc = ring + (gq & (kNS - 1)) * kStageFloats;        // seq t
-            const bool need1 = row1 >= 0 && row1 < H;      // rows outside the grid are never read
-            float* s1row = s1 + ((t - 1) & (kS1 - 1)) * kRowF;
-            if (need1) {
-                // sweep 1 on columns j0..j0+3 (N/S = rows t-2 / t, order-independent)
-                const float4 c = *reinterpret_cast<const float4*>(sb + cx);
-                const float4 a = *reinterpret_cast<const float4*>(sa + cx);
-                const float4 b = *reinterpret_cast<const float4*>(sc + cx);
-                const float4 p = *reinterpret_cast<const float4*>(sb + kRowF + cx);
-                float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
-                float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
-                if (lane == 0) wv = sb[cw];
-                if (lane == 31 || j0 + 4 >= W) ev = sb[ce];
-                if (j0 == 0) wv = c.x;
+            const float* sc = ring + (size_t)(gq & (kNS - 1)) * kStageFloats;        // seq t
+            const float* sb = ring + (size_t)((gq - 1) & (kNS - 1)) * kStageFloats;  // seq t-1
+            const float4 inC = *reinterpret_cast<const float4*>(sc + cx);
+            const float4 pB = *reinterpret_cast<const float4*>(sb + kRowF + cx);     // power, seq t-1
+            const float xC = sc[xc], xfar = sb[xf], xp = sb[kRowF + xc];
+            // ---- sweep 1 at seq t-1 (own 4 columns + the edge lane's extra column)
+            float wv = __shfl_up_sync(0xffffffffu, inB.w, 1);
+            float ev = __shfl_down_sync(0xffffffffu, inB.x, 1);
+            if (use_xw) wv = xB;
+            if (use_xe) ev = xB;
+            if (wclamp) wv = inB.x;
+            if (eclamp) ev = inB.w;
+            float4 s1C;
+            s1C.x = hs(inB.x, inA.x, inC.x, inB.y, wv, pB.x);
+            s1C.y = hs(inB.y, inA.y, inC.y, inB.z, inB.x, pB.y);
+            s1C.z = hs(inB.z, inA.z, inC.z, inB.w, inB.y, pB.z);
+            s1C.w = hs(inB.w, inA.w, inC.w, ev, inB.z, pB.w);
+            // extra column xe: its near neighbour is the lane's own j0 (left) / j0+3 (right)
+            const float eC = left ? hs(xB, xA, xC, inB.x, xfar, xp) : hs(xB, xA, xC, xfar, inB.w, xp);
+            // ---- sweep 2 at seq t-2 (rows r0 .. rend-1), from the sweep-1 window
+            if (t >= 4) {
+                const int row2 = row1 - dir;
+                const bool nin = (unsigned)(row2 - dir) < (unsigned)Hi, sin_ = (unsigned)row1 < (unsigned)Hi;
+                const float4 n4 = nin ? s1A : s1B, s4 = sin_ ? s1C : s1B;
+                float w2 = __shfl_up_sync(0xffffffffu, s1B.w, 1);
+                float e2 = __shfl_down_sync(0xffffffffu, s1B.x, 1);
+                if (use_xw) w2 = eB;
+                if (use_xe) e2 = eB;
+                if (wclamp) w2 = s1B.x;
+                if (eclamp) e2 = s1B.w;
                 float4 o;
-                o.x = hs(c.x, a.x, b.x, c.y, wv, p.x);
-                o.y = hs(c.y, a.y, b.y, c.z, c.x, p.y);
-                o.z = hs(c.z, a.z, b.z, c.w, c.y, p.z);
-                o.w = hs(c.w, a.w, b.w, ev, c.z, p.w);
-                *reinterpret_cast<float4*>(s1row + cx) = o;
-                // the two sweep-1 halo columns c0-1 and c0+512 (if inside the grid)
-                if (tc == 0 && c0 > 0) {
-                    const int k = kHalo - 1;  // column c0-1: neighbours c0-2 (clamped) and c0
-                    const int kw = c0 - 2 >= 0 ? k - 1 : k;
-                    s1row[k] = hs(sb[k], sa[k], sc[k], sb[k + 1], sb[kw], sb[kRowF + k]);
-                }
-                if (tc == kConsumers - 1 && c0 + kTC < W) {
-                    const int k = kHalo + kTC;  // column c0+512
-                    const int ke = c0 + kTC + 1 < W ? k + 1 : k;
-                    s1row[k] = hs(sb[k], sa[k], sc[k], sb[ke], sb[k - 1], sb[kRowF + k]);
-                }
-            }
-            consumer_bar();
-            const bool need2 = t >= 4;  // sweep-2 rows: sequence 2 .. nr+1
-            if (need2) {  // uniform: every lane joins the shuffles
-                // sweep-1 rows t-3, t-2, t-1 (clamped to the grid: the row outside the grid
-                // mirrors row2 = row1 - dir itself)
-                const int row2 = row1 - (int)dir;
-                const float* m0 = s1 + ((t - 2) & (kS1 - 1)) * kRowF;
-                const int rn = row2 - (int)dir, rs = row1;
-                const float* mn = (rn < 0 || rn >= H) ? m0 : s1 + ((t - 3) & (kS1 - 1)) * kRowF;
-                const float* ms = (rs < 0 || rs >= H) ? m0 : s1 + ((t - 1) & (kS1 - 1)) * kRowF;
-                const float4 c = *reinterpret_cast<const float4*>(m0 + cx);
-                const float4 a = *reinterpret_cast<const float4*>(mn + cx);
-                const float4 b = *reinterpret_cast<const float4*>(ms + cx);
-                const float4 p = *reinterpret_cast<const float4*>(sa + kRowF + cx);  // power of row2 (seq t-2)
-                float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
-                float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
-                if (lane == 0) wv = m0[cw];
-                if (lane == 31 || j0 + 4 >= W) ev = m0[ce];
-                if (j0 == 0) wv = c.x;
-                float4 o;
-                o.x = hs(c.x, a.x, b.x, c.y, wv, p.x);
-                o.y = hs(c.y, a.y, b.y, c.z, c.x, p.y);
-                o.z = hs(c.z, a.z, b.z, c.w, c.y, p.z);
-                o.w = hs(c.w, a.w, b.w, ev, c.z, p.w);
+                o.x = hs(s1B.x, n4.x, s4.x, s1B.y, w2, pA.x);
+                o.y = hs(s1B.y, n4.y, s4.y, s1B.z, s1B.x, pA.y);
+                o.z = hs(s1B.z, n4.z, s4.z, s1B.w, s1B.y, pA.z);
+                o.w = hs(s1B.w, n4.w, s4.w, e2, s1B.z, pA.w);
                 if (active) *reinterpret_cast<float4*>(outp) = o;
                 outp += dW;
             }
+            // ---- rotate the register windows; stage seq t-2 is no longer read by this warp
+            inA = inB; inB = inC; xA = xB; xB = xC;
+            s1A = s1B; s1B = s1C; eB = eC; pA = pB;
             __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&empty[(gq - 2) & (kNS - 1)]);  // seq t-2 fully used
+            if (lane == 0) ptx::mbar_arrive(&empty[(gq - 2) & (kNS - 1)]);
         }
         __syncwarp();
         if (lane == 0) {
-            ptx::mbar_arrive(&empty[(g + nr + 2) % kNS]);
-            ptx::mbar_arrive(&empty[(g + nr + 3) % kNS]);
+            ptx::mbar_arrive(&empty[(g + nr + 2) & (kNS - 1)]);
+            ptx::mbar_arrive(&empty[(g + nr + 3) & (kNS - 1)]);
         }
         g += (uint32_t)nr + 4;
-        consumer_bar();  // the sweep-1 ring is reused by the next tile
     }
 }
 
