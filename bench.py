@@ -183,9 +183,10 @@ class Workload:
         tile = getattr(self, "tile", 0)
         if self.name == "hotspot2d":
             self.pr = K.hotspot2d_setup(ctx, *self.host, ty=tile or K.HOTSPOT_TY,
-                                        kernel=getattr(self, "variant", None) or "hotspot2d_tb2",
-                                        tiles=self.tiles)
-            # sweeps fused per launch: 2 for hotspot2d_tb2 (one HBM pass = 12 B per cell per launch)
+                                        kernel=getattr(self, "variant", None) or "hotspot2d_tbk",
+                                        tiles=self.tiles, sweeps=getattr(self, "sweeps_arg", 4))
+            # sweeps fused per launch: 4 for the default hotspot2d_tbk, 2 for hotspot2d_tb2
+            # (one HBM pass = 12 B per cell per launch)
             self.sweeps = self.pr.sweeps
             self.bytes_per_unit = 12 / self.sweeps
             self.upload_bufs = [(self.pr.tb[0], self.host[0]), (self.pr.tb[2], self.host[1])]
@@ -356,6 +357,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
+    ap.add_argument("--sweeps", type=int, default=4, help="time steps per launch of --variant hotspot2d_tbk (2..4)")
     ap.add_argument("--tile", type=int, default=0, help="rows per block (hotspot2d TY) / planes per block (heat3d ZC)")
     ap.add_argument("--tiles", default=None,
                     help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")
@@ -374,6 +376,7 @@ def main():
         dist.init_process_group("gloo")
     w = Workload(args.workload, args.iters or WORKLOADS[args.workload][1])
     w.variant = args.variant
+    w.sweeps_arg = args.sweeps
     w.tile = args.tile
     w.tiles = None
     if args.tiles:
@@ -461,7 +464,7 @@ def main():
     units = w.units_per_iter * w.iters * args.steps
     value = units / (elapsed_ms / 1e3) / w.scale
     peaks = load_peaks()
-    kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tb2"}.get(w.name, w.name)
+    kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk"}.get(w.name, w.name)
     avg_kernel_ms = st["kernel_ms"] / max(1, st["timed_kernels"])
     per_launch_units = w.units_per_iter * getattr(w, "sweeps", 1) / P
     if w.name == "sgemm":
@@ -499,7 +502,7 @@ def main():
                    "l2": "inputs larger than the 126 MB L2 (no flush)" if w.name != "jacobi2d"
                    else "1 MB working set stays in L2 (latency-bound C1)",
                    "process_model": process_model,
-                   "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tb2"}.get(w.name, w.name),
+                   "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk"}.get(w.name, w.name),
                    "sweeps_per_launch": getattr(w, "sweeps", 1),
                    "partition_shape": list(w.tiles) if w.tiles else "1-D slabs of the slowest grid dim"},
         "gpu_launches": int(st["kernel_launches"] + st["copy_kernels"]),

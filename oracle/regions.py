@@ -96,6 +96,23 @@ def hotspot2d_tb2(box, block, h, w, ty, vec=4):
     return {(0, READ): _uniq(rt), (1, READ): _uniq(rp), (2, WRITE): _uniq([_ravel(I, J, (h, w))])}
 
 
+def hotspot2d_tbk(box, block, h, w, ty, k, cols=480):
+    """K fused sweeps per launch (hotspot2d_tbk): logical block (bx, by) owns rows
+    [by*ty, +ty) x columns [cols*bx, +cols); every owned cell reads the clamped
+    (2K+1)^2 square of temp_in and the clamped (2K-1)^2 square of power around it
+    (sweep s at distance <= K-s from the output needs power), writes temp_out."""
+    _, bys, bxs = _block_ranges(box)
+    i = (bys[:, None] * ty + np.arange(ty)[None, :]).ravel()
+    j = (bxs[:, None] * cols + np.arange(cols)[None, :]).ravel()
+    i = i[i < h]
+    j = j[j < w]
+    I, J = np.meshgrid(i, j, indexing="ij")
+    rt = [_ravel(_clamp(I + di, h), _clamp(J + dj, w), (h, w)) for di in range(-k, k + 1) for dj in range(-k, k + 1)]
+    rp = [_ravel(_clamp(I + di, h), _clamp(J + dj, w), (h, w))
+          for di in range(-k + 1, k) for dj in range(-k + 1, k)]
+    return {(0, READ): _uniq(rt), (1, READ): _uniq(rp), (2, WRITE): _uniq([_ravel(I, J, (h, w))])}
+
+
 # ---------------------------------------------------------------------------
 # C3 heat3d(u_in, u_out; D, H, W, ZC): block (bdx, bdy); thread owns VEC=4
 #   columns j = bx*4*bdx + 4*tx + v, row i = by*bdy + ty, and marches ZC planes

@@ -48,7 +48,7 @@ def _compile(src, verbose):
         cmd = ["g++", "-std=c++17", "-O2", "-fPIC", "-Wall", "-c", src, "-o", out] + inc
     else:
         cmd = [NVCC, "-std=c++17", "-O3", "-lineinfo", *ARCH, "-Xcompiler", "-fPIC",
-               "--expt-relaxed-constexpr", "-c", src, "-o", out] + inc
+               "--expt-relaxed-constexpr", "-c", src, "-o", out] + inc + os.environ.get("PK_NVCC_FLAGS", "").split()
         if verbose:
             cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)

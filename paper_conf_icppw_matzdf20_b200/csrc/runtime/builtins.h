@@ -42,6 +42,7 @@ extern const Builtin kBuiltinJacobi2d;
 extern const Builtin kBuiltinHotspot2d;     // hotspot2d_regs (register window)
 extern const Builtin kBuiltinHotspot2dTma;  // hotspot2d (TMA bulk ring, default)
 extern const Builtin kBuiltinHotspot2dTb2;  // hotspot2d_tb2 (two sweeps per launch)
+extern const Builtin kBuiltinHotspot2dTbk;  // hotspot2d_tbk (K = 2..4 sweeps per launch, scalar 3)
 extern const Builtin kBuiltinHeat3d;
 extern const Builtin kBuiltinHeat3dTma;      // heat3d (TMA plane ring, default); kBuiltinHeat3d = heat3d_regs
 extern const Builtin kBuiltinNbody;

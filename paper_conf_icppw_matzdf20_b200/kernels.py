@@ -32,6 +32,14 @@ def hotspot2d_launch(h, w, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX):
     return (_cdiv(w, 4 * bdx), _cdiv(h, ty), 1), (bdx, 1, 1), [h, w, ty]
 
 
+TBK_COLS = 480                         # "hotspot2d_tbk": owned columns per logical block
+
+
+def hotspot2d_tbk_launch(h, w, ty=HOTSPOT_TY, k=4):
+    """Logical block = 480 columns x ty rows, k sweeps per launch (scalar 3)."""
+    return (_cdiv(w, TBK_COLS), _cdiv(h, ty), 1), (128, 1, 1), [h, w, ty, k]
+
+
 def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
     return (_cdiv(w, 128), _cdiv(h, bdy), _cdiv(d, zc)), (32, bdy, 1), [d, h, w, zc]
 
@@ -100,27 +108,32 @@ def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None):
 
 
 def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None,
-                    kernel="hotspot2d", tiles=None):
+                    kernel="hotspot2d", tiles=None, sweeps=4):
+    """kernel: hotspot2d (one sweep per launch), hotspot2d_regs, hotspot2d_tb2 (two),
+    hotspot2d_tbk (`sweeps` = 2..4 per launch)."""
     h, w = temp_host.shape
     pr = Problem(ctx, kernel, tiles)
     t0 = pr.buffer((h, w), 4, host=temp_host, dev_ptrs=dev_ptrs[0] if dev_ptrs else None)
     t1 = pr.buffer((h, w), 4, dev_ptrs=dev_ptrs[1] if dev_ptrs else None)   # undefined (reading Q3)
     pw = pr.buffer((h, w), 4, host=power_host, dev_ptrs=dev_ptrs[2] if dev_ptrs else None)
-    pr.geom = hotspot2d_launch(h, w, ty, bdx)
+    if kernel == "hotspot2d_tbk":
+        pr.geom = hotspot2d_tbk_launch(h, w, ty, sweeps)
+    else:
+        pr.geom = hotspot2d_launch(h, w, ty, bdx)
     pr.hw = (h, w)
     pr.tb = (t0, t1, pw)
-    pr.sweeps = 2 if kernel == "hotspot2d_tb2" else 1   # time steps per launch
+    pr.sweeps = {"hotspot2d_tb2": 2, "hotspot2d_tbk": sweeps}.get(kernel, 1)   # time steps per launch
     return pr
 
 
 def hotspot2d_iterate(pr, iters, start=0):
-    """`iters` Hotspot time steps starting at step `start` (the tb2 kernel advances two
-    steps per launch: iters and start must then be even)."""
+    """`iters` Hotspot time steps starting at step `start` (the tb2/tbk kernels advance
+    pr.sweeps steps per launch: iters and start must then be multiples of it)."""
     (t0, t1, pw), (h, w) = pr.tb, pr.hw
     grid, blk, sc = pr.geom
     k = pr.sweeps
     if iters % k or start % k:
-        raise ValueError("hotspot2d_tb2 advances two steps per launch")
+        raise ValueError(f"this kernel advances {k} steps per launch")
     for t in range(start // k, (start + iters) // k):
         a, b = (t0, t1) if t % 2 == 0 else (t1, t0)
         pr.launch(grid, blk, [a, pw, b, h, w, sc[2]], sc)

@@ -73,23 +73,24 @@ def main():
     # --- hotspot2d (one sweep, TMA ring) and hotspot2d_tb2 (two sweeps per launch)
     h, w, iters = 300, 2048, 10
     t, p = synth.hotspot_grids(h, w)
-    for kern, ty in (("hotspot2d", 32), ("hotspot2d_tb2", 32)):
+    for kern, ty in (("hotspot2d", 32), ("hotspot2d_tb2", 32), ("hotspot2d_tbk", 32)):
         for mode in (0, abi.PK_MODE_GLOBAL_BARRIER):
+            its = 8 if kern == "hotspot2d_tbk" else iters      # K = 4 sweeps per launch
             ctx = new_ctx(mode)
             pr = K.hotspot2d_setup(ctx, t, p, ty=ty, kernel=kern)
-            ob = K.hotspot2d_iterate(pr, iters)
+            ob = K.hotspot2d_iterate(pr, its)
             g = gather(ctx, ob, (h, w))
             s = summed(ctx)
             abi.pk_finalize(ctx)
             if rank == 0:
                 def f1(c):
                     q = K.hotspot2d_setup(c, t, p, ty=ty, kernel=kern)
-                    o = K.hotspot2d_iterate(q, iters)
+                    o = K.hotspot2d_iterate(q, its)
                     r = np.empty((h, w), np.float32)
                     abi.pk_sync_to_host(c, o, r)
                     return r
                 ref = one_way(f1)
-                launches = iters // pr.sweeps
+                launches = its // pr.sweeps
                 # halo rows per cut and launch: 1 row per sweep of temp (+1 power row for tb2, once)
                 ok = np.array_equal(g, ref) and s["stale"] == s["moved"] and s["launches"] == launches * world
                 record(f"{kern}/mode{mode}", ok, bitwise=bool(np.array_equal(g, ref)), **s)

@@ -122,6 +122,43 @@ def test_hotspot_tb2_oracle_and_bitwise(h, w, ty):
         assert st["moved_bytes"] == st["stale_bytes"]
 
 
+@pytest.mark.parametrize("h,w,ty,k", [(200, 520, 16, 4), (129, 1028, 64, 3), (3, 4, 64, 2), (300, 2048, 7, 4),
+                                      (64, 1536, 128, 4), (40, 960, 5, 2), (257, 964, 32, 3)])
+def test_hotspot_tbk_oracle_and_bitwise(h, w, ty, k):
+    """K fused sweeps per launch (NEXT-3, K = 2..4): oracle within 1e-5, P-way bit-identical."""
+    t, p = synth.hotspot_grids(h, w)
+    iters = 12
+    ref = ok.hotspot2d(t, p, iters)
+    g1, s1 = _hotspot_k(t, p, iters, 1, ty, k)
+    ok_, err = rel_ok(g1, ref, 1e-5)
+    assert ok_, err
+    assert s1["kernel_launches"] == iters // k
+    for P in (2, 3, 4, 8):
+        gp, st = _hotspot_k(t, p, iters, P, ty, k)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def _hotspot_k(t, p, iters, P, ty, k):
+    ctx = gpu_ctx(P)
+    pr = K.hotspot2d_setup(ctx, t, p, ty=ty, kernel="hotspot2d_tbk", sweeps=k)
+    out = K.hotspot2d_iterate(pr, iters)
+    res = fetch(ctx, out, t.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st
+
+
+def test_hotspot_tbk_long_run_tolerance():
+    """100 time steps (the C2 step) in 25 four-sweep launches stay within 1e-5 of the oracle."""
+    h, w = 256, 1920
+    t, p = synth.hotspot_grids(h, w)
+    ref = ok.hotspot2d(t, p, 100)
+    g, _ = _hotspot_k(t, p, 100, 2, 32, 4)
+    ok_, err = rel_ok(g, ref, 1e-5)
+    assert ok_, err
+
+
 def test_hotspot_uniform_closed_form_on_gpu():
     h, w = 96, 256
     t = np.full((h, w), 323.0, np.float32)

@@ -542,6 +542,22 @@ def test_hotspot_tb2_regions(h, w, ty, P):
     abi.pk_finalize(ctx)
 
 
+@pytest.mark.parametrize("h,w,ty,k", [(33, 1100, 4, 4), (200, 1028, 16, 3), (5, 8, 64, 2), (40, 960, 7, 4)])
+@pytest.mark.parametrize("P", [1, 2, 3, 7])
+def test_hotspot_tbk_regions(h, w, ty, k, P):
+    """K-sweep Hotspot: one dilated tap per argument == brute-force (2K+1)^2 / (2K-1)^2 squares."""
+    ctx = host_ctx(P)
+    kk = abi.pk_builtin_kernel(ctx, "hotspot2d_tbk")
+    bufs = [abi.pk_register_buffer(ctx, (h, w), 4) for _ in range(3)]
+    grid, blk, sc = K.hotspot2d_tbk_launch(h, w, ty, k)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, kk, grid, p)
+        lib = _lib_sets(ctx, kk, 6, bufs + [None] * 3, box, blk, sc)
+        ora = _oracle_sets(regions.hotspot2d_tbk(box, blk, h, w, ty, k), {0: 4, 1: 4, 2: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
 @pytest.mark.parametrize("P", [2, 4])
 def test_hotspot_tb2_sequence(P):
     h, w = 64, 1024
