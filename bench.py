@@ -363,6 +363,8 @@ def main():
                     help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
                     help="SPMD (torchrun, N > 1) cross-rank transport: CUDA IPC peer memory or NCCL send/recv")
+    ap.add_argument("--push", action="store_true",
+                    help="PK_MODE_PUSH: halo rows stored into the neighbours' instances by the producing kernel")
     ap.add_argument("--abg", action="store_true",
                     help="also run the paper's alpha/beta/gamma overhead decomposition (P:L1164-1181)")
     args = ap.parse_args()
@@ -425,6 +427,8 @@ def main():
         ctx = abi.pk_init(P, part_device=[p % ngpu for p in range(P)])
         devices = sorted(set(p % ngpu for p in range(P)))
         process_model = "one host process drives all partitions"
+    base_mode = abi.PK_MODE_PUSH if args.push else 0
+    abi.pk_set_mode(ctx, base_mode)
     w.setup(ctx)
     for _ in range(args.warmup):
         w.step()
@@ -445,21 +449,23 @@ def main():
     st = abi.pk_get_stats(ctx)
     # (2) per-kernel CUDA events for the roofline (events around every partition kernel)
     abi.pk_reset_stats(ctx)
-    abi.pk_set_mode(ctx, abi.PK_MODE_TIME_KERNELS)
+    abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
     for _ in range(max(1, min(args.steps, 3))):
         w.step()
     abi.pk_synchronize(ctx)
     stk = abi.pk_get_stats(ctx)
-    abi.pk_set_mode(ctx, 0)
+    abi.pk_set_mode(ctx, base_mode)
     clocks = sampler.stop() if sampler else {}
     st["kernel_ms"], st["timed_kernels"] = stk["kernel_ms"], stk["timed_kernels"]
     if dist:
-        tt = torch.tensor([elapsed_ms, st["kernel_launches"], st["moved_bytes"], st["copies"]], dtype=torch.float64)
+        tt = torch.tensor([elapsed_ms, st["kernel_launches"], st["moved_bytes"], st["copies"], st["pushed_bytes"]],
+                          dtype=torch.float64)
         mx = tt.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
         dist.all_reduce(tt, op=dist.ReduceOp.SUM)
         elapsed_ms = float(mx[0])                 # max over ranks
         st["kernel_launches"], st["moved_bytes"], st["copies"] = int(tt[1]), int(tt[2]), int(tt[3])
+        st["pushed_bytes"] = int(tt[4])
 
     units = w.units_per_iter * w.iters * args.steps
     value = units / (elapsed_ms / 1e3) / w.scale
@@ -502,6 +508,7 @@ def main():
                    "l2": "inputs larger than the 126 MB L2 (no flush)" if w.name != "jacobi2d"
                    else "1 MB working set stays in L2 (latency-bound C1)",
                    "process_model": process_model,
+                   "halo_push": bool(args.push),
                    "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk"}.get(w.name, w.name),
                    "sweeps_per_launch": getattr(w, "sweeps", 1),
                    "partition_shape": list(w.tiles) if w.tiles else "1-D slabs of the slowest grid dim"},
@@ -513,6 +520,7 @@ def main():
         "transfers": {"stale_bytes": int(st["stale_bytes"]), "moved_bytes": int(st["moved_bytes"]),
                       "analytic_min_bytes": w.stale_min(P) * args.steps if not w.tiles else None,
                       "copies": int(st["copies"]), "strided_copies": int(st["strided_copies"]),
+                      "pushed_bytes": int(st["pushed_bytes"]),
                       "halo_copy_kernels": int(st["copy_kernels"])},
         "host_us_per_launch": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"]
                                + st["host_ns_issue"] + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
@@ -525,7 +533,7 @@ def main():
     if args.abg:
         times = {}
         for name, mode in (("alpha", 0), ("beta", abi.PK_MODE_NO_TRANSFERS), ("gamma", abi.PK_MODE_NO_TRACKING)):
-            abi.pk_set_mode(ctx, mode)
+            abi.pk_set_mode(ctx, mode | (base_mode if mode == 0 else 0))
             w.step()                                   # settle the mode (tracker state, caches)
             abi.pk_synchronize(ctx)
             if dist:
@@ -540,7 +548,7 @@ def main():
                 dist.all_reduce(te, op=dist.ReduceOp.MAX)
                 el = float(te[0])
             times[name] = el
-        abi.pk_set_mode(ctx, 0)
+        abi.pk_set_mode(ctx, base_mode)
         a, b, g = times["alpha"], times["beta"], times["gamma"]
         result["overhead"] = {"alpha_s": a, "beta_s": b, "gamma_s": g, "T_application": g / a,
                               "T_transfers": (a - b) / a, "T_patterns": (b - g) / a,

@@ -327,6 +327,7 @@ typedef struct {
     uint64_t graph_captures;     /* launches captured into a replay graph */
     uint64_t strided_copies;     /* of `copies`: equal pieces at a constant pitch (2-D / 3-D) */
     uint64_t copy_kernels;       /* of `strided_copies`: narrow runs moved by the SM halo-copy kernel */
+    uint64_t pushed_bytes;       /* bytes stored into other partitions' instances by producing kernels (PK_MODE_PUSH) */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);
@@ -338,8 +339,23 @@ enum {
     PK_MODE_NO_TRACKING = 1u << 2,   /* gamma of §9.2: no resolution, no tracker, no copies */
     PK_MODE_GLOBAL_BARRIER = 1u << 3,/* literal all_devs_synchronize() between sync and launch (Fig. 4 l. 8) */
     PK_MODE_TIME_KERNELS = 1u << 4,  /* CUDA events around every partition kernel -> pk_stats.kernel_ms */
-    PK_MODE_NO_GRAPHS = 1u << 5      /* disable steady-state graph replay (see pk_launch_partitioned) */
+    PK_MODE_NO_GRAPHS = 1u << 5,     /* disable steady-state graph replay (see pk_launch_partitioned) */
+    PK_MODE_PUSH = 1u << 6           /* fused halo push, see below */
 };
+/* PK_MODE_PUSH -- the transfer fused into the producing kernel (B200 design; the paper
+ * only pulls).  For a kernel whose builtin can push its output (jacobi2d,
+ * hotspot2d, hotspot2d_tbk, heat3d), the library predicts that the next reader of the
+ * written buffer reads what its last reader read: the bytes partition q writes that
+ * partition p read last time (W_q n R_p, at most 4 ranges per writer, 4-byte aligned)
+ * are stored by q's kernel ALSO into p's instance (peer stores over NVLink/NVSwitch, or
+ * an IPC mapping in peer-memory SPMD), and the tracker marks p as a holder, so the next
+ * launch finds nothing stale and issues no copy.  A wrong prediction only costs bytes:
+ * whatever is still stale is pulled as usual.  Ordering: q's kernel first waits for p's
+ * previous kernel and the copies that read (b,p) (WAR); p's kernel and copies out of
+ * (b,p) wait for q's kernel (RAW).  Not applied when the buffer is also read by the
+ * same launch, in PK_MODE_SINGLE_OWNER (no shared copies), with NO_TRANSFERS/NO_TRACKING,
+ * or in NCCL SPMD contexts.  pk_stats.pushed_bytes counts what was pushed; stale_bytes
+ * keeps counting what a launch still finds stale. */
 /* Steady-state replay: when a launch repeats with the same kernel, bindings, geometry,
  * scalars, mode and pre-launch tracker states of its buffers (e.g. the second sweep of
  * a ping-pong pair), the library captures its copies + partition kernels once into a

@@ -21,6 +21,11 @@ Readings:
       the masks as they were BEFORE this launch's synchronisation.
   Q6  a "may" write is synchronised as a read and owned as a write.
   P:L568-577  two partitions writing the same element is a WAW hazard -> error.
+  Q25 halo push (PK_MODE_PUSH, not in the paper, which only pulls): after the update,
+      for a push-capable output buffer that this launch does not read, the elements
+      writer q wrote that partition p read in the last launch that read the buffer
+      become valid on p as well -- unless q's pushes would need more than 4 contiguous
+      byte runs in total (then q pushes nothing; those bytes are pulled later).
 """
 from __future__ import annotations
 
@@ -82,12 +87,23 @@ def choose_source(mask: int, p: int, nparts: int) -> int:
     return best[1]
 
 
+MAX_PUSH_RUNS = 4
+
+
+def _runs(el):
+    """Number of contiguous runs in a sorted element index array."""
+    el = np.asarray(el)
+    return 0 if el.size == 0 else int(np.count_nonzero(np.diff(el) != 1)) + 1
+
+
 class Shadow:
     def __init__(self, nparts: int, single_owner: bool = False):
         self.P = nparts
         self.single_owner = single_owner
         self.buffers = {}
         self.stale_bytes = 0
+        self.pushed_bytes = 0
+        self.last_read = {}   # name -> [elements p read in the last launch that read it] (Q25)
         self.pair_bytes = np.zeros((nparts, nparts), dtype=np.int64)
 
     def register(self, name, nelem, elem_bytes, uploaded: bool):
@@ -97,8 +113,9 @@ class Shadow:
         self.buffers[name] = b
         return b
 
-    def launch(self, per_part):
-        """per_part[p] = {buffer_name: (read_elems, write_elems)} (None for empty partitions).
+    def launch(self, per_part, push=()):
+        """per_part[p] = {buffer_name: (read_elems, write_elems)} (None for empty partitions);
+        push = names of the buffers the kernel may halo-push (Q25; empty: the paper's pull only).
 
         Returns {"stale": [bytes per p], "copies": {(name, src, dst): sorted elems}}.
         """
@@ -153,5 +170,35 @@ class Shadow:
             for name, (_r, w) in per_part[p].items():
                 if w is not None and len(w):
                     self.buffers[name].mask[w] = np.uint64(1 << p)
+        # Q25: halo push of written buffers that this launch does not read
+        if not self.single_owner:
+            for name in push:
+                if any(per_part[p] is not None and name in per_part[p] and per_part[p][name][0] is not None
+                       and len(per_part[p][name][0]) for p in range(P)):
+                    continue
+                last = self.last_read.get(name)
+                if last is None:
+                    continue
+                for q in range(P):
+                    if per_part[q] is None or name not in per_part[q]:
+                        continue
+                    w = per_part[q][name][1]
+                    if w is None or not len(w):
+                        continue
+                    xs = {p: np.intersect1d(w, last[p]) for p in range(P)
+                          if p != q and last[p] is not None and len(last[p])}
+                    xs = {p: x for p, x in xs.items() if x.size}
+                    if not xs or sum(_runs(x) for x in xs.values()) > MAX_PUSH_RUNS:
+                        continue
+                    for p, x in xs.items():
+                        self.buffers[name].mask[x] |= np.uint64(1 << p)
+                        self.pushed_bytes += int(x.size) * self.buffers[name].eb
+        # read sets of this launch: the prediction for the next writer (Q25)
+        for p in range(P):
+            if per_part[p] is None:
+                continue
+            for name, (r, _w) in per_part[p].items():
+                if r is not None and len(r):
+                    self.last_read.setdefault(name, [None] * P)[p] = np.asarray(r)
         self.stale_bytes += sum(stale)
         return {"stale": stale, "copies": copies}

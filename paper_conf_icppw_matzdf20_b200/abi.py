@@ -27,6 +27,7 @@ PK_MODE_NO_TRACKING = 1 << 2
 PK_MODE_GLOBAL_BARRIER = 1 << 3
 PK_MODE_TIME_KERNELS = 1 << 4
 PK_MODE_NO_GRAPHS = 1 << 5
+PK_MODE_PUSH = 1 << 6
 
 
 class PkError(RuntimeError):
@@ -71,7 +72,7 @@ class pk_stats(C.Structure):
                 ("host_ns_update", C.c_uint64), ("kernel_ms", C.c_double),
                 ("kernel_ms_max_launch", C.c_double), ("timed_kernels", C.c_uint64),
                 ("graph_replays", C.c_uint64), ("graph_captures", C.c_uint64),
-                ("strided_copies", C.c_uint64), ("copy_kernels", C.c_uint64)]
+                ("strided_copies", C.c_uint64), ("copy_kernels", C.c_uint64), ("pushed_bytes", C.c_uint64)]
 
 
 RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)

@@ -60,6 +60,7 @@ Status tap_ranges(const pk_affine_access& tap, const int64_t box6[6], int ndim,
 void canonicalize(RangeList* r);
 // Union of canonical lists.
 RangeList union_ranges(const RangeList& a, const RangeList& b);
+RangeList intersect_ranges(const RangeList& a, const RangeList& b);  // a, b canonical
 uint64_t total_bytes(const RangeList& r);
 
 // ---------------------------------------------------------------- tracker

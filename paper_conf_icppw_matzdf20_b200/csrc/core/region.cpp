@@ -202,6 +202,19 @@ RangeList union_ranges(const RangeList& a, const RangeList& b) {
     return r;
 }
 
+RangeList intersect_ranges(const RangeList& a, const RangeList& b) {
+    // both canonical (sorted, disjoint): linear merge
+    RangeList r;
+    size_t i = 0, j = 0;
+    while (i < a.size() && j < b.size()) {
+        const uint64_t lo = std::max(a[i].b, b[j].b), hi = std::min(a[i].e, b[j].e);
+        if (lo < hi) r.push_back(Range{lo, hi});
+        if (a[i].e < b[j].e) ++i;
+        else ++j;
+    }
+    return r;
+}
+
 uint64_t total_bytes(const RangeList& r) {
     uint64_t t = 0;
     for (const Range& x : r) t += x.e - x.b;

@@ -37,3 +37,21 @@ __device__ __forceinline__ void st4(float* p, float4 v) {
 
 }  // namespace dev
 }  // namespace pk
+
+#include "../runtime/builtins.h"
+
+namespace pk {
+namespace dev {
+// Halo push (PK_MODE_PUSH): the value just stored at byte offset `off` of the output
+// instance also goes to every destination instance whose push range covers it
+// (4-byte granularity ranges; `n` is uniform, usually 0 or 2).
+__device__ __forceinline__ void push4(const PushList& pl, uint64_t off, const float4& v) {
+    for (int i = 0; i < pl.n; ++i)
+        if (off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float4*>(pl.dst[i] + off) = v;
+}
+__device__ __forceinline__ void push1(const PushList& pl, uint64_t off, float v) {
+    for (int i = 0; i < pl.n; ++i)
+        if (off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float*>(pl.dst[i] + off) = v;
+}
+}  // namespace dev
+}  // namespace pk

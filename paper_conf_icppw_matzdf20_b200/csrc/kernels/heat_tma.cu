@@ -27,6 +27,7 @@
 #include <unordered_map>
 
 #include "../runtime/builtins.h"
+#include "common.cuh"
 #include "ptx.cuh"
 #include "tma_host.h"
 
@@ -58,7 +59,7 @@ __device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_
 
 __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUtensorMap tm_u,
                                                     float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
-                                                    int64_t ZC, int bdy, pk_partition part) {
+                                                    int64_t ZC, int bdy, pk_partition part, PushList push) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
     // bdy = logical rows per block; warps 0..nw-1 consume (kRPW rows each), warp nw produces
@@ -140,6 +141,7 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUt
             o.z = c.z + kAlpha * ((zm.z + zp.z + ym.z + yp.z + c.y + c.w) - 6.0f * c.z);
             o.w = c.w + kAlpha * ((zm.w + zp.w + ym.w + yp.w + c.z + ev) - 6.0f * c.w);
             *reinterpret_cast<float4*>(uout + kout + i * W + j0) = o;
+            if (push.n) dev::push4(push, (uint64_t)(kout + i * W + j0) * 4u, o);  // fused halo push
         }
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&empty[s_m]);  // slot z-1 no longer needed by this warp
@@ -204,7 +206,9 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
         }
     }
     int bdy_arg = bdy;
-    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part};
+    PushList pl{};
+    if (li.push) pl = *li.push;
+    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part, &pl};
     return cudaLaunchKernel((const void*)k_heat3d_tma, li.grid, dim3(32, warp_count(bdy) + 1), argv, smem_bytes(bdy),
                             li.stream);
 }
@@ -214,6 +218,6 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
 const Builtin kBuiltinHeat3dTma = {
     "heat3d", (const void*)k_heat3d_tma, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
-    describe_heat3d_tma, launch_heat3d_tma};
+    describe_heat3d_tma, launch_heat3d_tma, /*push_arg=*/1};
 
 }  // namespace pk

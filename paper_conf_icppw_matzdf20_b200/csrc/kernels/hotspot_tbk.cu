@@ -30,6 +30,7 @@
 #include <cuda_runtime.h>
 
 #include "../runtime/builtins.h"
+#include "common.cuh"
 #include "ptx.cuh"
 
 namespace pk {
@@ -90,7 +91,7 @@ __device__ __forceinline__ float4 level(const float4& c, const float4& n, const 
 template <int K, bool EDGE, bool COLEDGE>
 __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, uint64_t* empty, float* tout,
                                              int64_t W, int H, int64_t c0, int64_t r0, int64_t rend, bool down,
-                                             uint32_t g, int lane, int warp) {
+                                             uint32_t g, int lane, int warp, const PushList& push) {
     constexpr int kW3 = 3;
     const int scol = kOwn * warp + 4 * lane;
     const int64_t col0 = c0 - 4 + scol;
@@ -133,7 +134,10 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
                 if (k < K) {
                     L[k - 1][sc] = o;
                 } else if (t >= 2 * K) {
-                    if (store) *reinterpret_cast<float4*>(outp) = o;
+                    if (store) {
+                        *reinterpret_cast<float4*>(outp) = o;
+                        if (push.n) dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
+                    }
                     outp += dW;
                 }
             }
@@ -152,7 +156,7 @@ template <int K>
 __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const float* __restrict__ tin,
                                                             const float* __restrict__ pw,
                                                             float* __restrict__ tout, int64_t H, int64_t W,
-                                                            int64_t TY, pk_partition part) {
+                                                            int64_t TY, pk_partition part, PushList push) {
     extern __shared__ __align__(128) unsigned char smem[];
     float* ring = reinterpret_cast<float*>(smem);
     uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)kNS * kStageFloats);
@@ -202,9 +206,9 @@ __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const f
         const bool redge = r0 < K + 1 || rend + K + 1 > H;
         const bool cedge = c0 == 0 || c0 + kTC + 4 >= W;
         if (redge || cedge)
-            consume_tile<K, true, true>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp);
+            consume_tile<K, true, true>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp, push);
         else
-            consume_tile<K, false, false>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp);
+            consume_tile<K, false, false>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp, push);
         g += (uint32_t)(rend - r0) + 2 * K;
     }
 }
@@ -263,7 +267,9 @@ cudaError_t launch_k(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
     if (ntiles == 0) return cudaSuccess;
     const int64_t cap = (int64_t)resident[d] * sms[d];
     dim3 grid((unsigned)(ntiles < cap ? ntiles : cap));
-    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part};
+    PushList pl{};
+    if (li.push) pl = *li.push;
+    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part, &pl};
     return cudaLaunchKernel((const void*)k_hotspot2d_tbk<K>, grid, dim3(kThreads), argv, kSmem, li.stream);
 }
 
@@ -286,6 +292,6 @@ cudaError_t launch_hotspot2d_tbk(const LaunchInfo& li) {
 const Builtin kBuiltinHotspot2dTbk = {
     "hotspot2d_tbk", (const void*)k_hotspot2d_tbk<4>, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
-    describe_hotspot2d_tbk, launch_hotspot2d_tbk};
+    describe_hotspot2d_tbk, launch_hotspot2d_tbk, /*push_arg=*/2};
 
 }  // namespace pk

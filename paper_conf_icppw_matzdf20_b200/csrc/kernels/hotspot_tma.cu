@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 
 #include "../runtime/builtins.h"
+#include "common.cuh"
 #include "ptx.cuh"
 
 namespace pk {
@@ -46,7 +47,7 @@ __device__ __forceinline__ float hs(float c, float n, float s, float e, float w,
 __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restrict__ tin,
                                                             const float* __restrict__ pw,
                                                             float* __restrict__ tout, int64_t H, int64_t W,
-                                                            int64_t TY, pk_partition part) {
+                                                            int64_t TY, pk_partition part, PushList push) {
     extern __shared__ __align__(128) unsigned char smem[];
     float* ring = reinterpret_cast<float*>(smem);
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + (size_t)kNS * kStageBytes);
@@ -125,6 +126,7 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restr
                 o.w = hs(c.w, a.w, b.w, ev, c.z, p.w);
                 const int64_t row = down ? r0 - 1 + t : rend - t;
                 *reinterpret_cast<float4*>(tout + row * W + j0) = o;
+                if (push.n) dev::push4(push, (uint64_t)(row * W + j0) * 4u, o);  // fused halo push
             }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&empty[gp % kNS]);
@@ -181,7 +183,9 @@ cudaError_t launch_hotspot2d_tma(const LaunchInfo& li) {
     if (ntiles == 0) return cudaSuccess;
     const int64_t cap = (int64_t)resident[d] * sms[d];
     dim3 grid((unsigned)(ntiles < cap ? ntiles : cap));
-    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part};
+    PushList pl{};
+    if (li.push) pl = *li.push;
+    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part, &pl};
     return cudaLaunchKernel((const void*)k_hotspot2d_tma, grid, dim3(kThreads), argv, kSmem, li.stream);
 }
 
@@ -190,6 +194,6 @@ cudaError_t launch_hotspot2d_tma(const LaunchInfo& li) {
 const Builtin kBuiltinHotspot2dTma = {
     "hotspot2d", (const void*)k_hotspot2d_tma, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
-    describe_hotspot2d_tma, launch_hotspot2d_tma};
+    describe_hotspot2d_tma, launch_hotspot2d_tma, /*push_arg=*/2};
 
 }  // namespace pk

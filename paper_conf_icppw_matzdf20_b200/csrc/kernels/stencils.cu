@@ -29,13 +29,15 @@ using dev::st4;
 // One thread per cell: i = by*bdy + ty, j = bx*bdx + tx; Dirichlet interior
 //   out[i][j] = 0.25 * (((in[i-1][j] + in[i+1][j]) + in[i][j-1]) + in[i][j+1])
 __global__ void __launch_bounds__(256) k_jacobi2d(const float* __restrict__ in, float* __restrict__ out,
-                                                  int64_t H, int64_t W, pk_partition part) {
+                                                  int64_t H, int64_t W, pk_partition part, PushList push) {
     const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y;  // Eq. 8
     const int64_t i = by * blockDim.y + threadIdx.y, j = bx * blockDim.x + threadIdx.x;
     if (i < 1 || i > H - 2 || j < 1 || j > W - 2) return;
     const float n = in[(i - 1) * W + j], s = in[(i + 1) * W + j];
     const float w = in[i * W + j - 1], e = in[i * W + j + 1];
-    out[i * W + j] = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(__fadd_rn(n, s), w), e));
+    const float v = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(__fadd_rn(n, s), w), e));
+    out[i * W + j] = v;
+    if (push.n) dev::push1(push, (uint64_t)(i * W + j) * 4u, v);  // fused halo push
 }
 
 int describe_jacobi2d(pk_ctx c, pk_kernel k) {
@@ -56,7 +58,9 @@ int describe_jacobi2d(pk_ctx c, pk_kernel k) {
 cudaError_t launch_jacobi2d(const LaunchInfo& li) {
     if (li.nscalars < 2) return cudaErrorInvalidValue;
     int64_t H = li.scalars[0], W = li.scalars[1];
-    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &H, &W, (void*)&li.part};
+    PushList pl{};
+    if (li.push) pl = *li.push;
+    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &H, &W, (void*)&li.part, &pl};
     return cudaLaunchKernel(li.fn, li.grid, li.block, argv, 0, li.stream);
 }
 
@@ -284,7 +288,8 @@ cudaError_t launch_heat3d(const LaunchInfo& li) {
 
 const Builtin kBuiltinJacobi2d = {
     "jacobi2d", (const void*)k_jacobi2d, 4,
-    {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1, describe_jacobi2d, launch_jacobi2d};
+    {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1, describe_jacobi2d, launch_jacobi2d,
+    /*push_arg=*/1};
 const Builtin kBuiltinHotspot2d = {
     "hotspot2d_regs", (const void*)k_hotspot2d, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,

@@ -7,6 +7,18 @@
 
 namespace pk {
 
+// Halo push (PK_MODE_PUSH): bytes [lo[i], hi[i]) of the kernel's push-capable output
+// instance are ALSO stored at dst[i] + offset (another partition's instance of the same
+// buffer, same layout; a peer GPU's memory over NVLink or an IPC mapping) by the kernel
+// that produces them.  Passed to the kernel by value.
+constexpr int kMaxPush = 4;
+struct PushList {
+    int32_t n;
+    int32_t pad;
+    uint64_t lo[kMaxPush], hi[kMaxPush];
+    uint64_t dst[kMaxPush];
+};
+
 // Everything a launcher needs for one partition (Fig. 4 lines 10-19).
 struct LaunchInfo {
     const void* fn;
@@ -20,6 +32,7 @@ struct LaunchInfo {
     const int64_t* scalars;
     int nscalars;
     pk_partition part;
+    const PushList* push = nullptr;  // halo push of the push-capable output (nullptr / n = 0: none)
 };
 using LauncherFn = cudaError_t (*)(const LaunchInfo&);
 
@@ -32,10 +45,12 @@ struct Builtin {
     // declares the kernel's access taps through pk_declare_affine_access
     int (*describe)(pk_ctx, pk_kernel);
     LauncherFn launcher;       // nullptr = generic cudaLaunchKernel
+    int32_t push_arg = -1;     // output buffer argument the kernel can halo-push (LaunchInfo::push), -1: none
 };
 
 const Builtin* find_builtin(const char* name);
 LauncherFn find_builtin_launcher(const void* fn);
+int32_t find_builtin_push_arg(const void* fn);
 
 // Per-kernel-file registration (defined in kernels/*.cu)
 extern const Builtin kBuiltinJacobi2d;

@@ -115,6 +115,11 @@ struct Buffer {
     std::vector<uint8_t> ep_kind;      // [q]: W_KERNEL / W_COPY (which flag word signals it)
     std::vector<uint64_t> ep_read;     // [q*P + r]: epoch at which r last copied out of (b,q); 0 = none
     std::vector<void*> ipc_base;       // [q]: mapped base of a remote instance (cudaIpcCloseMemHandle)
+    // halo push (PK_MODE_PUSH)
+    std::vector<RangeList> last_read;  // [p]: bytes p read in the last launch that read this buffer (prediction)
+    std::vector<uint64_t> pushers;     // [p]: partitions whose kernels pushed into (b,p) (event RAW, 1 process)
+    std::vector<uint64_t> ep_push;     // [p*P+q]: epoch of q's last push into (b,p) (peer-memory SPMD)
+    std::vector<uint64_t> ep_kread;    // [p]: epoch of p's last kernel that read b (peer-memory SPMD, push WAR)
 };
 
 struct Tap {
@@ -132,6 +137,7 @@ struct Kernel {
     int32_t tiles[3] = {0, 0, 0};  // (tx, ty, tz) tile partition; 0 = 1-D split
     std::vector<Tap> taps;
     LauncherFn launcher = nullptr;
+    int32_t push_arg = -1;  // output buffer argument the kernel can halo-push (builtin capability)
     uint64_t version = 0;  // bumps when taps change (region cache key)
 };
 
@@ -168,6 +174,7 @@ struct pk_ctx_s {
     std::vector<int> sm_count;  // per partition's device (halo copy kernel grid)
     std::vector<cudaStream_t> stream;
     std::vector<cudaEvent_t> ev_kernel, ev_copy;
+    std::vector<uint8_t> kernel_recorded;  // [p]: ev_kernel[p] recorded since the hazards were last cleared
     std::vector<Buffer> bufs;
     std::vector<Kernel> kernels;
     pk_stats stats{};
@@ -192,6 +199,7 @@ struct pk_ctx_s {
     std::vector<void*> flag_mapped;      // [p]: mapped bases to close
     uint64_t epoch = 0;                  // replicated launch epoch (flags are compared GEQ)
     bool flags_on_sm = false;            // epoch flags by SM kernels instead of stream memory operations
+    std::vector<uint8_t> flag_on_peer_gpu;  // [p]: p's flag words live on another physical GPU
     std::unordered_map<std::string, std::pair<void*, int>> ipc_maps;  // handle -> (mapped base, refs)
     // steady-state graph replay (pk_api.h, PK_MODE_NO_GRAPHS)
     struct Memo {
@@ -287,6 +295,8 @@ void ipc_settle(pk_ctx c) {
         if (B.alive) {
             std::fill(B.ep_mod.begin(), B.ep_mod.end(), 0ull);
             std::fill(B.ep_read.begin(), B.ep_read.end(), 0ull);
+            std::fill(B.ep_push.begin(), B.ep_push.end(), 0ull);
+            std::fill(B.ep_kread.begin(), B.ep_kread.end(), 0ull);
         }
 }
 
@@ -318,9 +328,13 @@ void ipc_close(pk_ctx c, void* base) {
 }
 
 // Per-stream wait list: the max epoch needed from each partition's two flag words.
-// Issued as stream memory operations (cuStreamWaitValue64, processed by the stream
-// front end, no SM); if the driver refuses them for a mapped peer address the
-// context switches to the SM spin-wait kernels for good (PK_FLAGS_SM env forces it).
+// Flags in this GPU's memory (ranks sharing the device) are waited for with stream
+// memory operations (cuStreamWaitValue64, processed by the stream front end, no SM).
+// Flags on another GPU are polled by the 1-thread SM kernel with system-scope
+// acquire loads over NVLink (peer loads are the documented path; PK_FLAGS_MEMOP_PEER
+// opts into stream memory operations on peer addresses instead).  If the driver
+// refuses a memory operation the context switches to the SM kernels for good
+// (PK_FLAGS_SM forces them everywhere).
 struct FlagWaits {
     std::vector<uint64_t> need;  // [q*2 + word]
     explicit FlagWaits(int P) : need(2 * P, 0) {}
@@ -331,7 +345,7 @@ struct FlagWaits {
         for (size_t i = 0; i < need.size(); ++i)
             if (need[i]) {
                 const uint64_t* f = c->flag[i / 2] + (i % 2);
-                if (!c->flags_on_sm) {
+                if (!c->flags_on_sm && !c->flag_on_peer_gpu[i / 2]) {
                     CUresult e = drv().ok ? drv().WaitValue64((CUstream)s, (CUdeviceptr)f, need[i],
                                                               CU_STREAM_WAIT_VALUE_GEQ)
                                           : CUDA_ERROR_NOT_SUPPORTED;
@@ -564,6 +578,7 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
         c->ev_copy.resize(c->P);
         c->event_pool.resize(c->P);
         c->ev_join.assign(c->P, nullptr);
+        c->kernel_recorded.assign(c->P, 0);
         c->sm_count.assign(c->P, 148);
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
@@ -580,6 +595,15 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
         c->cur_device = c->dev[c->first_local];
         if (c->ipc) {
             c->flags_on_sm = getenv("PK_FLAGS_SM") != nullptr;
+            // which ranks sit on another physical GPU (their flags are polled by SM kernels)
+            cudaDeviceProp prop;
+            PK_CUDA(cudaGetDeviceProperties(&prop, c->dev[c->first_local]));
+            std::vector<cudaUUID_t> uu(c->world);
+            if (int r = host_allgather(c.get(), &prop.uuid, uu.data(), sizeof(cudaUUID_t))) return r;
+            const bool memop_peer = getenv("PK_FLAGS_MEMOP_PEER") != nullptr;
+            c->flag_on_peer_gpu.assign(c->P, 0);
+            for (int p = 0; p < c->P; ++p)
+                c->flag_on_peer_gpu[p] = !memop_peer && std::memcmp(&uu[c->prank[p]], &prop.uuid, sizeof(cudaUUID_t)) != 0;
             // epoch flag words of this rank, mapped by every other rank
             if (int r = c->set_device(c->dev[c->first_local])) return r;
             PK_CUDA(cudaMalloc((void**)&c->flag_local, 256));
@@ -613,10 +637,12 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
 }
 
 static void clear_hazards(pk_ctx c) {
+    std::fill(c->kernel_recorded.begin(), c->kernel_recorded.end(), (uint8_t)0);
     for (Buffer& B : c->bufs)
         if (B.alive) {
             std::fill(B.last_writer.begin(), B.last_writer.end(), (uint8_t)W_NONE);
             std::fill(B.readers.begin(), B.readers.end(), 0ull);
+            std::fill(B.pushers.begin(), B.pushers.end(), 0ull);
         }
 }
 
@@ -808,6 +834,10 @@ int pk_register_buffer(pk_ctx c, int ndim, const int64_t* shape, int elem_bytes,
     B.ep_kind.assign(c->P, W_NONE);
     B.ep_read.assign((size_t)c->P * c->P, 0);
     B.ipc_base.assign(c->P, nullptr);
+    B.last_read.assign(c->P, RangeList{});
+    B.pushers.assign(c->P, 0);
+    B.ep_push.assign((size_t)c->P * c->P, 0);
+    B.ep_kread.assign(c->P, 0);
     const uint64_t all = c->P == 64 ? ~0ull : ((1ull << c->P) - 1);
     B.tracker.init(B.bytes, all);  // reading Q3: undefined contents are valid everywhere
     if (!c->host_only) {
@@ -1104,6 +1134,12 @@ int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
     if (c->host_only) return fail(PK_ERR_STATE, "host-only context holds no data");
     if (!host && (c->world == 1 || c->rank == 0)) return fail(PK_ERR_INVALID, "null host buffer");
     if (c->world > 1) return c->ipc ? sync_to_host_ipc(c, B, host) : sync_to_host_spmd(c, B, host);
+    // bytes pushed into an instance by another partition's kernel: drain everything first
+    for (uint64_t m : B.pushers)
+        if (m) {
+            if (int r = pk_synchronize(c)) return r;
+            break;
+        }
     // replay graphs run on stream[p0]: fork the other streams from its tail first
     if (int r = exit_graph_mode(c)) return r;
     // query all segments, copy each from a partition that holds it.
@@ -1137,6 +1173,7 @@ int pk_register_kernel(pk_ctx c, const char* name, const void* fn, int nargs, co
     k.name = name ? name : "";
     k.fn = fn;
     k.launcher = find_builtin_launcher(fn);  // a builtin __global__ keeps its own launch geometry
+    k.push_arg = find_builtin_push_arg(fn);
     k.nargs = nargs;
     k.partition_dim = partition_dim;
     for (int i = 0; i < nargs; ++i) {
@@ -1248,7 +1285,7 @@ int pk_reset_stats(pk_ctx c) {
 
 int pk_set_mode(pk_ctx c, uint32_t flags) {
     if (!c) return fail(PK_ERR_INVALID, "bad argument");
-    if (flags & ~0x3Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
+    if (flags & ~0x7Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
     c->mode = flags;
     return PK_OK;
 }
@@ -1266,6 +1303,7 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
     a.copy_kernels += sign * d.copy_kernels;
     a.stale_bytes += sign * d.stale_bytes;
     a.moved_bytes += sign * d.moved_bytes;
+    a.pushed_bytes += sign * d.pushed_bytes;
     for (int i = 0; i < 16; ++i)
         for (int j = 0; j < 16; ++j) a.pair_bytes[i][j] += sign * d.pair_bytes[i][j];
 }
@@ -1500,6 +1538,49 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 for (auto& bs : sets[p])
                     if (!bs.r.empty()) c->bufs[bs.b].tracker.add_bit(bs.r, p);
     }
+    // ---- halo push plan (PK_MODE_PUSH): predict that the next reader of a written buffer
+    // reads what its last reader read; the producing kernel then also stores those bytes
+    // straight into the reader's instance (fused, peer stores over NVLink), and the tracker
+    // records the reader as a holder, so the next launch finds nothing stale.
+    struct PushRec { int64_t b; int q, p; RangeList r; };
+    std::vector<PushList> push(P);
+    std::vector<PushRec> pushed;
+    const int pa = K.push_arg;
+    if ((mode & PK_MODE_PUSH) && !single_owner && transfer && pa >= 0 && pa < K.nargs && bound[pa] &&
+        (c->world == 1 || c->ipc)) {
+        const int64_t b = bid[pa];
+        bool read_here = false;  // the buffer must not also be read by this launch
+        for (int p = 0; p < P && !read_here; ++p)
+            for (auto& bs : sets[p])
+                if (bs.b == b && !bs.r.empty()) read_here = true;
+        const Buffer& B = c->bufs[b];
+        for (int q = 0; q < P && !read_here; ++q) {
+            const RangeList* Wq = nullptr;
+            for (auto& bs : sets[q])
+                if (bs.b == b) Wq = &bs.w;
+            if (!Wq || Wq->empty()) continue;
+            PushList pl{};
+            std::vector<PushRec> recs;
+            bool fits = true;
+            for (int p = 0; p < P && fits; ++p) {
+                if (p == q || B.last_read[p].empty()) continue;
+                RangeList x = intersect_ranges(*Wq, B.last_read[p]);
+                if (x.empty()) continue;
+                for (const Range& r : x) {
+                    if (pl.n == kMaxPush || (r.b | r.e) % 4) { fits = false; break; }
+                    pl.lo[pl.n] = r.b;
+                    pl.hi[pl.n] = r.e;
+                    pl.dst[pl.n] = (uint64_t)(uintptr_t)B.inst[p];
+                    pl.n++;
+                }
+                recs.push_back(PushRec{b, q, p, std::move(x)});
+            }
+            if (!fits || recs.empty()) continue;  // too fragmented: those bytes are pulled as usual
+            push[q] = pl;
+            for (auto& r : recs) pushed.push_back(std::move(r));
+        }
+    }
+
     uint64_t t3 = now_ns();
     c->stats.host_ns_plan += t3 - t2;
     c->stats.launches += 1;
@@ -1526,6 +1607,8 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                         const Buffer& B = c->bufs[o.buf];
                         if (B.ep_mod[o.src])
                             fw.add(o.src, B.ep_kind[o.src] == W_COPY ? kFlagCopied : kFlagDone, B.ep_mod[o.src]);
+                        for (int q = 0; q < P; ++q)  // bytes pushed into (b, src) by q's kernel
+                            if (B.ep_push[(size_t)o.src * P + q]) fw.add(q, kFlagDone, B.ep_push[(size_t)o.src * P + q]);
                         for (int r = 0; r < P; ++r)
                             if (B.ep_read[(size_t)p * P + r]) fw.add(r, kFlagCopied, B.ep_read[(size_t)p * P + r]);
                     }
@@ -1538,6 +1621,10 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     if (!c->local(o.src)) continue;
                     Buffer& B = c->bufs[o.buf];
                     if (B.readers[p]) if (int r = wait_readers(c, B, p)) return r;
+                    for (uint64_t m = B.pushers[o.src]; m; m &= m - 1) {  // bytes pushed into (b, src)
+                        const int q = __builtin_ctzll(m);
+                        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_kernel[q], 0));
+                    }
                     const uint8_t lw = B.last_writer[o.src];
                     uint64_t bit = 1ull << o.src;
                     if (lw != W_NONE && !(waited_src & bit)) {
@@ -1728,6 +1815,43 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         for (const Tap& t : K.taps)
             if (t.arg == a && t.mode != PK_READ) writes_arg[a] = true;
     if (!c->host_only) {
+        // Push hazards, enqueued before ANY kernel of this launch so that ev_kernel[*] still
+        // names the previous launch's kernels (no false serialisation within a launch):
+        //   RAW  p's kernel reads bytes an earlier kernel of q pushed into (b,p);
+        //   WAR  q's kernel pushes into (b,p): p's previous kernel and the copies that read
+        //        (b,p) must be done.
+        for (int p = 0; p < P; ++p) {
+            if ((*regs)[p].empty || !c->local(p)) continue;
+            if (int r = c->set_device(c->dev[p])) return r;
+            FlagWaits fw(c->ipc ? P : 0);
+            for (int a = 0; a < K.nargs; ++a) {
+                if (!bound[a]) continue;
+                const Buffer& B = c->bufs[bid[a]];
+                if (c->ipc) {
+                    for (int q = 0; q < P; ++q)
+                        if (B.ep_push[(size_t)p * P + q]) fw.add(q, kFlagDone, B.ep_push[(size_t)p * P + q]);
+                } else {
+                    for (uint64_t m = B.pushers[p]; m; m &= m - 1)
+                        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_kernel[__builtin_ctzll(m)], 0));
+                }
+            }
+            for (const PushRec& pr : pushed) {
+                if (pr.q != p) continue;
+                const Buffer& B = c->bufs[pr.b];
+                if (c->ipc) {
+                    if (B.ep_kread[pr.p]) fw.add(pr.p, kFlagDone, B.ep_kread[pr.p]);
+                    for (int r = 0; r < P; ++r)
+                        if (B.ep_read[(size_t)pr.p * P + r]) fw.add(r, kFlagCopied, B.ep_read[(size_t)pr.p * P + r]);
+                } else {
+                    if (c->kernel_recorded[pr.p])
+                        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_kernel[pr.p], 0));
+                    for (uint64_t m = B.readers[pr.p]; m; m &= m - 1)
+                        PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_copy[__builtin_ctzll(m)], 0));
+                }
+            }
+            if (c->ipc)
+                if (int r = fw.issue(c, c->stream[p])) return r;
+        }
         void* inst[PK_MAX_ARGS];
         void* argv[PK_MAX_ARGS + 1];
         for (int p = 0; p < P; ++p) {
@@ -1779,7 +1903,8 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             }
             cudaError_t err;
             if (K.launcher) {
-                LaunchInfo li{K.fn, g, bl, smem, c->stream[p], c->dev[p], inst, args, scalars, ns, part};
+                LaunchInfo li{K.fn, g, bl, smem, c->stream[p], c->dev[p], inst, args, scalars, ns, part,
+                              push[p].n ? &push[p] : nullptr};
                 err = K.launcher(li);
             } else {
                 err = cudaLaunchKernel(K.fn, g, bl, argv, smem, c->stream[p]);
@@ -1791,7 +1916,10 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 PK_CUDA(cudaEventRecord(e1, c->stream[p]));
                 c->pending_timing.push_back(TimedLaunch{e0, e1, p, launch_id});
             }
-            if (P > 1) PK_CUDA(cudaEventRecord(c->ev_kernel[p], c->stream[p]));
+            if (P > 1) {
+                PK_CUDA(cudaEventRecord(c->ev_kernel[p], c->stream[p]));
+                c->kernel_recorded[p] = 1;
+            }
             if (c->ipc)
                 if (int r = ipc_signal(c, p, kFlagDone, E)) return r;
             c->stats.kernel_launches += 1;
@@ -1828,6 +1956,23 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         for (int p = 0; p < P; ++p)
             for (auto& bs : sets[p])
                 if (!bs.w.empty()) c->bufs[bs.b].tracker.assign(bs.w, 1ull << p);
+    // pushed bytes are valid on the receiving partition too
+    for (const PushRec& pr : pushed) {
+        Buffer& B = c->bufs[pr.b];
+        B.tracker.add_bit(pr.r, pr.p);
+        B.pushers[pr.p] |= 1ull << pr.q;
+        if (c->ipc) B.ep_push[(size_t)pr.p * P + pr.q] = E;
+        if (c->local(pr.q)) c->stats.pushed_bytes += total_bytes(pr.r);
+    }
+    // read sets of this launch: the push prediction of the next writer (+ push WAR epochs)
+    if (track)
+        for (int p = 0; p < P; ++p)
+            for (auto& bs : sets[p])
+                if (!bs.r.empty()) {
+                    Buffer& B = c->bufs[bs.b];
+                    B.last_read[p] = bs.r;
+                    if (c->ipc) B.ep_kread[p] = E;
+                }
     c->stats.host_ns_update += now_ns() - t5;
     return PK_OK;
 }
@@ -1835,6 +1980,14 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
 }  // extern "C"
 
 namespace pk {
+int32_t find_builtin_push_arg(const void* fn) {
+    if (!fn) return -1;
+    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_tbk", "heat3d"}) {
+        const Builtin* b = find_builtin(n);
+        if (b && b->fn == fn) return b->push_arg;
+    }
+    return -1;
+}
 LauncherFn find_builtin_launcher(const void* fn) {
     if (!fn) return nullptr;
     for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk", "heat3d", "heat3d_regs",

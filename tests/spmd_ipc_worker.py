@@ -54,9 +54,11 @@ def main():
         st = abi.pk_get_stats(ctx)
         # stale bytes are counted by the replicated plan (identical on every rank); moved
         # bytes, copies and kernels by the rank that pulls / launches them -> summed
-        t = torch.tensor([st["moved_bytes"], st["copies"], st["kernel_launches"]], dtype=torch.float64)
+        t = torch.tensor([st["moved_bytes"], st["copies"], st["kernel_launches"], st["pushed_bytes"]],
+                         dtype=torch.float64)
         dist.all_reduce(t)
-        return {"stale": int(st["stale_bytes"]), "moved": int(t[0]), "copies": int(t[1]), "launches": int(t[2])}
+        return {"stale": int(st["stale_bytes"]), "moved": int(t[0]), "copies": int(t[1]), "launches": int(t[2]),
+                "pushed": int(t[3])}
 
     def one_way(fn):
         ctx = abi.pk_init(1, part_device=[0])
@@ -74,7 +76,7 @@ def main():
     h, w, iters = 300, 2048, 10
     t, p = synth.hotspot_grids(h, w)
     for kern, ty in (("hotspot2d", 32), ("hotspot2d_tb2", 32), ("hotspot2d_tbk", 32)):
-        for mode in (0, abi.PK_MODE_GLOBAL_BARRIER):
+        for mode in (0, abi.PK_MODE_GLOBAL_BARRIER, abi.PK_MODE_PUSH):
             its = 8 if kern == "hotspot2d_tbk" else iters      # K = 4 sweeps per launch
             ctx = new_ctx(mode)
             pr = K.hotspot2d_setup(ctx, t, p, ty=ty, kernel=kern)
@@ -93,6 +95,8 @@ def main():
                 launches = its // pr.sweeps
                 # halo rows per cut and launch: 1 row per sweep of temp (+1 power row for tb2, once)
                 ok = np.array_equal(g, ref) and s["stale"] == s["moved"] and s["launches"] == launches * world
+                if mode == abi.PK_MODE_PUSH and kern != "hotspot2d_tb2":   # tb2 cannot push
+                    ok = ok and s["pushed"] > 0
                 record(f"{kern}/mode{mode}", ok, bitwise=bool(np.array_equal(g, ref)), **s)
             dist.barrier()
 

@@ -467,3 +467,60 @@ def test_heat_tile_partitions_bitwise(kernel):
             gp, st = _heat(u, iters, tiles[0] * tiles[1] * tiles[2], 4, 8, kernel, tiles=tiles, mode=mode)
             assert np.array_equal(g1, gp), (tiles, mode)
             assert st["moved_bytes"] == st["stale_bytes"] > 0
+
+
+# ------------------------------------------------------------------ fused halo push (PK_MODE_PUSH, Q25)
+_PUSH_MODES = [abi.PK_MODE_PUSH, abi.PK_MODE_PUSH | abi.PK_MODE_NO_GRAPHS,
+               abi.PK_MODE_PUSH | abi.PK_MODE_GLOBAL_BARRIER]
+
+
+@pytest.mark.parametrize("mode", _PUSH_MODES)
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_push_hotspot_bitwise(P, mode):
+    """Producing kernels store the neighbours' halo rows into their instances: after the
+    first two launches nothing is stale, the result stays bit-identical to 1-way."""
+    h, w, iters = 300, 2048, 12
+    t, p = synth.hotspot_grids(h, w)
+    g1, _ = _hotspot(t, p, iters, 1, 16)
+    gp, st = _hotspot(t, p, iters, P, 16, mode=mode)
+    assert np.array_equal(g1, gp)
+    assert st["pushed_bytes"] > 0 and st["moved_bytes"] == st["stale_bytes"]
+    # launches 3.. need nothing: stale bytes = those of the first two launches only
+    _, st2 = _hotspot(t, p, 2, P, 16)
+    assert st["stale_bytes"] == st2["stale_bytes"]
+
+
+@pytest.mark.parametrize("P", [2, 4, 5])
+def test_push_hotspot_tbk_bitwise(P):
+    h, w, iters = 260, 1920, 16
+    t, p = synth.hotspot_grids(h, w)
+    g1, _ = _hotspot_k(t, p, iters, 1, 32, 4)
+    ctx = gpu_ctx(P, abi.PK_MODE_PUSH)
+    pr = K.hotspot2d_setup(ctx, t, p, ty=32, kernel="hotspot2d_tbk", sweeps=4)
+    gp = fetch(ctx, K.hotspot2d_iterate(pr, iters), t.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g1, gp)
+    # steady state: every launch pushes 4 rows each way per cut
+    assert st["pushed_bytes"] == (iters // 4 - 1) * 4 * cf.hotspot2d_stale_per_iter(w, P)
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_push_heat_and_jacobi_bitwise(P):
+    u = synth.heat_grid(40, 36, 132)
+    r1, _ = _heat(u, 6, 1)
+    rp, st = _heat(u, 6, P, mode=abi.PK_MODE_PUSH)
+    assert np.array_equal(r1, rp) and st["pushed_bytes"] == 5 * cf.heat3d_stale_per_iter(36, 132, P)
+    uj = synth.jacobi_grid(512, 512)
+    c1 = gpu_ctx(1)
+    _, ob = K.jacobi2d_program(c1, uj, 10)
+    j1 = fetch(c1, ob, uj.shape)
+    abi.pk_finalize(c1)
+    cp = gpu_ctx(P, abi.PK_MODE_PUSH)
+    _, ob = K.jacobi2d_program(cp, uj, 10)
+    jp = fetch(cp, ob, uj.shape)
+    st = abi.pk_get_stats(cp)
+    abi.pk_finalize(cp)
+    assert np.array_equal(j1, jp)
+    if P == 2:   # C1: 2 x 4,080 B pulled instead of 40,800 B, the rest pushed
+        assert st["stale_bytes"] == 8160 and st["pushed_bytes"] == 9 * 4080

@@ -217,7 +217,7 @@ def _norm_plan(plan, names):
     return res
 
 
-def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0, tiles=None):
+def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0, tiles=None, push_arg=None):
     """specs: {name: (shape, eb, uploaded)}; launches: list of [arg binding names or None];
     thread_prog(box) -> oracle access dict keyed by (arg, 'r'/'w'); tiles: NEXT-2 tile shape."""
     ctx = host_ctx(P, mode)
@@ -254,8 +254,9 @@ def _run_pair(P, kernel, specs, launches, geom, thread_prog, mode=0, tiles=None)
                     w = np.union1d(w, el)
                 d[name] = (r, w)
             per.append(d)
-        res = sh.launch(per)
+        res = sh.launch(per, push=(binding[push_arg],) if (mode & abi.PK_MODE_PUSH) and push_arg is not None else ())
         st_ = abi.pk_get_stats(ctx)
+        assert st_["pushed_bytes"] == sh.pushed_bytes
         assert st_["stale_bytes"] - stale_prev == sum(res["stale"])
         stale_prev = st_["stale_bytes"]
         exp_plan = {key: regions.to_byte_ranges(el, specs[key[0]][1]) for key, el in res["copies"].items()}
@@ -568,3 +569,57 @@ def test_hotspot_tb2_sequence(P):
                        lambda box: regions.hotspot2d_tb2(box, geom[1], h, w, 4))
     # 2 halo rows of temp each way per boundary per launch, + the 1-row power halo once
     assert st_["stale_bytes"] == 4 * 2 * cf.hotspot2d_stale_per_iter(w, P) + cf.hotspot2d_stale_per_iter(w, P)
+
+
+# ------------------------------------------------------------ fused halo push (PK_MODE_PUSH, reading Q25)
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_push_jacobi_sequence_vs_shadow(P):
+    """Tracker, plans, stale and pushed bytes with the predictive push == shadow oracle;
+    after the first two launches nothing is stale any more."""
+    n, iters = 64, 8
+    geom = K.jacobi2d_launch(n, n)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), n, n] for t in range(iters)]
+    st_, sh = _run_pair(P, "jacobi2d", {"u0": ((n, n), 4, True), "u1": ((n, n), 4, True)}, launches, geom,
+                        lambda box: regions.jacobi2d(box, geom[1], n, n), mode=abi.PK_MODE_PUSH, push_arg=1)
+    per_iter = cf.jacobi2d_stale_per_iter(n, P)
+    pull2, _ = _jacobi_case(n, P, 2)                      # launches 1 and 2 pull, then everything is pushed
+    assert st_["stale_bytes"] == pull2["stale_bytes"]
+    if P == 2:                                            # (P = 3 also repairs the linear H2D split, reading Q2)
+        assert st_["stale_bytes"] == 2 * per_iter
+    assert st_["pushed_bytes"] == (iters - 1) * per_iter
+
+
+@pytest.mark.parametrize("kernel,P", [("hotspot2d", 2), ("hotspot2d", 4), ("hotspot2d_tbk", 3)])
+def test_push_hotspot_sequence_vs_shadow(kernel, P):
+    h, w = 64, 1024
+    if kernel == "hotspot2d_tbk":
+        geom = K.hotspot2d_tbk_launch(h, w, 8, 4)
+        prog = lambda box: regions.hotspot2d_tbk(box, geom[1], h, w, 8, 4)
+    else:
+        geom = K.hotspot2d_launch(h, w, 4, 128)
+        prog = lambda box: regions.hotspot2d(box, geom[1], h, w, 4)
+    launches = [[("t0" if t % 2 == 0 else "t1"), "pw", ("t1" if t % 2 == 0 else "t0"), h, w, geom[2][2]]
+                for t in range(6)]
+    st_, _ = _run_pair(P, kernel, {"t0": ((h, w), 4, True), "t1": ((h, w), 4, False), "pw": ((h, w), 4, True)},
+                       launches, geom, prog, mode=abi.PK_MODE_PUSH, push_arg=2)
+    assert st_["pushed_bytes"] > 0
+
+
+def test_push_heat_sequence_vs_shadow():
+    d, h, w = 16, 8, 64
+    geom = K.heat3d_launch(d, h, w, 4, 8)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), d, h, w, 4] for t in range(5)]
+    st_, _ = _run_pair(2, "heat3d", {"u0": ((d, h, w), 4, True), "u1": ((d, h, w), 4, False)}, launches, geom,
+                       lambda box: regions.heat3d(box, geom[1], d, h, w, 4), mode=abi.PK_MODE_PUSH, push_arg=1)
+    assert st_["pushed_bytes"] == 4 * cf.heat3d_stale_per_iter(h, w, 2)   # launches 2..5 push
+
+
+def test_push_tiles_fall_back_to_pull():
+    """A 2x2 tile split makes W_q n R_p per-row pieces (> 4 runs): no push, everything pulled."""
+    n = 64
+    geom = K.jacobi2d_launch(n, n)
+    launches = [[("u0" if t % 2 == 0 else "u1"), ("u1" if t % 2 == 0 else "u0"), n, n] for t in range(4)]
+    st_, _ = _run_pair(4, "jacobi2d", {"u0": ((n, n), 4, True), "u1": ((n, n), 4, True)}, launches, geom,
+                       lambda box: regions.jacobi2d(box, geom[1], n, n), mode=abi.PK_MODE_PUSH, push_arg=1,
+                       tiles=(2, 2, 1))
+    assert st_["pushed_bytes"] == 0
