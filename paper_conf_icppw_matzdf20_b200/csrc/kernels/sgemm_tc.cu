@@ -8,18 +8,30 @@
 // Split (reading Q17): x = hi + lo with hi = x truncated to TF32 (low 13
 // mantissa bits cleared, exactly representable), lo = round_tf32(x - hi);
 //   C = A_hi B_hi + A_hi B_lo + A_lo B_hi     (the A_lo B_lo term is < 2^-20 relative)
-// accumulated in FP32 in TMEM, fixed K order, no split-K (so a P-way row
-// partition is bit-identical to the 1-way launch).
+// accumulated in FP32, fixed K order, no split-K (so a P-way row partition is
+// bit-identical to the 1-way launch).
+//
+// Chunked accumulation: the tensor core's FP32 accumulator loses the bits below
+// its alignment on every MMA (measured: the error relative to RMS(C) grows
+// LINEARLY with K -- 2.3e-5 at K = 1024, 3.5e-4 at K = 16384, 1.4e-3 at 65536 for a
+// single TMEM accumulator, i.e. each element drifts toward zero by ~2^-23 of its
+// running value per MMA).  So the TMEM accumulator only spans KC = 512 of K: the
+// MMA warp alternates between two TMEM accumulators, and the epilogue warps add
+// each finished chunk into FP32 registers (round-to-nearest) while the next chunk
+// is being computed.  The error then grows with the chunk length, not with K.
 //
 // Per partitioned launch the launcher runs, on the partition's stream:
 //   1. k_split_rows   : A rows of this partition -> A_hi, A_lo (M x K, K-major)
 //   2. k_split_transp : all of B (K x N) -> Bt_hi, Bt_lo (N x K, K-major)
-//   3. k_sgemm_tf32x3 : one CTA per 128 x 256 C tile (logical block), 8 warps:
+//   3. k_sgemm_tf32x3 : one CTA per 128 x 256 C tile (logical block), 12 warps:
 //        warp 0   TMA producer (cp.async.bulk.tensor.2d, 64-B swizzle, 4 stages)
 //        warp 1   MMA issuer (one thread: tcgen05.mma.cta_group::1.kind::tf32,
 //                 M = 128, N = 256, K = 8 per instruction, 3 per K-step)
-//        warp 2   TMEM allocator (256 columns = the 128 x 256 FP32 accumulator)
-//        warps 4-7 epilogue (tcgen05.ld 32x32b -> registers -> global)
+//        warp 2   TMEM allocator (2 x 256 columns: two 128 x 256 FP32 accumulators)
+//        warps 4-11 epilogue (tcgen05.ld 32x32b -> FP32 running sums in registers,
+//                 128 per thread = half a C row -> global)
+// (N = 128 tiles with 4 epilogue warps were tried for the chunked accumulation:
+// shared-memory bound, 181 vs 258 TF/s: operand reads + TMA fills exceed 128 B/clk.)
 // Scratch (hi/lo operands) is private to the launch, allocated per stream.
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -37,7 +49,10 @@ constexpr int BM = 128, BN = 256, BK = 16, STAGES = 4;
 constexpr int A_TILE = BM * BK * 4;                 // 8 KB
 constexpr int B_TILE = BN * BK * 4;                 // 16 KB
 constexpr int STAGE_BYTES = 2 * A_TILE + 2 * B_TILE; // 48 KB
-constexpr int TMEM_COLS = 256;
+constexpr int kThreads = 384;                       // 4 role warps + 8 epilogue warps
+constexpr int EPI_COLS = BN / 2;                    // columns per epilogue thread
+constexpr int TMEM_COLS = 2 * BN;                   // two accumulators
+constexpr int KC_BLOCKS = 32;                       // K per TMEM accumulator chunk = 32 * BK = 512
 constexpr size_t SMEM_BYTES = (size_t)STAGES * STAGE_BYTES + 1024 + 256;
 
 // ---------------------------------------------------------------- split kernels
@@ -127,6 +142,18 @@ __device__ __forceinline__ void tma_2d(void* dst, const CUtensorMap* map, int32_
         : "memory");
 }
 
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
+    uint32_t r[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
     uint32_t r[32];
     asm volatile(
@@ -143,7 +170,7 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
 }
 
 // ---------------------------------------------------------------- the GEMM
-__global__ void __launch_bounds__(256, 1)
+__global__ void __launch_bounds__(kThreads, 1)
     k_sgemm_tf32x3(const __grid_constant__ CUtensorMap tm_ahi, const __grid_constant__ CUtensorMap tm_alo,
                    const __grid_constant__ CUtensorMap tm_bhi, const __grid_constant__ CUtensorMap tm_blo,
                    float* __restrict__ C, int64_t M, int64_t N, int64_t K, pk_partition part) {
@@ -151,8 +178,9 @@ __global__ void __launch_bounds__(256, 1)
     unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + (size_t)STAGES * STAGE_BYTES);
     uint64_t* empty = full + STAGES;
-    uint64_t* tmem_full = empty + STAGES;
-    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(tmem_full + 1);
+    uint64_t* acc_full = empty + STAGES;   // [2]: chunk finished in accumulator a
+    uint64_t* acc_empty = acc_full + 2;    // [2]: accumulator a drained by the epilogue
+    uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(acc_empty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // Grouped rasterisation: the CTAs running at the same time cover kGroup tile
@@ -176,7 +204,10 @@ __global__ void __launch_bounds__(256, 1)
             ptx::mbar_init(&full[s], 1);
             ptx::mbar_init(&empty[s], 1);
         }
-        ptx::mbar_init(tmem_full, 1);
+        for (int a = 0; a < 2; ++a) {
+            ptx::mbar_init(&acc_full[a], 1);
+            ptx::mbar_init(&acc_empty[a], 8);   // one arrival per epilogue warp
+        }
         ptx::fence_mbar_init();
         asm volatile("prefetch.tensormap [%0];" ::"l"(&tm_ahi) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(&tm_alo) : "memory");
@@ -215,41 +246,62 @@ __global__ void __launch_bounds__(256, 1)
         for (int kb = 0; kb < nk; ++kb) {
             const int s = kb % STAGES;
             const uint32_t ph = (kb / STAGES) & 1u;
+            const int chunk = kb / KC_BLOCKS, a = chunk & 1;
+            const bool first = kb % KC_BLOCKS == 0;
+            if (first && chunk >= 2) {  // accumulator a still holds chunk-2 until the epilogue drained it
+                ptx::mbar_wait(&acc_empty[a], (uint32_t)((chunk / 2 - 1) & 1));
+            }
             ptx::mbar_wait(&full[s], ph);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             const uint32_t st = ptx::smem_u32(smem + (size_t)s * STAGE_BYTES);
+            const uint32_t acc = tmem + (uint32_t)(a * BN);
 #pragma unroll
             for (int kk = 0; kk < BK / 8; ++kk) {
                 const uint32_t ko = kk * 32;  // 8 TF32 = 32 B along K inside the 64-B swizzle row
                 const uint64_t ahi = umma_desc_k_sw64(st + ko), alo = umma_desc_k_sw64(st + A_TILE + ko);
                 const uint64_t bhi = umma_desc_k_sw64(st + 2 * A_TILE + ko);
                 const uint64_t blo = umma_desc_k_sw64(st + 2 * A_TILE + B_TILE + ko);
-                umma_tf32(tmem, ahi, bhi, idesc, (kb | kk) ? 1u : 0u);
-                umma_tf32(tmem, ahi, blo, idesc, 1u);
-                umma_tf32(tmem, alo, bhi, idesc, 1u);
+                umma_tf32(acc, ahi, bhi, idesc, (first && kk == 0) ? 0u : 1u);
+                umma_tf32(acc, ahi, blo, idesc, 1u);
+                umma_tf32(acc, alo, bhi, idesc, 1u);
             }
             umma_commit(&empty[s]);  // frees the smem stage when these MMAs complete
+            if (kb % KC_BLOCKS == KC_BLOCKS - 1 || kb == nk - 1) umma_commit(&acc_full[a]);
         }
-        umma_commit(tmem_full);
     } else if (warp >= 4) {
-        // ---------------- epilogue: TMEM -> registers -> global
-        ptx::mbar_wait(tmem_full, 0);
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const int q = warp & 3;
+        // ---------------- epilogue: chunk accumulators -> FP32 running sums -> global
+        const int q = warp & 3;                     // TMEM lane quarter of this warp
+        const int half = (warp - 4) >> 2;           // column half of the tile
         const int64_t row = m0 + 32 * q + lane;
-#pragma unroll 1
-        for (int c = 0; c < BN; c += 32) {
-            float v[32];
-            tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)c, v);
-            if (row < M) {
-                float* dst = C + row * N + n0 + c;
-                if (n0 + c + 32 <= N && (N % 4) == 0) {
+        const int nchunks = (nk + KC_BLOCKS - 1) / KC_BLOCKS;
+        float sum[EPI_COLS];
 #pragma unroll
-                    for (int i = 0; i < 32; i += 4)
-                        *reinterpret_cast<float4*>(dst + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+        for (int i = 0; i < EPI_COLS; ++i) sum[i] = 0.f;
+        for (int chunk = 0; chunk < nchunks; ++chunk) {
+            const int a = chunk & 1;
+            ptx::mbar_wait(&acc_full[a], (uint32_t)((chunk / 2) & 1));
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll
+            for (int c = 0; c < EPI_COLS; c += 16) {
+                float v[16];
+                tmem_ld16(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(a * BN + half * EPI_COLS + c), v);
+#pragma unroll
+                for (int i = 0; i < 16; ++i) sum[c + i] += v[i];   // round-to-nearest FP32 add
+            }
+            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&acc_empty[a]);
+        }
+        if (row < M) {
+            const int64_t c0 = n0 + half * EPI_COLS;
+            float* dst = C + row * N + c0;
+#pragma unroll
+            for (int c = 0; c < EPI_COLS; c += 4) {
+                if (c0 + c + 4 <= N && (N % 4) == 0) {
+                    *reinterpret_cast<float4*>(dst + c) = make_float4(sum[c], sum[c + 1], sum[c + 2], sum[c + 3]);
                 } else {
-                    for (int i = 0; i < 32; ++i)
-                        if (n0 + c + i < N) dst[i] = v[i];
+                    for (int i = 0; i < 4; ++i)
+                        if (c0 + c + i < N) dst[c + i] = sum[c + i];
                 }
             }
         }
@@ -372,7 +424,7 @@ cudaError_t launch_sgemm(const LaunchInfo& li) {
         attr = true;
     }
     void* argv[] = {&tm[0], &tm[1], &tm[2], &tm[3], &C, &M, &N, &K, (void*)&li.part};
-    return cudaLaunchKernel((const void*)k_sgemm_tf32x3, li.grid, dim3(256), argv, SMEM_BYTES, li.stream);
+    return cudaLaunchKernel((const void*)k_sgemm_tf32x3, li.grid, dim3(kThreads), argv, SMEM_BYTES, li.stream);
 }
 
 }  // namespace

@@ -52,7 +52,7 @@ GEMM_BM, GEMM_BN = 128, 256
 
 
 def sgemm_launch(m, n, k):
-    """Logical block = one 128 x 256 C tile (the kernel runs 8 warps per tile)."""
+    """Logical block = one 128 x 256 C tile (the kernel runs 12 warps per tile)."""
     return (_cdiv(n, GEMM_BN), _cdiv(m, GEMM_BM), 1), (256, 1, 1), [m, n, k]
 
 
