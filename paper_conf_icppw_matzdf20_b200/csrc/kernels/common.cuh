@@ -45,13 +45,17 @@ namespace dev {
 // Halo push (PK_MODE_PUSH): the value just stored at byte offset `off` of the output
 // instance also goes to every destination instance whose push range covers it
 // (4-byte granularity ranges; `n` is uniform, usually 0 or 2).
+// (static indices only: a runtime-indexed by-value struct would be copied to local
+// memory.  Kernels instantiate a PUSH=false variant without any of this.)
 __device__ __forceinline__ void push4(const PushList& pl, uint64_t off, const float4& v) {
-    for (int i = 0; i < pl.n; ++i)
-        if (off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float4*>(pl.dst[i] + off) = v;
+#pragma unroll
+    for (int i = 0; i < kMaxPush; ++i)
+        if (i < pl.n && off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float4*>(pl.dst[i] + off) = v;
 }
 __device__ __forceinline__ void push1(const PushList& pl, uint64_t off, float v) {
-    for (int i = 0; i < pl.n; ++i)
-        if (off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float*>(pl.dst[i] + off) = v;
+#pragma unroll
+    for (int i = 0; i < kMaxPush; ++i)
+        if (i < pl.n && off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float*>(pl.dst[i] + off) = v;
 }
 }  // namespace dev
 }  // namespace pk

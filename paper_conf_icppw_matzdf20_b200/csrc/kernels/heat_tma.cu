@@ -57,6 +57,7 @@ __device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_
         : "memory");
 }
 
+template <bool PUSH>
 __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUtensorMap tm_u,
                                                     float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
                                                     int64_t ZC, int bdy, pk_partition part, PushList push) {
@@ -141,7 +142,7 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUt
             o.z = c.z + kAlpha * ((zm.z + zp.z + ym.z + yp.z + c.y + c.w) - 6.0f * c.z);
             o.w = c.w + kAlpha * ((zm.w + zp.w + ym.w + yp.w + c.z + ev) - 6.0f * c.w);
             *reinterpret_cast<float4*>(uout + kout + i * W + j0) = o;
-            if (push.n) dev::push4(push, (uint64_t)(kout + i * W + j0) * 4u, o);  // fused halo push
+            if (PUSH) dev::push4(push, (uint64_t)(kout + i * W + j0) * 4u, o);  // fused halo push
         }
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&empty[s_m]);  // slot z-1 no longer needed by this warp
@@ -183,8 +184,11 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
     static std::once_flag once;
     static cudaError_t attr_err = cudaSuccess;
     std::call_once(once, [] {
-        attr_err = cudaFuncSetAttribute(k_heat3d_tma, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        attr_err = cudaFuncSetAttribute(k_heat3d_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         (int)smem_bytes(kMaxBdy));
+        if (attr_err == cudaSuccess)
+            attr_err = cudaFuncSetAttribute(k_heat3d_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)smem_bytes(kMaxBdy));
     });
     if (attr_err != cudaSuccess) return attr_err;
     // tensor map of this instance: dims (W, H, D), box (136, bdy + 2, 1), OOB zero fill
@@ -209,14 +213,14 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part, &pl};
-    return cudaLaunchKernel((const void*)k_heat3d_tma, li.grid, dim3(32, warp_count(bdy) + 1), argv, smem_bytes(bdy),
-                            li.stream);
+    const void* fn = (li.push && li.push->n > 0) ? (const void*)k_heat3d_tma<true> : (const void*)k_heat3d_tma<false>;
+    return cudaLaunchKernel(fn, li.grid, dim3(32, warp_count(bdy) + 1), argv, smem_bytes(bdy), li.stream);
 }
 
 }  // namespace
 
 const Builtin kBuiltinHeat3dTma = {
-    "heat3d", (const void*)k_heat3d_tma, 6,
+    "heat3d", (const void*)k_heat3d_tma<false>, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
     describe_heat3d_tma, launch_heat3d_tma, /*push_arg=*/1};
 

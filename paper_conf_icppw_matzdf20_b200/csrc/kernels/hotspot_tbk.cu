@@ -88,7 +88,7 @@ __device__ __forceinline__ float4 level(const float4& c, const float4& n, const 
 // in registers (4-fold unroll) needs 168 registers -> 2 CTAs/SM, 1764 GLUP/s; a
 // skewed level schedule (level k at row t-2k+1, independent levels) 1476 GLUP/s;
 // this variant at 128 registers, 3 CTAs/SM and a 16-stage ring: 1940 GLUP/s.
-template <int K, bool EDGE, bool COLEDGE>
+template <int K, bool EDGE, bool COLEDGE, bool PUSH>
 __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, uint64_t* empty, float* tout,
                                              int64_t W, int H, int64_t c0, int64_t r0, int64_t rend, bool down,
                                              uint32_t g, int lane, int warp, const PushList& push) {
@@ -136,7 +136,7 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
                 } else if (t >= 2 * K) {
                     if (store) {
                         *reinterpret_cast<float4*>(outp) = o;
-                        if (push.n) dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
+                        if (PUSH) dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
                     }
                     outp += dW;
                 }
@@ -152,7 +152,7 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
 #ifndef PK_TBK_MINB
 #define PK_TBK_MINB 3
 #endif
-template <int K>
+template <int K, bool PUSH>
 __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const float* __restrict__ tin,
                                                             const float* __restrict__ pw,
                                                             float* __restrict__ tout, int64_t H, int64_t W,
@@ -206,9 +206,11 @@ __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const f
         const bool redge = r0 < K + 1 || rend + K + 1 > H;
         const bool cedge = c0 == 0 || c0 + kTC + 4 >= W;
         if (redge || cedge)
-            consume_tile<K, true, true>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp, push);
+            consume_tile<K, true, true, PUSH>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp,
+                                              push);
         else
-            consume_tile<K, false, false>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp, push);
+            consume_tile<K, false, false, PUSH>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp,
+                                                push);
         g += (uint32_t)(rend - r0) + 2 * K;
     }
 }
@@ -246,18 +248,18 @@ int describe_hotspot2d_tbk(pk_ctx c, pk_kernel k) {
     return pk_declare_affine_access(c, k, 2, PK_WRITE, &w);
 }
 
-template <int K>
+template <int K, bool PUSH>
 cudaError_t launch_k(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
     static int resident[64] = {0};
     static int sms[64] = {0};
     const int d = li.device;
     if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
     if (!resident[d]) {
-        cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tbk<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tbk<K, PUSH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)kSmem);
         if (e != cudaSuccess) return e;
         int nb = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_hotspot2d_tbk<K>, kThreads, kSmem);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_hotspot2d_tbk<K, PUSH>, kThreads, kSmem);
         if (e != cudaSuccess) return e;
         e = cudaDeviceGetAttribute(&sms[d], cudaDevAttrMultiProcessorCount, d);
         if (e != cudaSuccess) return e;
@@ -270,7 +272,7 @@ cudaError_t launch_k(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part, &pl};
-    return cudaLaunchKernel((const void*)k_hotspot2d_tbk<K>, grid, dim3(kThreads), argv, kSmem, li.stream);
+    return cudaLaunchKernel((const void*)k_hotspot2d_tbk<K, PUSH>, grid, dim3(kThreads), argv, kSmem, li.stream);
 }
 
 cudaError_t launch_hotspot2d_tbk(const LaunchInfo& li) {
@@ -279,10 +281,11 @@ cudaError_t launch_hotspot2d_tbk(const LaunchInfo& li) {
     if (W % 4 || W < 4 || TY < 1 || H < 1 || H > (1ll << 30) || li.block.x != kConsumers || li.block.y != 1 ||
         li.block.z != 1)
         return cudaErrorInvalidValue;
+    const bool push = li.push && li.push->n > 0;
     switch (K) {
-        case 2: return launch_k<2>(li, H, W, TY);
-        case 3: return launch_k<3>(li, H, W, TY);
-        case 4: return launch_k<4>(li, H, W, TY);
+        case 2: return push ? launch_k<2, true>(li, H, W, TY) : launch_k<2, false>(li, H, W, TY);
+        case 3: return push ? launch_k<3, true>(li, H, W, TY) : launch_k<3, false>(li, H, W, TY);
+        case 4: return push ? launch_k<4, true>(li, H, W, TY) : launch_k<4, false>(li, H, W, TY);
         default: return cudaErrorInvalidValue;
     }
 }
@@ -290,7 +293,7 @@ cudaError_t launch_hotspot2d_tbk(const LaunchInfo& li) {
 }  // namespace
 
 const Builtin kBuiltinHotspot2dTbk = {
-    "hotspot2d_tbk", (const void*)k_hotspot2d_tbk<4>, 6,
+    "hotspot2d_tbk", (const void*)k_hotspot2d_tbk<4, false>, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
     describe_hotspot2d_tbk, launch_hotspot2d_tbk, /*push_arg=*/2};
 

@@ -44,6 +44,7 @@ __device__ __forceinline__ float hs(float c, float n, float s, float e, float w,
     return c + kCap * (p + (s + n - 2.0f * c) * kRy1 + (e + w - 2.0f * c) * kRx1 + (kAmb - c) * kRz1);
 }
 
+template <bool PUSH>
 __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restrict__ tin,
                                                             const float* __restrict__ pw,
                                                             float* __restrict__ tout, int64_t H, int64_t W,
@@ -126,7 +127,7 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restr
                 o.w = hs(c.w, a.w, b.w, ev, c.z, p.w);
                 const int64_t row = down ? r0 - 1 + t : rend - t;
                 *reinterpret_cast<float4*>(tout + row * W + j0) = o;
-                if (push.n) dev::push4(push, (uint64_t)(row * W + j0) * 4u, o);  // fused halo push
+                if (PUSH) dev::push4(push, (uint64_t)(row * W + j0) * 4u, o);  // fused halo push
             }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&empty[gp % kNS]);
@@ -159,21 +160,17 @@ int describe_hotspot2d_tma(pk_ctx c, pk_kernel k) {
     return PK_OK;
 }
 
-cudaError_t launch_hotspot2d_tma(const LaunchInfo& li) {
-    if (li.nscalars < 3) return cudaErrorInvalidValue;
-    int64_t H = li.scalars[0], W = li.scalars[1], TY = li.scalars[2];
-    // logical block = 128 threads x 4 columns (the launcher adds the producer warp)
-    if (W % 4 || W < 4 || TY < 1 || li.block.x != kConsumers || li.block.y != 1 || li.block.z != 1)
-        return cudaErrorInvalidValue;
+template <bool PUSH>
+cudaError_t launch_tma(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
     static int resident[64] = {0};
     static int sms[64] = {0};
     const int d = li.device;
     if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
     if (!resident[d]) {
-        cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
+        cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tma<PUSH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
         if (e != cudaSuccess) return e;
         int nb = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_hotspot2d_tma, kThreads, kSmem);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_hotspot2d_tma<PUSH>, kThreads, kSmem);
         if (e != cudaSuccess) return e;
         e = cudaDeviceGetAttribute(&sms[d], cudaDevAttrMultiProcessorCount, d);
         if (e != cudaSuccess) return e;
@@ -186,13 +183,24 @@ cudaError_t launch_hotspot2d_tma(const LaunchInfo& li) {
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part, &pl};
-    return cudaLaunchKernel((const void*)k_hotspot2d_tma, grid, dim3(kThreads), argv, kSmem, li.stream);
+    return cudaLaunchKernel((const void*)k_hotspot2d_tma<PUSH>, grid, dim3(kThreads), argv, kSmem, li.stream);
 }
+
+cudaError_t launch_hotspot2d_tma(const LaunchInfo& li) {
+    if (li.nscalars < 3) return cudaErrorInvalidValue;
+    int64_t H = li.scalars[0], W = li.scalars[1], TY = li.scalars[2];
+    // logical block = 128 threads x 4 columns (the launcher adds the producer warp)
+    if (W % 4 || W < 4 || TY < 1 || li.block.x != kConsumers || li.block.y != 1 || li.block.z != 1)
+        return cudaErrorInvalidValue;
+    if (li.push && li.push->n > 0) return launch_tma<true>(li, H, W, TY);
+    return launch_tma<false>(li, H, W, TY);
+}
+
 
 }  // namespace
 
 const Builtin kBuiltinHotspot2dTma = {
-    "hotspot2d", (const void*)k_hotspot2d_tma, 6,
+    "hotspot2d", (const void*)k_hotspot2d_tma<false>, 6,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
     describe_hotspot2d_tma, launch_hotspot2d_tma, /*push_arg=*/2};
 

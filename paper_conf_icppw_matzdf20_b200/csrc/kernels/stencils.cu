@@ -28,6 +28,7 @@ using dev::st4;
 // ============================================================ C1 jacobi2d
 // One thread per cell: i = by*bdy + ty, j = bx*bdx + tx; Dirichlet interior
 //   out[i][j] = 0.25 * (((in[i-1][j] + in[i+1][j]) + in[i][j-1]) + in[i][j+1])
+template <bool PUSH>
 __global__ void __launch_bounds__(256) k_jacobi2d(const float* __restrict__ in, float* __restrict__ out,
                                                   int64_t H, int64_t W, pk_partition part, PushList push) {
     const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y;  // Eq. 8
@@ -37,7 +38,7 @@ __global__ void __launch_bounds__(256) k_jacobi2d(const float* __restrict__ in, 
     const float w = in[i * W + j - 1], e = in[i * W + j + 1];
     const float v = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(__fadd_rn(n, s), w), e));
     out[i * W + j] = v;
-    if (push.n) dev::push1(push, (uint64_t)(i * W + j) * 4u, v);  // fused halo push
+    if (PUSH) dev::push1(push, (uint64_t)(i * W + j) * 4u, v);  // fused halo push
 }
 
 int describe_jacobi2d(pk_ctx c, pk_kernel k) {
@@ -61,7 +62,8 @@ cudaError_t launch_jacobi2d(const LaunchInfo& li) {
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &H, &W, (void*)&li.part, &pl};
-    return cudaLaunchKernel(li.fn, li.grid, li.block, argv, 0, li.stream);
+    const void* fn = (li.push && li.push->n > 0) ? (const void*)k_jacobi2d<true> : (const void*)k_jacobi2d<false>;
+    return cudaLaunchKernel(fn, li.grid, li.block, argv, 0, li.stream);
 }
 
 // ============================================================ C2 hotspot2d
@@ -287,7 +289,7 @@ cudaError_t launch_heat3d(const LaunchInfo& li) {
 }  // namespace
 
 const Builtin kBuiltinJacobi2d = {
-    "jacobi2d", (const void*)k_jacobi2d, 4,
+    "jacobi2d", (const void*)k_jacobi2d<false>, 4,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1, describe_jacobi2d, launch_jacobi2d,
     /*push_arg=*/1};
 const Builtin kBuiltinHotspot2d = {
