@@ -95,7 +95,11 @@ int pk_finalize(pk_ctx ctx);
  * (replicated, deterministic) on every rank; a rank executes only the kernels of
  * the partitions it owns (part_rank[p] == my_rank) and its side of each copy.
  * Copies between partitions of different ranks are NCCL send/recv pairs on the
- * owning partitions' streams (NCCL is loaded at run time from libnccl.so.2).
+ * owning partitions' streams (NCCL is loaded at run time from libnccl.so.2); when
+ * a launch's plan for a buffer is exactly "every partition reads the whole buffer
+ * and partition q holds the q-th of P equal linear slabs" (N-body positions every
+ * step, GEMM B), that buffer moves as ONE in-place ncclAllGather instead
+ * (pk_stats.collectives; NVLS multicast on NVSwitch).
  * Execution requires exactly one partition per rank; host-only contexts accept
  * any mapping (planning / tests).
  * pk_nccl_unique_id writes the 128-byte ncclUniqueId (rank 0 creates it, the
@@ -328,6 +332,7 @@ typedef struct {
     uint64_t strided_copies;     /* of `copies`: equal pieces at a constant pitch (2-D / 3-D) */
     uint64_t copy_kernels;       /* of `strided_copies`: narrow runs moved by the SM halo-copy kernel */
     uint64_t pushed_bytes;       /* bytes stored into other partitions' instances by producing kernels (PK_MODE_PUSH) */
+    uint64_t collectives;        /* NCCL SPMD: whole-buffer reads moved as one in-place all-gather */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);

@@ -69,6 +69,7 @@ struct NcclApi {
     int (*CommDestroy)(void* comm) = nullptr;
     int (*Send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
     int (*Recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+    int (*AllGather)(const void*, void*, size_t, int, void*, cudaStream_t) = nullptr;
     int (*GroupStart)() = nullptr;
     int (*GroupEnd)() = nullptr;
     const char* (*GetErrorString)(int) = nullptr;
@@ -91,10 +92,12 @@ const NcclApi& nccl() {
     api.CommDestroy = (int (*)(void*))dlsym(h, "ncclCommDestroy");
     api.Send = (int (*)(const void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclSend");
     api.Recv = (int (*)(void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclRecv");
+    api.AllGather = (int (*)(const void*, void*, size_t, int, void*, cudaStream_t))dlsym(h, "ncclAllGather");
     api.GroupStart = (int (*)())dlsym(h, "ncclGroupStart");
     api.GroupEnd = (int (*)())dlsym(h, "ncclGroupEnd");
     api.GetErrorString = (const char* (*)(int))dlsym(h, "ncclGetErrorString");
-    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv && api.GroupStart &&
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv && api.AllGather &&
+             api.GroupStart &&
              api.GroupEnd && api.GetErrorString;
     return api;
 }
@@ -387,6 +390,36 @@ int choose_source(uint64_t mask, int p, int P) {
         if (d < bestd) { bestd = d; best = q; }
     }
     return best;
+}
+
+// when every partition reads a whole buffer whose holders are exactly
+// the linear slabs in rank order (N-body positions each step, GEMM B once), the
+// plan for that buffer is P(P-1) copies, slab q -> every p != q: one all-gather.
+// Returns the buffers whose plan entries form exactly that pattern (equal slabs).
+std::vector<int64_t> allgather_buffers(const std::vector<CopyOp>& plan, int P,
+                                       const std::vector<Buffer>& bufs) {
+    std::vector<int64_t> out;
+    if (P < 2) return out;
+    std::unordered_map<int64_t, std::vector<const CopyOp*>> by;
+    for (const CopyOp& o : plan) by[o.buf].push_back(&o);
+    for (auto& kv : by) {
+        const Buffer& B = bufs[kv.first];
+        const uint64_t n = B.bytes / B.eb;
+        if (n % P || kv.second.size() != (size_t)P * (P - 1)) continue;
+        const uint64_t slab = n / P * B.eb;
+        std::vector<uint8_t> seen((size_t)P * P, 0);
+        bool ok = true;
+        for (const CopyOp* o : kv.second) {
+            if (o->src == o->dst || o->b != (uint64_t)o->src * slab || o->e != (uint64_t)(o->src + 1) * slab ||
+                seen[(size_t)o->src * P + o->dst]++) {
+                ok = false;
+                break;
+            }
+        }
+        if (ok) out.push_back(kv.first);
+    }
+    std::sort(out.begin(), out.end());
+    return out;
 }
 
 int split_dim(const int32_t grid[3], int forced) {
@@ -1304,6 +1337,7 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
     a.stale_bytes += sign * d.stale_bytes;
     a.moved_bytes += sign * d.moved_bytes;
     a.pushed_bytes += sign * d.pushed_bytes;
+    a.collectives += sign * d.collectives;
     for (int i = 0; i < 16; ++i)
         for (int j = 0; j < 16; ++j) a.pair_bytes[i][j] += sign * d.pair_bytes[i][j];
 }
@@ -1581,6 +1615,13 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         }
     }
 
+    // NCCL SPMD: whole-buffer reads become one in-place all-gather per buffer
+    std::vector<int64_t> ag_bufs;
+    if (c->world > 1 && !c->ipc && transfer) {
+        ag_bufs = allgather_buffers(c->last_plan, P, c->bufs);
+        c->stats.collectives += ag_bufs.size();
+    }
+
     uint64_t t3 = now_ns();
     c->stats.host_ns_plan += t3 - t2;
     c->stats.launches += 1;
@@ -1770,9 +1811,28 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             } else if (c->world > 1) {
                 const NcclApi& n = nccl();
                 bool open = false;
+                // whole-buffer reads: one in-place ncclAllGather each (NVLS multicast on NVSwitch)
+                for (int64_t b : ag_bufs) {
+                    Buffer& B = c->bufs[b];
+                    const int me = c->first_local;
+                    const uint64_t slab = B.bytes / c->P;
+                    if (!open) {
+                        if (int r = c->set_device(c->dev[me])) return r;
+                        n.GroupStart();
+                        open = true;
+                    }
+                    int r = n.AllGather((const char*)B.inst[me] + (uint64_t)me * slab, B.inst[me], slab, kNcclUint8,
+                                        c->comm, c->stream[me]);
+                    if (r) { n.GroupEnd(); return fail(PK_ERR_NCCL, std::string("ncclAllGather: ") + n.GetErrorString(r)); }
+                    c->stats.copies += P - 1;
+                    c->stats.moved_bytes += (uint64_t)(P - 1) * slab;
+                    for (int q = 0; q < P && q < 16; ++q)
+                        if (q != me && me < 16) c->stats.pair_bytes[q][me] += slab;
+                }
                 for (const CopyOp& o : c->last_plan) {
                     const bool sl = c->local(o.src), dl = c->local(o.dst);
                     if (sl == dl) continue;
+                    if (std::binary_search(ag_bufs.begin(), ag_bufs.end(), o.buf)) continue;
                     if (!open) {
                         if (int r = c->set_device(c->dev[c->first_local])) return r;
                         n.GroupStart();

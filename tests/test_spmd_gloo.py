@@ -74,10 +74,11 @@ def _worker(rank, world, port, kernel, qdir, transport="nccl"):
     else:
         ctx = abi.pk_init_spmd(world, rank, world, list(range(world)), flags=abi.PK_INIT_HOST_ONLY)
     seq = _sequence(abi, K, ctx, kernel, world)
-    launches = abi.pk_get_stats(ctx)["kernel_launches"]
+    st = abi.pk_get_stats(ctx)
+    launches = st["kernel_launches"]
     abi.pk_finalize(ctx)
     allseq = [None] * world
-    dist.all_gather_object(allseq, (seq, launches))
+    dist.all_gather_object(allseq, (seq, launches, st["collectives"]))
     if rank == 0:
         import pickle
         with open(os.path.join(qdir, "res.pkl"), "wb") as f:
@@ -87,13 +88,16 @@ def _worker(rank, world, port, kernel, qdir, transport="nccl"):
 
 
 @pytest.mark.parametrize("kernel,transport", [("jacobi2d", "nccl"), ("hotspot2d", "nccl"), ("nbody", "nccl"),
-                                              ("hotspot2d", "ipc")])
+                                              ("hotspot2d", "ipc"), ("nbody", "ipc")])
 def test_spmd_two_ranks_replicated_plan_and_matched_transfers(kernel, transport, tmp_path):
     world = 2
     mp.spawn(_worker, args=(world, _free_port(), kernel, str(tmp_path), transport), nprocs=world, join=True)
     import pickle
     allseq = pickle.load(open(tmp_path / "res.pkl", "rb"))
-    (seq0, l0), (seq1, l1) = allseq
+    (seq0, l0, c0), (seq1, l1, c1) = allseq
+    # NCCL transport: the N-body position reads (every partition reads all bodies, slab
+    # holders in rank order) are one in-place all-gather per step; stencils have none
+    assert c0 == c1 == (3 if (kernel == "nbody" and transport == "nccl") else 0)
     # 1. replicated host state is identical on both ranks
     assert seq0 == seq1
     # 2. ... and identical to the single-process plan for the same P
