@@ -192,7 +192,10 @@ class Workload:
             self.upload_bufs = [(self.pr.tb[0], self.host[0]), (self.pr.tb[2], self.host[1])]
         elif self.name == "heat3d":
             self.pr = K.heat3d_setup(ctx, self.host[0], zc=tile or K.HEAT_ZC,
-                                     kernel=getattr(self, "variant", None) or "heat3d", tiles=self.tiles)
+                                     kernel=getattr(self, "variant", None) or "heat3d_tb2", tiles=self.tiles)
+            # two sweeps per launch for the default heat3d_tb2: 8 B per cell per launch = 4 B/LU
+            self.sweeps = self.pr.sweeps
+            self.bytes_per_unit = 8 / self.sweeps
             self.upload_bufs = [(self.pr.ub[0], self.host[0])]
         elif self.name == "sgemm":
             self.pr, _ = K.sgemm_program(ctx, *self.host, launches=0)
@@ -470,7 +473,7 @@ def main():
     units = w.units_per_iter * w.iters * args.steps
     value = units / (elapsed_ms / 1e3) / w.scale
     peaks = load_peaks()
-    kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk"}.get(w.name, w.name)
+    kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk", "heat3d": "heat3d_tb2"}.get(w.name, w.name)
     avg_kernel_ms = st["kernel_ms"] / max(1, st["timed_kernels"])
     per_launch_units = w.units_per_iter * getattr(w, "sweeps", 1) / P
     if w.name == "sgemm":
@@ -509,7 +512,8 @@ def main():
                    else "1 MB working set stays in L2 (latency-bound C1)",
                    "process_model": process_model,
                    "halo_push": bool(args.push),
-                   "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk"}.get(w.name, w.name),
+                   "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk",
+                                                             "heat3d": "heat3d_tb2"}.get(w.name, w.name),
                    "sweeps_per_launch": getattr(w, "sweeps", 1),
                    "partition_shape": list(w.tiles) if w.tiles else "1-D slabs of the slowest grid dim"},
         "gpu_launches": int(st["kernel_launches"] + st["copy_kernels"]),

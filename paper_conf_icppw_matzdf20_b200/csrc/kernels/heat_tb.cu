@@ -1,0 +1,278 @@
+// heat_tb.cu -- C3 3-D 7-point heat stencil, temporally blocked: TWO time steps
+// per launch (the 3-D counterpart of hotspot2d_tbk).
+//
+// Semantics: one launch = two consecutive sweeps of reading Q15
+//   u' = u + alpha((zm + zp + ym + yp + xm + xp) - 6u),  alpha = 1/8,
+// replicate-clamped at every sweep.  An output cell depends on the clamped
+// 5x5x5 cube of u_in around it, so a partition's read set is its box dilated by 2
+// and its write set its own cells: 8 B per cell per launch = 4 B per lattice
+// update (half the one-sweep kernel's 8 B/LU).
+//
+// Design (B200): logical block = 120 columns x 24 rows x ZC planes.  A producer
+// warp streams one 3-D tensor-TMA box per plane -- 128 columns [c0-4, c0+124) x
+// 28 rows [y0-2, y0+26) x 1 plane, out-of-grid columns/rows zero-filled, the plane
+// index clamped -- into a 6-slot mbarrier ring.  6 consumer warps march z; warp w
+// owns rows y0+4w .. +3, a lane owns 4 columns.  Per input plane q a warp computes
+// sweep 1 of plane q-1 on its 4 rows plus one halo row above and below (6 rows,
+// inputs from shared memory) into a register window of 3 planes x 6 rows, and
+// sweep 2 of plane q-2 on its own 4 rows from that window, which it stores.
+// x neighbours are warp shuffles; lanes 0 and 31 are halo lanes whose outer
+// column is wrong after each sweep (shuffle wrap), so lanes 1..30 store: 120
+// owned columns.  Halo rows, columns and planes of sweep 1 are recomputed by the
+// blocks that need them from identical inputs in identical order, so P-way
+// launches are bit-identical to 1-way; no barrier among consumers.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <mutex>
+#include <unordered_map>
+
+#include "../runtime/builtins.h"
+#include "common.cuh"
+#include "ptx.cuh"
+#include "tma_host.h"
+
+namespace pk {
+namespace {
+
+constexpr float kAlpha = 0.125f;
+constexpr int kCols = 128;                // columns per warp window (box width)
+constexpr int kOwnC = 120;                // owned columns per block (lanes 1..30)
+constexpr int kRW = 4;                    // owned rows per consumer warp
+constexpr int kNW = 6;                    // consumer warps
+constexpr int kRows = kRW * kNW;          // owned rows per block (24)
+constexpr int kBoxRows = kRows + 4;       // rows y0-2 .. y0+kRows+1
+constexpr int kL1 = kRW + 2;              // sweep-1 rows per warp (one halo row each side)
+#ifndef PK_HEATTB_NS
+#define PK_HEATTB_NS 6
+#endif
+constexpr int kNS = PK_HEATTB_NS;         // plane ring depth
+constexpr int kSlot = kBoxRows * kCols;   // floats per plane slot (14 KB)
+constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + 2 * kNS * 8 + 128;
+#ifndef PK_HEATTB_MINB
+#define PK_HEATTB_MINB 2
+#endif
+
+__device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, int32_t z,
+                                       uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+        "[%5];" ::"r"(ptx::smem_u32(dst)),
+        "l"(map), "r"(x), "r"(y), "r"(z), "r"(ptx::smem_u32(bar))
+        : "memory");
+}
+
+// u + alpha((zm + zp + ym + yp + w + e) - 6u), same operation order for every cell
+__device__ __forceinline__ float upd(float c, float zm, float zp, float ym, float yp, float w, float e) {
+    return c + kAlpha * ((zm + zp + ym + yp + w + e) - 6.0f * c);
+}
+
+__device__ __forceinline__ float4 sweep(const float4& c, const float4& zm, const float4& zp, const float4& ym,
+                                        const float4& yp, bool wclamp, bool eclamp) {
+    float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
+    float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
+    if (wclamp) wv = c.x;
+    if (eclamp) ev = c.w;
+    float4 o;
+    o.x = upd(c.x, zm.x, zp.x, ym.x, yp.x, wv, c.y);
+    o.y = upd(c.y, zm.y, zp.y, ym.y, yp.y, c.x, c.z);
+    o.z = upd(c.z, zm.z, zp.z, ym.z, yp.z, c.y, c.w);
+    o.w = upd(c.w, zm.w, zp.w, ym.w, yp.w, c.z, ev);
+    return o;
+}
+
+template <bool PUSH, bool EDGE>
+__device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint64_t* empty, float* __restrict__ uout,
+                                        int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
+                                        int lane, int warp, const PushList& push);
+
+template <bool PUSH>
+__global__ void __launch_bounds__((kNW + 1) * 32, PK_HEATTB_MINB)
+    k_heat3d_tb2(const __grid_constant__ CUtensorMap tm_u, float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
+                 int64_t ZC, pk_partition part, PushList push) {
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    // 128-B aligned ring; pointer arithmetic on the shared array (not a uintptr_t round
+    // trip) keeps the shared address space visible, so the loads below are LDS, not LD
+    float* ring = reinterpret_cast<float*>(smem_raw + ((128u - ((uint32_t)(uintptr_t)smem_raw & 127u)) & 127u));
+    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)kNS * kSlot);
+    uint64_t* empty = full + kNS;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y, bz = part.min[2] + blockIdx.z;
+    const int64_t c0 = bx * kOwnC, y0 = by * kRows, k0 = bz * ZC;  // Eq. 8
+    if (c0 >= W || y0 >= H || k0 >= D) return;                      // block-uniform
+    const int64_t k1 = min(k0 + ZC, D);
+    const int nz = (int)(k1 - k0);
+    const int nq = nz + 4;                                           // planes k0-2 .. k1+1 (clamped)
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kNS; ++s) {
+            ptx::mbar_init(&full[s], 1);
+            ptx::mbar_init(&empty[s], kNW);
+        }
+        ptx::fence_mbar_init();
+        asm volatile("prefetch.tensormap [%0];" ::"l"(&tm_u) : "memory");
+    }
+    __syncthreads();
+
+    if (warp == kNW) {  // ---------------- producer: one TMA box per plane
+        if (lane != 0) return;
+        constexpr uint32_t bytes = (uint32_t)kSlot * 4u;
+        for (int q = 0; q < nq; ++q) {
+            const int s = q % kNS;
+            ptx::mbar_wait(&empty[s], ((q / kNS) & 1u) ^ 1u);
+            int64_t p = k0 - 2 + q;
+            p = p < 0 ? 0 : (p >= D ? D - 1 : p);
+            ptx::mbar_arrive_expect_tx(&full[s], bytes);
+            tma_3d(ring + (size_t)s * kSlot, &tm_u, (int32_t)(c0 - 4), (int32_t)(y0 - 2), (int32_t)p, &full[s]);
+        }
+        return;
+    }
+
+    // ---------------- consumers: blocks touching the grid's first/last row or plane apply
+    // the replicate clamp of the intermediate sweep; interior blocks skip the selects
+    const bool edge = y0 < 2 || y0 + kRows + 2 > H || k0 < 2 || k0 + ZC + 2 > D;
+    if (edge)
+        consume<PUSH, true>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+    else
+        consume<PUSH, false>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+}
+
+template <bool PUSH, bool EDGE>
+__device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint64_t* empty, float* __restrict__ uout,
+                                        int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
+                                        int lane, int warp, const PushList& push) {
+    const int cx = 4 * lane;                          // smem column of the lane's first column
+    const int64_t col0 = c0 - 4 + cx;                 // its grid column
+    const bool wclamp = col0 == 0, eclamp = col0 + 4 >= W;
+    const bool store_col = lane >= 1 && lane <= 30 && col0 < W;
+    const int64_t gr1 = y0 + kRW * warp - 1;          // grid row of sweep-1 row j = 0
+    const int br1 = kRW * warp + 1;                   // box row of sweep-1 row j = 0
+    const int64_t HW = H * W;
+    float4 L1[3][kL1];                                // sweep-1 window, slot = plane sequence mod 3
+    ptx::mbar_wait(&full[0], 0);
+    ptx::mbar_wait(&full[1], 0);
+    for (int q0 = 2; q0 < nq; q0 += 3) {
+#pragma unroll
+        for (int u = 0; u < 3; ++u) {
+            const int q = q0 + u;                     // q == 2 + u (mod 3)
+            if (q >= nq) break;
+            ptx::mbar_wait(&full[q % kNS], (uint32_t)((q / kNS) & 1));
+            const float* sm = ring + (size_t)((q - 2) % kNS) * kSlot;   // plane seq q-2
+            const float* sc = ring + (size_t)((q - 1) % kNS) * kSlot;   // plane seq q-1
+            const float* sp = ring + (size_t)(q % kNS) * kSlot;         // plane seq q
+            // sweep 1 on plane seq q-1, rows j = 0..5 (grid rows gr1 + j)
+            float4 up = *reinterpret_cast<const float4*>(sc + (br1 - 1) * kCols + cx);
+            float4 cc = *reinterpret_cast<const float4*>(sc + br1 * kCols + cx);
+            const int s1 = (2 + u - 1 + 3) % 3;       // slot of plane seq q-1 (constant after unrolling)
+#pragma unroll
+            for (int j = 0; j < kL1; ++j) {
+                const int br = br1 + j;
+                const int64_t gr = gr1 + j;
+                const float4 dn = *reinterpret_cast<const float4*>(sc + (br + 1) * kCols + cx);
+                const float4 zm = *reinterpret_cast<const float4*>(sm + br * kCols + cx);
+                const float4 zp = *reinterpret_cast<const float4*>(sp + br * kCols + cx);
+                const float4 ym = (EDGE && gr == 0) ? cc : up;        // replicate clamp (TMA zero-filled row -1)
+                const float4 yp = (EDGE && gr == H - 1) ? cc : dn;    // ... and row H
+                L1[s1][j] = sweep(cc, zm, zp, ym, yp, wclamp, eclamp);
+                up = cc;
+                cc = dn;
+            }
+            // sweep 2 on plane seq q-2 = grid plane k0 + q - 4, own rows j = 1..4
+            if (q >= 4) {
+                const int s0 = (2 + u - 2 + 3) % 3, sM = (2 + u - 3 + 3) % 3;
+                const int64_t pz = k0 + q - 4;
+                const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == D - 1;   // sweep-1 planes outside: clamp
+                float* outp = uout + pz * HW + (y0 + kRW * warp) * W + col0;
+#pragma unroll
+                for (int j = 1; j <= kRW; ++j) {
+                    const int64_t gr = gr1 + j;
+                    const float4 c = L1[s0][j];
+                    const float4 zm = zlo ? c : L1[sM][j];
+                    const float4 zp = zhi ? c : L1[s1][j];
+                    const float4 ym = (EDGE && gr == 0) ? c : L1[s0][j - 1];
+                    const float4 yp = (EDGE && gr == H - 1) ? c : L1[s0][j + 1];
+                    const float4 o = sweep(c, zm, zp, ym, yp, wclamp, eclamp);
+                    if (store_col && gr < H) {
+                        *reinterpret_cast<float4*>(outp) = o;
+                        if (PUSH) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);  // fused halo push
+                    }
+                    outp += W;
+                }
+            }
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&empty[(q - 2) % kNS]);   // plane seq q-2 fully read
+        }
+    }
+    __syncwarp();
+    if (lane == 0) {
+        ptx::mbar_arrive(&empty[(nq - 2) % kNS]);
+        ptx::mbar_arrive(&empty[(nq - 1) % kNS]);
+    }
+}
+
+int describe_heat3d_tb2(pk_ctx c, pk_kernel k) {
+    // scalars: 0 = D, 1 = H, 2 = W, 3 = ZC.  Logical block (bx, by, bz) = columns
+    // [120 bx, +120) x rows [24 by, +24) x planes [ZC bz, +ZC), guarded.  Reads the
+    // clamped 5x5x5 cube around every cell (the box dilated by 2 in every dimension:
+    // one tap, positions [b*scale, b*scale + extent + 4) with the guard shifted by 4,
+    // offset -2, clamped; corners included -- a read over-approximation);
+    // writes its own cells.
+    const uint32_t f = PK_DIM_GUARD | PK_DIM_CLAMP;
+    pk_affine_access a{};
+    a.ndim = 3;
+    a.dim[0] = DimMap(2, S(3), S(3, 1, 4), E(-2), f, E(0), S(0, 1, 4));
+    a.dim[1] = DimMap(1, E(kRows), E(kRows + 4), E(-2), f, E(0), S(1, 1, 4));
+    a.dim[2] = DimMap(0, E(kOwnC), E(kOwnC + 4), E(-2), f, E(0), S(2, 1, 4));
+    if (int r = pk_declare_affine_access(c, k, 0, PK_READ, &a)) return r;
+    pk_affine_access w{};
+    w.ndim = 3;
+    w.dim[0] = DimMap(2, S(3), S(3), E(0), f, E(0), S(0));
+    w.dim[1] = DimMap(1, E(kRows), E(kRows), E(0), f, E(0), S(1));
+    w.dim[2] = DimMap(0, E(kOwnC), E(kOwnC), E(0), f, E(0), S(2));
+    return pk_declare_affine_access(c, k, 1, PK_WRITE, &w);
+}
+
+cudaError_t launch_heat3d_tb2(const LaunchInfo& li) {
+    if (li.nscalars < 4) return cudaErrorInvalidValue;
+    int64_t D = li.scalars[0], H = li.scalars[1], W = li.scalars[2], ZC = li.scalars[3];
+    if (W % 4 || W < 4 || ZC < 1 || H < 1 || D < 1) return cudaErrorInvalidValue;
+    static std::once_flag once;
+    static cudaError_t attr_err = cudaSuccess;
+    std::call_once(once, [] {
+        attr_err = cudaFuncSetAttribute(k_heat3d_tb2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
+        if (attr_err == cudaSuccess)
+            attr_err = cudaFuncSetAttribute(k_heat3d_tb2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
+    });
+    if (attr_err != cudaSuccess) return attr_err;
+    // tensor map of this instance: dims (W, H, D), box (128, 28, 1), OOB zero fill
+    static std::mutex mu;
+    static std::unordered_map<const void*, std::pair<uint64_t, CUtensorMap>> cache;
+    CUtensorMap tm;
+    {
+        std::lock_guard<std::mutex> g(mu);
+        const uint64_t key = ((uint64_t)W * 1315423911ull) ^ ((uint64_t)H << 20) ^ ((uint64_t)D << 40);
+        auto it = cache.find(li.inst[0]);
+        if (it != cache.end() && it->second.first == key) {
+            tm = it->second.second;
+        } else {
+            cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)D};
+            cuuint32_t box[3] = {(cuuint32_t)kCols, (cuuint32_t)kBoxRows, 1};
+            if (!tma_encode_f32(&tm, li.inst[0], 3, dims, box, CU_TENSOR_MAP_SWIZZLE_NONE))
+                return cudaErrorInvalidValue;
+            cache[li.inst[0]] = {key, tm};
+        }
+    }
+    PushList pl{};
+    if (li.push) pl = *li.push;
+    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, (void*)&li.part, &pl};
+    const void* fn = (li.push && li.push->n > 0) ? (const void*)k_heat3d_tb2<true> : (const void*)k_heat3d_tb2<false>;
+    return cudaLaunchKernel(fn, li.grid, dim3((kNW + 1) * 32), argv, kSmem, li.stream);
+}
+
+}  // namespace
+
+const Builtin kBuiltinHeat3dTb2 = {
+    "heat3d_tb2", (const void*)k_heat3d_tb2<false>, 6,
+    {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
+    describe_heat3d_tb2, launch_heat3d_tb2, /*push_arg=*/1};
+
+}  // namespace pk

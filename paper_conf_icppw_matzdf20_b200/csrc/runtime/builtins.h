@@ -60,6 +60,7 @@ extern const Builtin kBuiltinHotspot2dTb2;  // hotspot2d_tb2 (two sweeps per lau
 extern const Builtin kBuiltinHotspot2dTbk;  // hotspot2d_tbk (K = 2..4 sweeps per launch, scalar 3)
 extern const Builtin kBuiltinHeat3d;
 extern const Builtin kBuiltinHeat3dTma;      // heat3d (TMA plane ring, default); kBuiltinHeat3d = heat3d_regs
+extern const Builtin kBuiltinHeat3dTb2;      // heat3d_tb2 (two sweeps per launch)
 extern const Builtin kBuiltinNbody;
 extern const Builtin kBuiltinSgemm;          // sgemm_tf32x3 (tcgen05 3xTF32)
 

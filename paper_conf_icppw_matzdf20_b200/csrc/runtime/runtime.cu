@@ -2042,7 +2042,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
 namespace pk {
 int32_t find_builtin_push_arg(const void* fn) {
     if (!fn) return -1;
-    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_tbk", "heat3d"}) {
+    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_tbk", "heat3d", "heat3d_tb2"}) {
         const Builtin* b = find_builtin(n);
         if (b && b->fn == fn) return b->push_arg;
     }
@@ -2050,7 +2050,7 @@ int32_t find_builtin_push_arg(const void* fn) {
 }
 LauncherFn find_builtin_launcher(const void* fn) {
     if (!fn) return nullptr;
-    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk", "heat3d", "heat3d_regs",
+    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk", "heat3d", "heat3d_regs", "heat3d_tb2",
                           "nbody", "sgemm_tf32x3"}) {
         const Builtin* b = find_builtin(n);
         if (b && b->fn == fn) return b->launcher;
@@ -2060,7 +2060,8 @@ LauncherFn find_builtin_launcher(const void* fn) {
 const Builtin* find_builtin(const char* name) {
     if (!name) return nullptr;
     static const Builtin* all[] = {&kBuiltinJacobi2d, &kBuiltinHotspot2dTma, &kBuiltinHotspot2d, &kBuiltinHotspot2dTb2,
-                                   &kBuiltinHotspot2dTbk, &kBuiltinHeat3dTma, &kBuiltinHeat3d, &kBuiltinNbody, &kBuiltinSgemm};
+                                   &kBuiltinHotspot2dTbk, &kBuiltinHeat3dTma, &kBuiltinHeat3d, &kBuiltinHeat3dTb2, &kBuiltinNbody,
+                                   &kBuiltinSgemm};
     for (const Builtin* b : all)
         if (std::strcmp(b->name, name) == 0) return b;
     return nullptr;

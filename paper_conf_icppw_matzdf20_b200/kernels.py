@@ -44,6 +44,14 @@ def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
     return (_cdiv(w, 128), _cdiv(h, bdy), _cdiv(d, zc)), (32, bdy, 1), [d, h, w, zc]
 
 
+HEAT_TB2_COLS, HEAT_TB2_ROWS = 120, 24    # "heat3d_tb2": owned columns x rows per logical block
+
+
+def heat3d_tb2_launch(d, h, w, zc=HEAT_ZC):
+    """Logical block = 120 columns x 24 rows x zc planes, two sweeps per launch."""
+    return (_cdiv(w, HEAT_TB2_COLS), _cdiv(h, HEAT_TB2_ROWS), _cdiv(d, zc)), (224, 1, 1), [d, h, w, zc]
+
+
 def nbody_launch(n, bdx=NBODY_BDX):
     return (_cdiv(n, NBODY_PER_THREAD * bdx), 1, 1), (bdx, 1, 1), [n]
 
@@ -141,23 +149,29 @@ def hotspot2d_iterate(pr, iters, start=0):
 
 
 def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY, kernel="heat3d", tiles=None):
+    """kernel: heat3d (one sweep per launch, TMA ring), heat3d_regs, heat3d_tb2 (two)."""
     d, h, w = u_host.shape
     pr = Problem(ctx, kernel, tiles)
     u0 = pr.buffer((d, h, w), 4, host=u_host)
     u1 = pr.buffer((d, h, w), 4)
-    pr.geom = heat3d_launch(d, h, w, zc, bdy)
+    pr.geom = heat3d_tb2_launch(d, h, w, zc) if kernel == "heat3d_tb2" else heat3d_launch(d, h, w, zc, bdy)
     pr.shape = (d, h, w)
     pr.ub = (u0, u1)
+    pr.sweeps = 2 if kernel == "heat3d_tb2" else 1
     return pr
 
 
 def heat3d_iterate(pr, iters, start=0):
+    """`iters` sweeps from sweep `start` (multiples of pr.sweeps for heat3d_tb2)."""
     (u0, u1), (d, h, w) = pr.ub, pr.shape
     grid, blk, sc = pr.geom
-    for t in range(start, start + iters):
+    k = pr.sweeps
+    if iters % k or start % k:
+        raise ValueError(f"this kernel advances {k} steps per launch")
+    for t in range(start // k, (start + iters) // k):
         a, b = (u0, u1) if t % 2 == 0 else (u1, u0)
         pr.launch(grid, blk, [a, b, d, h, w, sc[3]], sc)
-    return u1 if (start + iters) % 2 == 1 else u0
+    return u1 if ((start + iters) // k) % 2 == 1 else u0
 
 
 def nbody_setup(ctx, pos_host, vel_host, bdx=NBODY_BDX):

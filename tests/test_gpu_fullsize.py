@@ -72,18 +72,20 @@ def test_c2_hotspot_fullsize_tbk_sampled():
 
 
 # ------------------------------------------------------------------ C3 Heat 1024^3, 50 it
-def test_c3_heat_fullsize_sampled():
+@pytest.mark.parametrize("kernel", ["heat3d_tb2", "heat3d"])
+def test_c3_heat_fullsize_sampled(kernel):
+    """heat3d_tb2 (bench default: 25 launches of two sweeps, ZC = 128) and heat3d (one sweep)."""
     d = h = w = 1024
     iters = 50
     u = synth.heat_grid(d, h, w)
     res = {}
     for P in (1, 2):
         ctx = gpu_ctx(P)
-        pr = K.heat3d_setup(ctx, u)                      # bench config: ZC = 128, bdy = 62
+        pr = K.heat3d_setup(ctx, u, kernel=kernel)       # bench config: ZC = 128 (heat3d: bdy = 62)
         res[P] = fetch(ctx, K.heat3d_iterate(pr, iters), (d, h, w))
         st = abi.pk_get_stats(ctx)
         abi.pk_finalize(ctx)
-        if P > 1:
+        if P > 1:   # one halo plane per sweep each way per cut (two per launch for tb2)
             assert st["stale_bytes"] == st["moved_bytes"] == iters * 2 * h * w * 4 * (P - 1)
     assert np.array_equal(res[1], res[2])
     g = res[1]

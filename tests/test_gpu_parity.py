@@ -524,3 +524,37 @@ def test_push_heat_and_jacobi_bitwise(P):
     assert np.array_equal(j1, jp)
     if P == 2:   # C1: 2 x 4,080 B pulled instead of 40,800 B, the rest pushed
         assert st["stale_bytes"] == 8160 and st["pushed_bytes"] == 9 * 4080
+
+
+
+# ------------------------------------------------------------------ two-sweep heat (NEXT-3, 3-D)
+@pytest.mark.parametrize("d,h,w,zc", [(40, 36, 132, 8), (17, 9, 256, 4), (9, 70, 260, 3), (30, 50, 124, 128),
+                                      (5, 3, 4, 2)])
+def test_heat3d_tb2_oracle_and_bitwise(d, h, w, zc):
+    u = synth.heat_grid(d, h, w)
+    iters = 6
+    ref = ok.heat3d(u, iters)
+    g1, s1 = _heat_tb2(u, iters, 1, zc)
+    ok_, err = rel_ok(g1, ref, 1e-5)
+    assert ok_, err
+    assert s1["kernel_launches"] == iters // 2
+    for P in (2, 3, 5):
+        gp, st = _heat_tb2(u, iters, P, zc)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def _heat_tb2(u, iters, P, zc, mode=0):
+    ctx = gpu_ctx(P, mode)
+    pr = K.heat3d_setup(ctx, u, zc, kernel="heat3d_tb2")
+    res = fetch(ctx, K.heat3d_iterate(pr, iters), u.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st
+
+
+def test_heat3d_tb2_push_bitwise():
+    u = synth.heat_grid(40, 36, 132)
+    r1, _ = _heat_tb2(u, 8, 1, 8)
+    rp, st = _heat_tb2(u, 8, 3, 8, abi.PK_MODE_PUSH)
+    assert np.array_equal(r1, rp) and st["pushed_bytes"] > 0

@@ -623,3 +623,20 @@ def test_push_tiles_fall_back_to_pull():
                        lambda box: regions.jacobi2d(box, geom[1], n, n), mode=abi.PK_MODE_PUSH, push_arg=1,
                        tiles=(2, 2, 1))
     assert st_["pushed_bytes"] == 0
+
+
+# ------------------------------------------------------------ two-sweep heat (NEXT-3, 3-D)
+@pytest.mark.parametrize("d,h,w,zc", [(10, 30, 260, 4), (7, 50, 124, 128), (3, 5, 8, 2)])
+@pytest.mark.parametrize("P", [1, 2, 3, 5])
+def test_heat3d_tb2_regions(d, h, w, zc, P):
+    """One dilated tap == brute-force clamped 5x5x5 cubes of every owned cell."""
+    ctx = host_ctx(P)
+    kk = abi.pk_builtin_kernel(ctx, "heat3d_tb2")
+    bufs = [abi.pk_register_buffer(ctx, (d, h, w), 4) for _ in range(2)]
+    grid, blk, sc = K.heat3d_tb2_launch(d, h, w, zc)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, kk, grid, p)
+        lib = _lib_sets(ctx, kk, 6, bufs + [None] * 4, box, blk, sc)
+        ora = _oracle_sets(regions.heat3d_tb2(box, d, h, w, zc), {0: 4, 1: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
