@@ -360,7 +360,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
-    ap.add_argument("--sweeps", type=int, default=4, help="time steps per launch of --variant hotspot2d_tbk (2..4)")
+    ap.add_argument("--sweeps", type=int, default=4, help="time steps per launch of hotspot2d_tbk (2..8; iterations must be a multiple)")
     ap.add_argument("--tile", type=int, default=0, help="rows per block (hotspot2d TY) / planes per block (heat3d ZC)")
     ap.add_argument("--tiles", default=None,
                     help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")

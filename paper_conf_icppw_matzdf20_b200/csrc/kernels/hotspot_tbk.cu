@@ -1,4 +1,4 @@
-// hotspot_tbk.cu -- C2 Hotspot, temporally blocked to depth K (2..4): K time steps
+// hotspot_tbk.cu -- C2 Hotspot, temporally blocked to depth K (2..8): K time steps
 // per launch ("halo width h per launch": the Rodinia
 // benchmark the paper runs is itself pyramid-blocked).
 //
@@ -16,9 +16,10 @@
 // in registers (slot = row sequence mod 3, so the 3-fold unrolled loop needs no
 // register moves): per input row it loads one new temp row, computes level k at
 // row sequence t-k for k = 1..K (power from the ring) and stores level K.  W/E neighbours are warp shuffles.
-// Warps overlap: a warp covers 128 columns, but its lanes 0 and 31 are halo lanes
-// whose values are wrong in their outer k columns after k sweeps (k <= 4), so
-// only lanes 1..30 store: 120 owned columns per warp, 480 per tile.  Consumers
+// Warps overlap: a warp covers 128 columns, but its HL = ceil(K/4) outermost lanes
+// on each side are halo lanes (a lane holds 4 columns; the shuffle wrap corrupts
+// one more column per sweep), so only lanes HL..31-HL store: 120 owned columns per
+// warp and 480 per tile for K <= 4, 112 and 448 for K = 5..8.  Consumers
 // therefore never synchronise with each other, only with the ring.  Halo rows and
 // columns are recomputed redundantly from identical inputs in identical operation
 // order, so P-way launches are bit-identical to 1-way.
@@ -26,7 +27,15 @@
 // Arithmetic per cell and sweep (6 FP32 ops, fixed order):
 //   T' = c*A + (((n + s) + e) + w)*B + (p*kCap + D)
 // with A = 1 - kCap(2 Ry1 + 2 Rx1 + Rz1), B = kCap Ry1 (Rx1 == Ry1), D = kCap Rz1 amb:
-// the Rodinia update of reading Q14 with its constant terms folded.
+// the Rodinia update of reading Q14 with its constant terms folded.  (Measured and
+// rejected: the order s*B + ((n + e) + w)*B + ..., which leaves only the last FMA
+// on the level chain -- equal speed at K = 4 within noise, more registers.)
+//
+// Depth: K = 2..8 are instantiated; K = 4 is the bench default.  K > 4 needs two
+// halo lanes per side and ~170 registers (2 CTAs/SM): measured on C2 at 96
+// sweeps, K = 4 / 6 / 8: 1977 / 1432 / 1270 GLUP/s -- beyond K = 4 the kernel is
+// bound by the K-level dependency chain per row at 8 consumer warps per SM, not by
+// HBM (0.44 / 0.29 of the measured HBM roof), so deeper blocking does not pay here.
 #include <cuda_runtime.h>
 
 #include "../runtime/builtins.h"
@@ -45,19 +54,26 @@ constexpr float kB = (float)(kCapD * kR1D);
 constexpr float kCap = (float)kCapD;
 constexpr float kD = (float)(kCapD * kRz1D * kAmbD);
 
-constexpr int kOwn = 120;                 // owned columns per warp (lanes 1..30)
-constexpr int kTC = 4 * kOwn;             // owned columns per tile (4 consumer warps)
-constexpr int kRowF = kTC + 8;            // row segment: [c0-4, c0+484)
-constexpr int kStageFloats = 2 * kRowF;   // temp + power
-constexpr int kStageBytes = kStageFloats * 4;
+// per-depth geometry: HL halo lanes per side, owned columns per warp / tile, row
+// segment [c0 - 4 HL, c0 + TC + 4 HL) of temp (then power) per ring stage
+template <int K>
+struct Geo {
+    static constexpr int HL = (K + 3) / 4;
+    static constexpr int Own = (32 - 2 * HL) * 4;
+    static constexpr int TC = 4 * Own;
+    static constexpr int RowF = TC + 8 * HL;
+    static constexpr int StageFloats = 2 * RowF;
+    static constexpr int StageBytes = StageFloats * 4;
+};
 #ifndef PK_TBK_NS
 #define PK_TBK_NS 16
 #endif
 constexpr int kNS = PK_TBK_NS;            // ring depth (power of two)
-static_assert((kNS & (kNS - 1)) == 0 && kNS >= 8, "ring holds K+1 <= 5 rows plus prefetch");
+static_assert((kNS & (kNS - 1)) == 0 && kNS >= 16, "ring holds K+1 <= 9 rows plus prefetch");
 constexpr int kConsumers = 128;
 constexpr int kThreads = kConsumers + 32;
-constexpr size_t kSmem = (size_t)kNS * kStageBytes + 2 * kNS * sizeof(uint64_t);
+template <int K>
+constexpr size_t smem_bytes() { return (size_t)kNS * Geo<K>::StageBytes + 2 * kNS * sizeof(uint64_t); }
 
 __device__ __forceinline__ float upd(float c, float n, float s, float e, float w, float p) {
     return fmaf(c, kA, fmaf(((n + s) + e) + w, kB, fmaf(p, kCap, kD)));
@@ -92,17 +108,18 @@ template <int K, bool EDGE, bool COLEDGE, bool PUSH>
 __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, uint64_t* empty, float* tout,
                                              int64_t W, int H, int64_t c0, int64_t r0, int64_t rend, bool down,
                                              uint32_t g, int lane, int warp, const PushList& push) {
+    using G = Geo<K>;
     constexpr int kW3 = 3;
-    const int scol = kOwn * warp + 4 * lane;
-    const int64_t col0 = c0 - 4 + scol;
-    const bool store = lane >= 1 && lane <= 30 && col0 < W;
+    const int scol = G::Own * warp + 4 * lane;
+    const int64_t col0 = c0 - 4 * G::HL + scol;
+    const bool store = lane >= G::HL && lane <= 31 - G::HL && col0 < W;
     const bool wclamp = col0 == 0, eclamp = col0 + 4 >= W;
     const int nr = (int)(rend - r0), nt = nr + 2 * K;
     const int dir = down ? 1 : -1;
     const int base = (int)(down ? r0 - K : rend - 1 + K);
     float4 in[kW3];
     float4 L[K > 1 ? K - 1 : 1][kW3];
-    auto stage = [&](int seq) { return ring + (size_t)((g + (uint32_t)seq) & (kNS - 1)) * kStageFloats; };
+    auto stage = [&](int seq) { return ring + (size_t)((g + (uint32_t)seq) & (kNS - 1)) * G::StageFloats; };
     ptx::mbar_wait(&full[g & (kNS - 1)], (g / kNS) & 1u);
     in[0] = *reinterpret_cast<const float4*>(stage(0) + scol);
     ptx::mbar_wait(&full[(g + 1) & (kNS - 1)], ((g + 1) / kNS) & 1u);
@@ -123,7 +140,7 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
                 const int sn = (2 + u - k - 1 + kW3 * K) % kW3;
                 const int ss = (2 + u - k + 1 + kW3 * K) % kW3;
                 const float4* prev = k == 1 ? in : L[k - 2 < 0 ? 0 : k - 2];
-                const float4 p = *reinterpret_cast<const float4*>(stage(t - k) + kRowF + scol);
+                const float4 p = *reinterpret_cast<const float4*>(stage(t - k) + G::RowF + scol);
                 float4 n4 = prev[sn], s4 = prev[ss];
                 if (EDGE && k > 1) {
                     const int R = base + dir * (t - k);
@@ -152,14 +169,18 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
 #ifndef PK_TBK_MINB
 #define PK_TBK_MINB 3
 #endif
+#ifndef PK_TBK8_MINB
+#define PK_TBK8_MINB 2
+#endif
 template <int K, bool PUSH>
-__global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const float* __restrict__ tin,
+__global__ void __launch_bounds__(kThreads, K <= 4 ? PK_TBK_MINB : PK_TBK8_MINB) k_hotspot2d_tbk(const float* __restrict__ tin,
                                                             const float* __restrict__ pw,
                                                             float* __restrict__ tout, int64_t H, int64_t W,
                                                             int64_t TY, pk_partition part, PushList push) {
+    using G = Geo<K>;
     extern __shared__ __align__(128) unsigned char smem[];
     float* ring = reinterpret_cast<float*>(smem);
-    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)kNS * kStageFloats);
+    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)kNS * G::StageFloats);
     uint64_t* empty = full + kNS;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
@@ -178,20 +199,20 @@ __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const f
         uint32_t g = 0;
         for (int64_t T = blockIdx.x; T < ntiles; T += gridDim.x) {
             const int64_t bx = part.min[0] + T % gx, by = part.min[1] + T / gx;  // Eq. 8
-            const int64_t c0 = bx * kTC, r0 = by * TY, rend = min(r0 + TY, H), nr = rend - r0;
+            const int64_t c0 = bx * G::TC, r0 = by * TY, rend = min(r0 + TY, H), nr = rend - r0;
             const bool down = (by & 1) == 0;
-            const int64_t tlo = max(c0 - 4, (int64_t)0), thi = min(c0 + kTC + 4, W);
+            const int64_t tlo = max(c0 - 4 * G::HL, (int64_t)0), thi = min(c0 + G::TC + 4 * G::HL, W);
             const uint32_t bytes = (uint32_t)(thi - tlo) * 4u;
-            const int64_t toff = tlo - (c0 - 4);
+            const int64_t toff = tlo - (c0 - 4 * G::HL);
             for (int64_t t = 0; t < nr + 2 * K; ++t, ++g) {
                 const uint32_t s = g % kNS, par = (g / kNS) & 1u;
                 ptx::mbar_wait(&empty[s], par ^ 1u);
                 int64_t row = down ? r0 - K + t : rend - 1 + K - t;
                 row = row < 0 ? 0 : (row >= H ? H - 1 : row);
-                float* st = ring + (size_t)s * kStageFloats;
+                float* st = ring + (size_t)s * G::StageFloats;
                 ptx::mbar_arrive_expect_tx(&full[s], 2u * bytes);
                 ptx::bulk_g2s(st + toff, tin + row * W + tlo, bytes, &full[s]);
-                ptx::bulk_g2s(st + kRowF + toff, pw + row * W + tlo, bytes, &full[s]);
+                ptx::bulk_g2s(st + G::RowF + toff, pw + row * W + tlo, bytes, &full[s]);
             }
         }
         return;
@@ -200,11 +221,11 @@ __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const f
     uint32_t g = 0;
     for (int64_t T = blockIdx.x; T < ntiles; T += gridDim.x) {
         const int64_t bx = part.min[0] + T % gx, by = part.min[1] + T / gx;
-        const int64_t c0 = bx * kTC, r0 = by * TY, rend = min(r0 + TY, H);
+        const int64_t c0 = bx * G::TC, r0 = by * TY, rend = min(r0 + TY, H);
         const bool down = (by & 1) == 0;
         // tiles whose (dilated) rows reach the grid's first/last row need the clamp selects
         const bool redge = r0 < K + 1 || rend + K + 1 > H;
-        const bool cedge = c0 == 0 || c0 + kTC + 4 >= W;
+        const bool cedge = c0 == 0 || c0 + G::TC + 4 * G::HL >= W;
         if (redge || cedge)
             consume_tile<K, true, true, PUSH>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp,
                                               push);
@@ -216,8 +237,9 @@ __global__ void __launch_bounds__(kThreads, PK_TBK_MINB) k_hotspot2d_tbk(const f
 }
 
 int describe_hotspot2d_tbk(pk_ctx c, pk_kernel k) {
-    // scalars: 0 = H, 1 = W, 2 = TY, 3 = K.  Logical block (bx, by) = rows [by*TY, +TY)
-    // x columns [480 bx, +480), guarded.  Reads the clamped (2K+1)^2 square of temp
+    // scalars: 0 = H, 1 = W, 2 = TY, 3 = K, 4 = TC (owned columns per logical block:
+    // 480 for K <= 4, 448 for K = 5..8, checked by the launcher).  Logical block
+    // (bx, by) = rows [by*TY, +TY) x columns [TC bx, +TC), guarded.  Reads the clamped (2K+1)^2 square of temp
     // (the dilated box: one tap, exact union of the shifted boxes; corners included,
     // a read over-approximation) and the (2K-1)^2 square of power; writes
     // its own cells.  Positions are taken in [b*scale, b*scale + extent + 2K) with the
@@ -229,7 +251,7 @@ int describe_hotspot2d_tbk(pk_ctx c, pk_kernel k) {
     a.dim[0] = DimMap(1, S(2), S(2, 1), S(3, -1), f, E(0), S(0));
     a.dim[0].extent.c_scalar[3] = 2;   // TY + 2K
     a.dim[0].guard_hi.c_scalar[3] = 2; // H + 2K
-    a.dim[1] = DimMap(0, E(kTC), E(kTC), S(3, -1), f, E(0), S(1));
+    a.dim[1] = DimMap(0, S(4), S(4), S(3, -1), f, E(0), S(1));
     a.dim[1].extent.c_scalar[3] = 2;
     a.dim[1].guard_hi.c_scalar[3] = 2;
     if (int r = pk_declare_affine_access(c, k, 0, PK_READ, &a)) return r;
@@ -244,7 +266,7 @@ int describe_hotspot2d_tbk(pk_ctx c, pk_kernel k) {
     pk_affine_access w{};
     w.ndim = 2;
     w.dim[0] = DimMap(1, S(2), S(2), E(0), f, E(0), S(0));
-    w.dim[1] = DimMap(0, E(kTC), E(kTC), E(0), f, E(0), S(1));
+    w.dim[1] = DimMap(0, S(4), S(4), E(0), f, E(0), S(1));
     return pk_declare_affine_access(c, k, 2, PK_WRITE, &w);
 }
 
@@ -253,6 +275,7 @@ cudaError_t launch_k(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
     static int resident[64] = {0};
     static int sms[64] = {0};
     const int d = li.device;
+    constexpr size_t kSmem = smem_bytes<K>();
     if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
     if (!resident[d]) {
         cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tbk<K, PUSH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -276,16 +299,20 @@ cudaError_t launch_k(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
 }
 
 cudaError_t launch_hotspot2d_tbk(const LaunchInfo& li) {
-    if (li.nscalars < 4) return cudaErrorInvalidValue;
-    const int64_t H = li.scalars[0], W = li.scalars[1], TY = li.scalars[2], K = li.scalars[3];
+    if (li.nscalars < 5) return cudaErrorInvalidValue;
+    const int64_t H = li.scalars[0], W = li.scalars[1], TY = li.scalars[2], K = li.scalars[3], TC = li.scalars[4];
     if (W % 4 || W < 4 || TY < 1 || H < 1 || H > (1ll << 30) || li.block.x != kConsumers || li.block.y != 1 ||
-        li.block.z != 1)
+        li.block.z != 1 || TC != (K <= 4 ? Geo<4>::TC : Geo<8>::TC))
         return cudaErrorInvalidValue;
     const bool push = li.push && li.push->n > 0;
     switch (K) {
         case 2: return push ? launch_k<2, true>(li, H, W, TY) : launch_k<2, false>(li, H, W, TY);
         case 3: return push ? launch_k<3, true>(li, H, W, TY) : launch_k<3, false>(li, H, W, TY);
         case 4: return push ? launch_k<4, true>(li, H, W, TY) : launch_k<4, false>(li, H, W, TY);
+        case 5: return push ? launch_k<5, true>(li, H, W, TY) : launch_k<5, false>(li, H, W, TY);
+        case 6: return push ? launch_k<6, true>(li, H, W, TY) : launch_k<6, false>(li, H, W, TY);
+        case 7: return push ? launch_k<7, true>(li, H, W, TY) : launch_k<7, false>(li, H, W, TY);
+        case 8: return push ? launch_k<8, true>(li, H, W, TY) : launch_k<8, false>(li, H, W, TY);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -32,12 +32,19 @@ def hotspot2d_launch(h, w, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX):
     return (_cdiv(w, 4 * bdx), _cdiv(h, ty), 1), (bdx, 1, 1), [h, w, ty]
 
 
-TBK_COLS = 480                         # "hotspot2d_tbk": owned columns per logical block
+def tbk_cols(k):
+    """"hotspot2d_tbk": owned columns per logical block (one halo lane per warp side
+    for K <= 4 sweeps, two for K = 5..8)."""
+    return 480 if k <= 4 else 448
+
+
+TBK_COLS = tbk_cols(4)
 
 
 def hotspot2d_tbk_launch(h, w, ty=HOTSPOT_TY, k=4):
-    """Logical block = 480 columns x ty rows, k sweeps per launch (scalar 3)."""
-    return (_cdiv(w, TBK_COLS), _cdiv(h, ty), 1), (128, 1, 1), [h, w, ty, k]
+    """Logical block = tbk_cols(k) columns x ty rows, k sweeps per launch (scalar 3,
+    K in 2, 3, 4, 6, 8); scalar 4 = the block's column count."""
+    return (_cdiv(w, tbk_cols(k)), _cdiv(h, ty), 1), (128, 1, 1), [h, w, ty, k, tbk_cols(k)]
 
 
 def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
@@ -118,7 +125,7 @@ def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None):
 def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None,
                     kernel="hotspot2d", tiles=None, sweeps=4):
     """kernel: hotspot2d (one sweep per launch), hotspot2d_regs, hotspot2d_tb2 (two),
-    hotspot2d_tbk (`sweeps` = 2..4 per launch)."""
+    hotspot2d_tbk (`sweeps` = 2, 3, 4, 6 or 8 per launch)."""
     h, w = temp_host.shape
     pr = Problem(ctx, kernel, tiles)
     t0 = pr.buffer((h, w), 4, host=temp_host, dev_ptrs=dev_ptrs[0] if dev_ptrs else None)

@@ -123,11 +123,12 @@ def test_hotspot_tb2_oracle_and_bitwise(h, w, ty):
 
 
 @pytest.mark.parametrize("h,w,ty,k", [(200, 520, 16, 4), (129, 1028, 64, 3), (3, 4, 64, 2), (300, 2048, 7, 4),
-                                      (64, 1536, 128, 4), (40, 960, 5, 2), (257, 964, 32, 3)])
+                                      (64, 1536, 128, 4), (40, 960, 5, 2), (257, 964, 32, 3),
+                                      (300, 2048, 32, 6), (131, 900, 16, 8), (70, 452, 9, 5), (64, 1348, 40, 7)])
 def test_hotspot_tbk_oracle_and_bitwise(h, w, ty, k):
-    """K fused sweeps per launch (NEXT-3, K = 2..4): oracle within 1e-5, P-way bit-identical."""
+    """K fused sweeps per launch (NEXT-3, K = 2..8): oracle within 1e-5, P-way bit-identical."""
     t, p = synth.hotspot_grids(h, w)
-    iters = 12
+    iters = 12 if 12 % k == 0 else 2 * k
     ref = ok.hotspot2d(t, p, iters)
     g1, s1 = _hotspot_k(t, p, iters, 1, ty, k)
     ok_, err = rel_ok(g1, ref, 1e-5)

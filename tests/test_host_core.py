@@ -543,10 +543,12 @@ def test_hotspot_tb2_regions(h, w, ty, P):
     abi.pk_finalize(ctx)
 
 
-@pytest.mark.parametrize("h,w,ty,k", [(33, 1100, 4, 4), (200, 1028, 16, 3), (5, 8, 64, 2), (40, 960, 7, 4)])
+@pytest.mark.parametrize("h,w,ty,k", [(33, 1100, 4, 4), (200, 1028, 16, 3), (5, 8, 64, 2), (40, 960, 7, 4),
+                                      (41, 1000, 9, 6), (70, 900, 16, 8), (20, 452, 5, 5)])
 @pytest.mark.parametrize("P", [1, 2, 3, 7])
 def test_hotspot_tbk_regions(h, w, ty, k, P):
-    """K-sweep Hotspot: one dilated tap per argument == brute-force (2K+1)^2 / (2K-1)^2 squares."""
+    """K-sweep Hotspot: one dilated tap per argument == brute-force (2K+1)^2 / (2K-1)^2 squares
+    (logical blocks 480 columns wide for K <= 4, 448 for K = 5..8)."""
     ctx = host_ctx(P)
     kk = abi.pk_builtin_kernel(ctx, "hotspot2d_tbk")
     bufs = [abi.pk_register_buffer(ctx, (h, w), 4) for _ in range(3)]
@@ -554,7 +556,8 @@ def test_hotspot_tbk_regions(h, w, ty, k, P):
     for p in range(P):
         box = abi.pk_partition_grid(ctx, kk, grid, p)
         lib = _lib_sets(ctx, kk, 6, bufs + [None] * 3, box, blk, sc)
-        ora = _oracle_sets(regions.hotspot2d_tbk(box, blk, h, w, ty, k), {0: 4, 1: 4, 2: 4})
+        ora = _oracle_sets(regions.hotspot2d_tbk(box, blk, h, w, ty, k, cols=480 if k <= 4 else 448),
+                           {0: 4, 1: 4, 2: 4})
         assert lib == ora
     abi.pk_finalize(ctx)
 
