@@ -191,7 +191,7 @@ class Workload:
             self.bytes_per_unit = 12 / self.sweeps
             self.upload_bufs = [(self.pr.tb[0], self.host[0]), (self.pr.tb[2], self.host[1])]
         elif self.name == "heat3d":
-            self.pr = K.heat3d_setup(ctx, self.host[0], zc=tile or K.HEAT_ZC,
+            self.pr = K.heat3d_setup(ctx, self.host[0], zc=tile or None,
                                      kernel=getattr(self, "variant", None) or "heat3d_tb2", tiles=self.tiles)
             # two sweeps per launch for the default heat3d_tb2: 8 B per cell per launch = 4 B/LU
             self.sweeps = self.pr.sweeps

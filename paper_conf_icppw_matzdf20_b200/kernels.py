@@ -54,7 +54,10 @@ def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
 HEAT_TB2_COLS, HEAT_TB2_ROWS = 120, 24    # "heat3d_tb2": owned columns x rows per logical block
 
 
-def heat3d_tb2_launch(d, h, w, zc=HEAT_ZC):
+HEAT_TB2_ZC = 64                          # "heat3d_tb2": planes per logical block (measured: 64 beats 128 by ~3%)
+
+
+def heat3d_tb2_launch(d, h, w, zc=HEAT_TB2_ZC):
     """Logical block = 120 columns x 24 rows x zc planes, two sweeps per launch."""
     return (_cdiv(w, HEAT_TB2_COLS), _cdiv(h, HEAT_TB2_ROWS), _cdiv(d, zc)), (224, 1, 1), [d, h, w, zc]
 
@@ -155,13 +158,16 @@ def hotspot2d_iterate(pr, iters, start=0):
     return t1 if ((start + iters) // k) % 2 == 1 else t0
 
 
-def heat3d_setup(ctx, u_host, zc=HEAT_ZC, bdy=HEAT_BDY, kernel="heat3d", tiles=None):
+def heat3d_setup(ctx, u_host, zc=None, bdy=HEAT_BDY, kernel="heat3d", tiles=None):
     """kernel: heat3d (one sweep per launch, TMA ring), heat3d_regs, heat3d_tb2 (two)."""
     d, h, w = u_host.shape
     pr = Problem(ctx, kernel, tiles)
     u0 = pr.buffer((d, h, w), 4, host=u_host)
     u1 = pr.buffer((d, h, w), 4)
-    pr.geom = heat3d_tb2_launch(d, h, w, zc) if kernel == "heat3d_tb2" else heat3d_launch(d, h, w, zc, bdy)
+    if kernel == "heat3d_tb2":
+        pr.geom = heat3d_tb2_launch(d, h, w, zc or HEAT_TB2_ZC)
+    else:
+        pr.geom = heat3d_launch(d, h, w, zc or HEAT_ZC, bdy)
     pr.shape = (d, h, w)
     pr.ub = (u0, u1)
     pr.sweeps = 2 if kernel == "heat3d_tb2" else 1

@@ -74,14 +74,14 @@ def test_c2_hotspot_fullsize_tbk_sampled():
 # ------------------------------------------------------------------ C3 Heat 1024^3, 50 it
 @pytest.mark.parametrize("kernel", ["heat3d_tb2", "heat3d"])
 def test_c3_heat_fullsize_sampled(kernel):
-    """heat3d_tb2 (bench default: 25 launches of two sweeps, ZC = 128) and heat3d (one sweep)."""
+    """heat3d_tb2 (bench default: 25 launches of two sweeps, ZC = 64) and heat3d (one sweep)."""
     d = h = w = 1024
     iters = 50
     u = synth.heat_grid(d, h, w)
     res = {}
     for P in (1, 2):
         ctx = gpu_ctx(P)
-        pr = K.heat3d_setup(ctx, u, kernel=kernel)       # bench config: ZC = 128 (heat3d: bdy = 62)
+        pr = K.heat3d_setup(ctx, u, kernel=kernel)       # bench config: ZC = 128 (heat3d, bdy = 62) / 64 (heat3d_tb2)
         res[P] = fetch(ctx, K.heat3d_iterate(pr, iters), (d, h, w))
         st = abi.pk_get_stats(ctx)
         abi.pk_finalize(ctx)
