@@ -367,7 +367,7 @@ enum {
  * multi-stream (multi-device) CUDA graph and afterwards replays the graph and restores
  * the memoised post-launch tracker states instead of re-planning and re-issuing every
  * CUDA call -- the host overhead the paper measures as "patterns".
- * Active for single-process contexts with more than one local partition, unless
+ * Active for single-process contexts (any number of local partitions, P = 1 included), unless
  * PK_MODE_TIME_KERNELS, PK_MODE_GLOBAL_BARRIER or PK_MODE_NO_GRAPHS is set. */
 int pk_set_mode(pk_ctx ctx, uint32_t flags);
 uint32_t pk_get_mode(pk_ctx ctx);

@@ -308,14 +308,23 @@ def pk_builtin_kernel(ctx, name) -> int:
     return out.value
 
 
+_LAUNCH_ARGS = {}   # marshalled ctypes arguments of recent launches (steady-state loops repeat them)
+
+
 def pk_launch_partitioned(ctx, kernel, grid, block, args, scalars=(), smem=0):
     """args: one int per kernel argument -- the pk_buf id for a buffer, the
     (int64) value for a scalar; None passes a NULL pointer."""
-    vals = [C.c_int64(a) if a is not None else None for a in args]
-    argv = (C.c_void_p * max(1, len(vals)))(*[C.addressof(v) if v is not None else None for v in vals])
-    sc = list(scalars)
-    _check(lib().pk_launch_partitioned(ctx, kernel, _i32(grid), _i32(block), smem, argv, _i64(sc), len(sc)),
-           "pk_launch_partitioned")
+    key = (kernel, tuple(grid), tuple(block), tuple(args), tuple(scalars))
+    m = _LAUNCH_ARGS.get(key)
+    if m is None:
+        vals = [C.c_int64(a) if a is not None else None for a in args]
+        argv = (C.c_void_p * max(1, len(vals)))(*[C.addressof(v) if v is not None else None for v in vals])
+        sc = list(scalars)
+        m = (_i32(grid), _i32(block), argv, _i64(sc), len(sc), vals)
+        if len(_LAUNCH_ARGS) > 1024:
+            _LAUNCH_ARGS.clear()
+        _LAUNCH_ARGS[key] = m
+    _check(lib().pk_launch_partitioned(ctx, kernel, m[0], m[1], smem, m[2], m[3], m[4]), "pk_launch_partitioned")
 
 
 def pk_synchronize(ctx):

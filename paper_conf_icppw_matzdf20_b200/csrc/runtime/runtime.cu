@@ -1349,7 +1349,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
     const Kernel& K = c->kernels[k];
     const uint32_t mode = c->mode;
     // builtin launchers take every scalar from `scalars`, so the key below captures the launch
-    const bool can_graph = !c->host_only && c->world == 1 && c->nlocal > 1 && K.nargs && args && K.launcher &&
+    const bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && K.nargs && args && K.launcher &&
                            !(mode & (PK_MODE_TIME_KERNELS | PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
     if (!can_graph) {
         if (!c->host_only)

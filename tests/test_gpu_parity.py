@@ -375,7 +375,7 @@ def test_gemm_read_pattern_placement_moves_nothing():
 
 
 # ------------------------------------------------------------------ steady-state graph replay
-@pytest.mark.parametrize("P", [2, 4])
+@pytest.mark.parametrize("P", [1, 2, 4])
 def test_graph_replay_matches_eager_and_one_way(P):
     t, p = synth.hotspot_grids(256, 1024)
     iters = 24
