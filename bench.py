@@ -356,7 +356,7 @@ def main():
     ap.add_argument("--parts", type=int, default=0, help="partitions (default: one per GPU)")
     ap.add_argument("--iters", type=int, default=0, help="iterations per step (default: the config's)")
     ap.add_argument("--impl", default="pk", choices=["pk", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=6)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
@@ -443,21 +443,31 @@ def main():
     if sampler:
         sampler.start()
         time.sleep(0.3)
-    # (1) the timed region: the production path (graph replay active when P > 1)
+    # (1) the timed region.  Kernels of 100 us and more (every config but the latency-bound
+    # C1) are timed live in it: PK_MODE_TIME_KERNELS records CUDA events around every
+    # partition kernel on its own stream.  C1 (microsecond launches) keeps steady-state
+    # graph replay in the timed region and gets its kernel events from a second pass.
+    live = w.name != "jacobi2d"
+    if live:
+        abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
     abi.pk_synchronize(ctx)
     abi.pk_timer_begin(ctx)
     for _ in range(args.steps):
         w.step()
     elapsed_ms = abi.pk_timer_end(ctx)
     st = abi.pk_get_stats(ctx)
-    # (2) per-kernel CUDA events for the roofline (events around every partition kernel)
-    abi.pk_reset_stats(ctx)
-    abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
-    for _ in range(max(1, min(args.steps, 3))):
-        w.step()
-    abi.pk_synchronize(ctx)
-    stk = abi.pk_get_stats(ctx)
-    abi.pk_set_mode(ctx, base_mode)
+    if live:
+        stk = st
+        abi.pk_set_mode(ctx, base_mode)
+    else:
+        # (2) per-kernel CUDA events for the roofline (events around every partition kernel)
+        abi.pk_reset_stats(ctx)
+        abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
+        for _ in range(max(1, min(args.steps, 3))):
+            w.step()
+        abi.pk_synchronize(ctx)
+        stk = abi.pk_get_stats(ctx)
+        abi.pk_set_mode(ctx, base_mode)
     clocks = sampler.stop() if sampler else {}
     st["kernel_ms"], st["timed_kernels"] = stk["kernel_ms"], stk["timed_kernels"]
     if dist:
@@ -521,6 +531,9 @@ def main():
         "clocks": clocks,
         "roofline": roofline,
         "kernel_ms_avg": avg_kernel_ms,
+        "kernel_timing": ("CUDA events around every partition kernel on its stream, inside the timed region"
+                          if live else "CUDA events around every partition kernel on its stream, second pass of "
+                          "the same steps right after the timed region (the timed region replays graphs)"),
         "transfers": {"stale_bytes": int(st["stale_bytes"]), "moved_bytes": int(st["moved_bytes"]),
                       "analytic_min_bytes": w.stale_min(P) * args.steps if not w.tiles else None,
                       "copies": int(st["copies"]), "strided_copies": int(st["strided_copies"]),
@@ -561,21 +574,45 @@ def main():
 
     # ---- e2e: same metric with the H2D upload and D2H gather inside every step ----
     if not args.no_e2e:
-        pinned = [(b, torch.from_numpy(h).pin_memory()) for b, h in w.upload_bufs]
-        out_host = torch.empty(w.out_shape(), dtype=torch.float32).pin_memory()
-        abi.pk_synchronize(ctx)
+        pinned_of = {}
+        def pinned(host):
+            if id(host) not in pinned_of:
+                pinned_of[id(host)] = torch.from_numpy(host).pin_memory()
+            return pinned_of[id(host)]
+        # Single process: two contexts (two device copies of the problem) and the asynchronous
+        # host copies, so that step i+1's H2D overlaps step i's kernels and D2H (the host link is
+        # full duplex); every step still uploads its inputs and reads its result back.
+        # SPMD ranks, or too little free HBM for a second copy: one context, blocking copies.
+        free_b, total_b = torch.cuda.mem_get_info(devices[0])
+        pipelined = dist is None and free_b > 1.2 * (total_b - free_b) + (8 << 30)
+        ctxs, ws = [ctx], [w]
+        if pipelined:
+            import copy
+            ctx2 = abi.pk_init(P, part_device=[p % ngpu for p in range(P)])
+            abi.pk_set_mode(ctx2, base_mode)
+            w2 = copy.copy(w)
+            w2.setup(ctx2)
+            ctxs.append(ctx2)
+            ws.append(w2)
+        outs = [torch.empty(w.out_shape(), dtype=torch.float32).pin_memory() for _ in ctxs]
+        for c in ctxs:
+            abi.pk_synchronize(c)
         if dist:
             dist.barrier()
         t0 = time.perf_counter()
         h2d = d2h = 0
-        for _ in range(args.e2e_steps):
-            for b, hbuf in pinned:
-                abi.pk_copy_from_host(ctx, b, hbuf)
+        for s in range(args.e2e_steps):
+            c, ws_, out_host = ctxs[s % len(ctxs)], ws[s % len(ctxs)], outs[s % len(ctxs)]
+            for b, host in ws_.upload_bufs:
+                hbuf = pinned(host)
+                (abi.pk_copy_from_host_async if pipelined else abi.pk_copy_from_host)(c, b, hbuf)
                 h2d += hbuf.numel() * hbuf.element_size()
-            w.t = 0
-            out = w.step()
-            abi.pk_sync_to_host(ctx, out, out_host)
+            ws_.t = 0
+            out = ws_.step()
+            (abi.pk_sync_to_host_async if pipelined else abi.pk_sync_to_host)(c, out, out_host)
             d2h += out_host.numel() * out_host.element_size()
+        for c in ctxs:
+            abi.pk_synchronize(c)
         el = time.perf_counter() - t0
         if dist:
             te = torch.tensor([el], dtype=torch.float64)
@@ -583,8 +620,15 @@ def main():
             el = float(te[0])
         result["e2e"] = {"value": w.units_per_iter * w.iters * args.e2e_steps / el / w.scale, "unit": w.unit,
                          "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
-                         "steps": args.e2e_steps, "timing": "wall clock around pk_copy_from_host + launches + "
-                                                           "pk_sync_to_host (pinned host buffers)"}
+                         "steps": args.e2e_steps,
+                         "timing": ("wall clock over all steps: per step pk_copy_from_host_async of the inputs + "
+                                    "launches + pk_sync_to_host_async of the result, steps alternating between two "
+                                    "contexts (H2D of one overlaps kernels + D2H of the other), pinned host buffers, "
+                                    "both contexts synchronised at the end" if pipelined else
+                                    "wall clock around pk_copy_from_host + launches + pk_sync_to_host per step "
+                                    "(pinned host buffers)")}
+        for c in ctxs[1:]:
+            abi.pk_finalize(c)
     abi.pk_finalize(ctx)
     if not args.no_cpu_baseline and ngpu == 1:
         result["cpu_baseline"] = cpu_oracle_rate(w)

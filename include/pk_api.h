@@ -161,6 +161,17 @@ int pk_copy_from_host(pk_ctx ctx, pk_buf buf, const void* host, size_t bytes);
 /* cudaMemcpy(DeviceToHost) replacement: n:1 gather, one copy per tracker segment
  * from a partition holding it (§8.2).  Blocking. */
 int pk_sync_to_host(pk_ctx ctx, pk_buf buf, void* host, size_t bytes);
+/* Asynchronous variants (cudaMemcpyAsync replacements, same distribution and tracker
+ * effect): the copies are enqueued on the partition streams, ordered by the same
+ * stream/event hazards as the transfers of pk_launch_partitioned, and the call returns
+ * without waiting.  The host buffer must stay valid (and, for overlap, pinned) until
+ * pk_synchronize; a D2H result is complete only then.  Lets a caller pipeline steps:
+ * the H2D of step i+1 (one context) overlaps the kernels and the D2H of step i (another
+ * context), the host link being full duplex.  In SPMD contexts (and, for the D2H, with
+ * PK_MODE_PUSH) they behave like the blocking calls.  Host-only contexts: tracker
+ * effect only, like pk_copy_from_host. */
+int pk_copy_from_host_async(pk_ctx ctx, pk_buf buf, const void* host, size_t bytes);
+int pk_sync_to_host_async(pk_ctx ctx, pk_buf buf, void* host, size_t bytes);
 /* Read-pattern-aware H2D (the paper's linear distribution is
  * "hoping that this pattern matches the read pattern of the following kernels",
  * P:L888-895, and its mismatch limits Matmul scaling): every

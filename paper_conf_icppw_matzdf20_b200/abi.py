@@ -115,6 +115,8 @@ def lib():
         "pk_register_buffer": [C.c_void_p, C.c_int, _I64P, C.c_int, C.POINTER(C.c_void_p), C.c_void_p, _I64P],
         "pk_copy_from_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
         "pk_sync_to_host": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
+        "pk_copy_from_host_async": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
+        "pk_sync_to_host_async": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t],
         "pk_copy_from_host_for": [C.c_void_p, C.c_int64, C.c_void_p, C.c_size_t, C.c_int64, C.c_int, _I32P, _I32P,
                                   _I64P, C.c_int],
         "pk_unregister_buffer": [C.c_void_p, C.c_int64],
@@ -274,6 +276,18 @@ def pk_sync_to_host(ctx, buf, host, nbytes=None):
     """host may be None on SPMD ranks other than 0 (then pass nbytes)."""
     _check(lib().pk_sync_to_host(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
            "pk_sync_to_host")
+
+
+def pk_copy_from_host_async(ctx, buf, host, nbytes=None):
+    """Enqueued H2D; `host` (pinned for overlap) must stay alive until pk_synchronize."""
+    _check(lib().pk_copy_from_host_async(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
+           "pk_copy_from_host_async")
+
+
+def pk_sync_to_host_async(ctx, buf, host, nbytes=None):
+    """Enqueued D2H gather; `host` is complete after pk_synchronize."""
+    _check(lib().pk_sync_to_host_async(ctx, buf, _addr(host), nbytes if nbytes is not None else _nbytes(host)),
+           "pk_sync_to_host_async")
 
 
 def pk_unregister_buffer(ctx, buf):

@@ -1013,6 +1013,43 @@ int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
     return PK_OK;
 }
 
+// Asynchronous H2D (single process): the same 1:n linear distribution, enqueued on
+// the partition streams behind what they already hold instead of draining the
+// context.  WAR: slab p's copy waits for the copies that read (b,p) on other streams
+// (wait_readers); everything else that touches instance p (its kernels, incoming
+// copies, D2H pieces) is on stream p already.  RAW: the copy is (b,p)'s last writer.
+int pk_copy_from_host_async(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
+    if (!valid_buf(c, b) || !host) return fail(PK_ERR_INVALID, "bad argument");
+    if (c->host_only || c->world > 1) return pk_copy_from_host(c, b, host, bytes);
+    Buffer& B = c->bufs[b];
+    if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (H2D copies the whole virtual buffer)");
+    for (uint64_t m : B.pushers)   // bytes pushed into an instance by another partition's kernel: drain
+        if (m) {
+            if (int r = pk_synchronize(c)) return r;
+            break;
+        }
+    if (int r = exit_graph_mode(c)) return r;
+    const uint64_t n = B.bytes / B.eb;
+    for (int p = 0; p < c->P; ++p) {
+        uint64_t lo = (uint64_t)p * n / c->P * B.eb, hi = (uint64_t)(p + 1) * n / c->P * B.eb;
+        if (hi <= lo || !c->local(p)) continue;
+        if (int r = c->set_device(c->dev[p])) return r;
+        if (int r = wait_readers(c, B, p)) return r;
+        PK_CUDA(cudaMemcpyAsync((char*)B.inst[p] + lo, (const char*)host + lo, hi - lo, cudaMemcpyHostToDevice,
+                                c->stream[p]));
+        if (c->P > 1) {
+            PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
+            B.last_writer[p] = W_COPY;
+        }
+    }
+    for (int p = 0; p < c->P; ++p) {
+        uint64_t lo = (uint64_t)p * n / c->P * B.eb, hi = (uint64_t)(p + 1) * n / c->P * B.eb;
+        if (hi > lo) B.tracker.assign(RangeList{Range{lo, hi}}, 1ull << p);
+    }
+    c->stats.h2d_bytes += B.bytes;
+    return PK_OK;
+}
+
 int pk_copy_from_host_for(pk_ctx c, pk_buf b, const void* host, size_t bytes, pk_kernel k, int arg,
                           const int32_t grid[3], const int32_t block[3], const int64_t* scalars, int ns) {
     if (!valid_buf(c, b) || !host || !valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
@@ -1160,7 +1197,7 @@ static int sync_to_host_ipc(pk_ctx c, Buffer& B, void* host) {
     return PK_OK;
 }
 
-int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
+static int sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes, bool async) {
     if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "bad argument");
     Buffer& B = c->bufs[b];
     if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (D2H gathers the whole virtual buffer)");
@@ -1191,9 +1228,19 @@ int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) {
         PK_CUDA(cudaMemcpyAsync((char*)host + pc.b, (const char*)B.inst[pc.src] + pc.b, pc.e - pc.b,
                                 cudaMemcpyDeviceToHost, c->stream[pc.src]));
     }
-    if (int r = pk_synchronize(c)) return r;
     c->stats.d2h_bytes += B.bytes;
-    return PK_OK;
+    return async ? PK_OK : pk_synchronize(c);
+}
+
+int pk_sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes) { return sync_to_host(c, b, host, bytes, false); }
+
+// Asynchronous D2H (single process, not with PK_MODE_PUSH): the pieces are enqueued on
+// the streams of the partitions that hold them, behind their writers; the host buffer
+// is complete after pk_synchronize.  A later write into a piece's instance is on the
+// same stream, so it cannot overtake the copy.
+int pk_sync_to_host_async(pk_ctx c, pk_buf b, void* host, size_t bytes) {
+    if (c && (c->world > 1 || (c->mode & PK_MODE_PUSH))) return pk_sync_to_host(c, b, host, bytes);
+    return sync_to_host(c, b, host, bytes, true);
 }
 
 // ------------------------------------------------------------------ kernels

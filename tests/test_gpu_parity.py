@@ -559,3 +559,36 @@ def test_heat3d_tb2_push_bitwise():
     r1, _ = _heat_tb2(u, 8, 1, 8)
     rp, st = _heat_tb2(u, 8, 3, 8, abi.PK_MODE_PUSH)
     assert np.array_equal(r1, rp) and st["pushed_bytes"] > 0
+
+
+# ------------------------------------------------------------------ asynchronous host copies (pipelined steps)
+@pytest.mark.parametrize("P", [1, 3])
+def test_async_host_copies_pipelined_contexts(P):
+    """bench.py's e2e pipeline: two contexts, every step = pk_copy_from_host_async of the inputs,
+    the launches, pk_sync_to_host_async of the result, no synchronisation between steps; every
+    step's result is bit-identical to the blocking path (and within 1e-5 of the oracle)."""
+    import torch
+    h, w, iters = 200, 1028, 12
+    t, p = synth.hotspot_grids(h, w)
+    ref, _ = _hotspot_k(t, p, iters, 1, 16, 4)
+    ok_, err = rel_ok(ref, ok.hotspot2d(t, p, iters), 1e-5)
+    assert ok_, err
+    ctxs = [gpu_ctx(P), gpu_ctx(P)]
+    zeros = np.zeros_like(t)
+    prs = [K.hotspot2d_setup(c, zeros, zeros, ty=16, kernel="hotspot2d_tbk", sweeps=4) for c in ctxs]
+    tp, pp = torch.from_numpy(t).pin_memory(), torch.from_numpy(p).pin_memory()
+    outs = [torch.full((h, w), -1.0, dtype=torch.float32).pin_memory() for _ in range(5)]
+    for s in range(5):
+        c, pr = ctxs[s % 2], prs[s % 2]
+        abi.pk_copy_from_host_async(c, pr.tb[0], tp)
+        abi.pk_copy_from_host_async(c, pr.tb[2], pp)
+        out = K.hotspot2d_iterate(pr, iters)
+        abi.pk_sync_to_host_async(c, out, outs[s])
+    for c in ctxs:
+        abi.pk_synchronize(c)
+    st = abi.pk_get_stats(ctxs[0])
+    for c in ctxs:
+        abi.pk_finalize(c)
+    for s in range(5):
+        assert np.array_equal(outs[s].numpy(), ref), s
+    assert st["moved_bytes"] == st["stale_bytes"]

@@ -465,6 +465,20 @@ def test_h2d_linear_distribution_tracker():
     abi.pk_finalize(ctx)
 
 
+@pytest.mark.parametrize("P", [1, 3, 5])
+def test_h2d_async_same_tracker_effect(P):
+    """pk_copy_from_host_async distributes like pk_copy_from_host (shadow oracle's linear H2D)."""
+    ctx = host_ctx(P)
+    b = abi.pk_register_buffer(ctx, (23, 3), 4)
+    abi.pk_copy_from_host_async(ctx, b, np.zeros((23, 3), np.float32))
+    sb = shadow.ShadowBuffer(69, 4, P)
+    sb.h2d_linear()
+    assert abi.pk_tracker_dump(ctx, b) == sb.rle()
+    with pytest.raises(abi.PkError):
+        abi.pk_sync_to_host_async(ctx, b, np.zeros((23, 3), np.float32))   # a host-only context holds no data
+    abi.pk_finalize(ctx)
+
+
 @pytest.mark.parametrize("m,n,k", [(300, 520, 200), (1024, 512, 64)])
 @pytest.mark.parametrize("P", [1, 2, 3])
 def test_gemm_regions(m, n, k, P):
