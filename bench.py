@@ -356,7 +356,7 @@ def main():
     ap.add_argument("--parts", type=int, default=0, help="partitions (default: one per GPU)")
     ap.add_argument("--iters", type=int, default=0, help="iterations per step (default: the config's)")
     ap.add_argument("--impl", default="pk", choices=["pk", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=6)
+    ap.add_argument("--e2e-steps", type=int, default=8)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
@@ -584,7 +584,8 @@ def main():
         # full duplex); every step still uploads its inputs and reads its result back.
         # SPMD ranks, or too little free HBM for a second copy: one context, blocking copies.
         free_b, total_b = torch.cuda.mem_get_info(devices[0])
-        pipelined = dist is None and free_b > 1.2 * (total_b - free_b) + (8 << 30)
+        pipelined = (dist is None and free_b > 1.2 * (total_b - free_b) + (8 << 30)
+                     and not os.environ.get("PK_E2E_BLOCKING"))
         ctxs, ws = [ctx], [w]
         if pipelined:
             import copy
@@ -595,6 +596,9 @@ def main():
             ctxs.append(ctx2)
             ws.append(w2)
         outs = [torch.empty(w.out_shape(), dtype=torch.float32).pin_memory() for _ in ctxs]
+        for ws_ in ws:                       # pin (once) before the timed region
+            for _, host in ws_.upload_bufs:
+                pinned(host)
         for c in ctxs:
             abi.pk_synchronize(c)
         if dist:
@@ -611,6 +615,8 @@ def main():
             out = ws_.step()
             (abi.pk_sync_to_host_async if pipelined else abi.pk_sync_to_host)(c, out, out_host)
             d2h += out_host.numel() * out_host.element_size()
+            if os.environ.get("PK_E2E_TRACE"):
+                print(f"e2e step {s}: enqueued at {time.perf_counter() - t0:.4f} s", file=sys.stderr, flush=True)
         for c in ctxs:
             abi.pk_synchronize(c)
         el = time.perf_counter() - t0
