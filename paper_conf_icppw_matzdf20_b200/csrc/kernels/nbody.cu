@@ -83,7 +83,10 @@ __device__ __forceinline__ u64 rsqrt2(u64 v) {
 // adds the kSplit partials in order s = 0..kSplit-1.  The persistent grid walks
 // (logical block, part) items, so ~kSplit x more, smaller work items than blocks
 // keep every SM busy to the end (no 2.3-wave tail).
-constexpr int kSplit = 8;
+#ifndef PK_NBODY_SPLIT
+#define PK_NBODY_SPLIT 16
+#endif
+constexpr int kSplit = PK_NBODY_SPLIT;  // 16: 16384 items over 444 CTAs (measured 8/16/32: 2386/2396/2397)
 
 __device__ __forceinline__ void part_chunks(int64_t N, int s, int64_t& c_begin, int64_t& c_end) {
     const int64_t nch = (N + kChunk - 1) / kChunk;
