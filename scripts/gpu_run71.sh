@@ -4,7 +4,7 @@ python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 |
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "PYTEST: $(tail -1 gpurun_out/pytest_gpu.log)"
 grep -E "FAILED|Error" gpurun_out/pytest_gpu.log | head -5
 timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('SMOKE OK')" > gpurun_out/smoke.log 2>&1; tail -1 gpurun_out/smoke.log
-/usr/bin/time -f "bench default wall %e s" timeout 900 python bench.py > gpurun_out/bench_default.log 2>gpurun_out/bench_default.err; tail -1 gpurun_out/bench_default.log > gpurun_out/bench_default.json; tail -1 gpurun_out/bench_default.err
+timeout 900 python bench.py > gpurun_out/bench_default.log 2>gpurun_out/bench_default.err; tail -1 gpurun_out/bench_default.log > gpurun_out/bench_default.json; tail -1 gpurun_out/bench_default.err
 timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.log 2>&1; tail -1 gpurun_out/bench_reference.log > gpurun_out/bench_reference.json
 for w in heat3d sgemm nbody jacobi2d; do
   timeout 900 python bench.py --workload $w --steps 5 --warmup 3 > gpurun_out/bench_$w.log 2>&1; tail -1 gpurun_out/bench_$w.log > gpurun_out/bench_$w.json
