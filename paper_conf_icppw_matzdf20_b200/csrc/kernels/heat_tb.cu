@@ -8,10 +8,10 @@
 // and its write set its own cells: 8 B per cell per launch = 4 B per lattice
 // update (half the one-sweep kernel's 8 B/LU).
 //
-// Design (B200): logical block = 120 columns x 24 rows x ZC planes.  A producer
+// Design (B200): logical block = 120 columns x 16 rows x ZC planes.  A producer
 // warp streams one 3-D tensor-TMA box per plane -- 128 columns [c0-4, c0+124) x
-// 28 rows [y0-2, y0+26) x 1 plane, out-of-grid columns/rows zero-filled, the plane
-// index clamped -- into an 8-slot mbarrier ring.  6 consumer warps march z; warp w
+// 20 rows [y0-2, y0+18) x 1 plane, out-of-grid columns/rows zero-filled, the plane
+// index clamped -- into a 6-slot mbarrier ring, 3 CTAs/SM.  4 consumer warps march z; warp w
 // owns rows y0+4w .. +3, a lane owns 4 columns.  Per input plane q a warp computes
 // sweep 1 of plane q-1 on its 4 rows plus one halo row above and below (6 rows,
 // inputs from shared memory) into a register window of 3 planes x 6 rows, and
@@ -39,18 +39,18 @@ constexpr float kAlpha = 0.125f;
 constexpr int kCols = 128;                // columns per warp window (box width)
 constexpr int kOwnC = 120;                // owned columns per block (lanes 1..30)
 constexpr int kRW = 4;                    // owned rows per consumer warp
-constexpr int kNW = 6;                    // consumer warps
-constexpr int kRows = kRW * kNW;          // owned rows per block (24)
+constexpr int kNW = 4;                    // consumer warps (3 CTAs/SM; measured 6 warps x 2 CTAs: -4 %)
+constexpr int kRows = kRW * kNW;          // owned rows per block (16)
 constexpr int kBoxRows = kRows + 4;       // rows y0-2 .. y0+kRows+1
 constexpr int kL1 = kRW + 2;              // sweep-1 rows per warp (one halo row each side)
 #ifndef PK_HEATTB_NS
-#define PK_HEATTB_NS 8
+#define PK_HEATTB_NS 6
 #endif
-constexpr int kNS = PK_HEATTB_NS;         // plane ring depth (measured 6 / 7 / 8: 1196 / 1188 / 1206 GLUP/s)
+constexpr int kNS = PK_HEATTB_NS;         // plane ring depth (3 CTAs x 6 x 10 KB per SM; 7 slots: -2 %)
 constexpr int kSlot = kBoxRows * kCols;   // floats per plane slot (14 KB)
 constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + 2 * kNS * 8 + 128;
 #ifndef PK_HEATTB_MINB
-#define PK_HEATTB_MINB 2
+#define PK_HEATTB_MINB 3
 #endif
 
 __device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, int32_t z,
@@ -211,7 +211,7 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
 
 int describe_heat3d_tb2(pk_ctx c, pk_kernel k) {
     // scalars: 0 = D, 1 = H, 2 = W, 3 = ZC.  Logical block (bx, by, bz) = columns
-    // [120 bx, +120) x rows [24 by, +24) x planes [ZC bz, +ZC), guarded.  Reads the
+    // [120 bx, +120) x rows [16 by, +16) x planes [ZC bz, +ZC), guarded.  Reads the
     // clamped 5x5x5 cube around every cell (the box dilated by 2 in every dimension:
     // one tap, positions [b*scale, b*scale + extent + 4) with the guard shifted by 4,
     // offset -2, clamped; corners included -- a read over-approximation);
@@ -243,7 +243,7 @@ cudaError_t launch_heat3d_tb2(const LaunchInfo& li) {
             attr_err = cudaFuncSetAttribute(k_heat3d_tb2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
     });
     if (attr_err != cudaSuccess) return attr_err;
-    // tensor map of this instance: dims (W, H, D), box (128, 28, 1), OOB zero fill
+    // tensor map of this instance: dims (W, H, D), box (128, 20, 1), OOB zero fill
     static std::mutex mu;
     static std::unordered_map<const void*, std::pair<uint64_t, CUtensorMap>> cache;
     CUtensorMap tm;

@@ -51,15 +51,15 @@ def heat3d_launch(d, h, w, zc=HEAT_ZC, bdy=HEAT_BDY):
     return (_cdiv(w, 128), _cdiv(h, bdy), _cdiv(d, zc)), (32, bdy, 1), [d, h, w, zc]
 
 
-HEAT_TB2_COLS, HEAT_TB2_ROWS = 120, 24    # "heat3d_tb2": owned columns x rows per logical block
+HEAT_TB2_COLS, HEAT_TB2_ROWS = 120, 16    # "heat3d_tb2": owned columns x rows per logical block
 
 
 HEAT_TB2_ZC = 64                          # "heat3d_tb2": planes per logical block (measured: 64 beats 128 by ~3%)
 
 
 def heat3d_tb2_launch(d, h, w, zc=HEAT_TB2_ZC):
-    """Logical block = 120 columns x 24 rows x zc planes, two sweeps per launch."""
-    return (_cdiv(w, HEAT_TB2_COLS), _cdiv(h, HEAT_TB2_ROWS), _cdiv(d, zc)), (224, 1, 1), [d, h, w, zc]
+    """Logical block = 120 columns x 16 rows x zc planes, two sweeps per launch."""
+    return (_cdiv(w, HEAT_TB2_COLS), _cdiv(h, HEAT_TB2_ROWS), _cdiv(d, zc)), (160, 1, 1), [d, h, w, zc]
 
 
 def nbody_launch(n, bdx=NBODY_BDX):

@@ -654,6 +654,6 @@ def test_heat3d_tb2_regions(d, h, w, zc, P):
     for p in range(P):
         box = abi.pk_partition_grid(ctx, kk, grid, p)
         lib = _lib_sets(ctx, kk, 6, bufs + [None] * 4, box, blk, sc)
-        ora = _oracle_sets(regions.heat3d_tb2(box, d, h, w, zc), {0: 4, 1: 4})
+        ora = _oracle_sets(regions.heat3d_tb2(box, d, h, w, zc, rows=16), {0: 4, 1: 4})   # 120 x 16 x zc blocks
         assert lib == ora
     abi.pk_finalize(ctx)
