@@ -332,6 +332,10 @@ def run_reference(args, w: Workload, rank):
     """--impl reference: the oracle as it stands, on the host cores, same metric."""
     if rank != 0:
         return None
+    # torchrun sets OMP_NUM_THREADS=1 per worker; rank 0 runs the oracle alone on the host
+    # cores (the other ranks do no work), so give its OpenMP runtime all of them
+    if env_int("WORLD_SIZE", 1) > 1:
+        os.environ["OMP_NUM_THREADS"] = str(len(os.sched_getaffinity(0)))
     # each step is a bounded sample; warmup steps are run untimed
     for _ in range(args.warmup):
         cpu_oracle_rate(w, budget_s=1.0, max_iters=1)
