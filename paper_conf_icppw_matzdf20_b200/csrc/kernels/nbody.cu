@@ -101,7 +101,19 @@ __device__ __forceinline__ void part_chunks(int64_t N, int s, int64_t& c_begin, 
 // FFMA2 take as a free broadcast operand; each body accumulates two interleaved
 // partial sums (even and odd sources) that are added at the end -- a fixed,
 // position-only order.
-__global__ void __launch_bounds__(256, 3) k_nbody_partial(const float4* __restrict__ pin, float4* __restrict__ partial,
+// 2 CTAs/SM (125 registers, no spill) and the source loop unrolled 32-fold give the
+// scheduler independent chains to cover the MUFU and FFMA2 latencies.  Measured
+// (CTAs/SM, unroll) on C5: (3, 4) 2408, (2, 4) 2491, (2, 8) 2557, (2, 16) 2605,
+// (2, 32) 2620, (2, 64) 2293, (1, 16) 2604 G interactions/s.
+#ifndef PK_NBODY_MINB
+#define PK_NBODY_MINB 2
+#endif
+#ifndef PK_NBODY_UNROLL
+#define PK_NBODY_UNROLL 32
+#endif
+#define PK_PRAGMA(x) _Pragma(#x)
+#define PK_UNROLL(n) PK_PRAGMA(unroll n)
+__global__ void __launch_bounds__(256, PK_NBODY_MINB) k_nbody_partial(const float4* __restrict__ pin, float4* __restrict__ partial,
                                                        int64_t N, pk_partition part) {
     __shared__ float4 sh[kTile];  // kTile / 2 source pairs: (x0,x1,y0,y1), (z0,z1,m0,m1)
     const int64_t nb = part.max[0] - part.min[0];
@@ -138,7 +150,7 @@ __global__ void __launch_bounds__(256, 3) k_nbody_partial(const float4* __restri
                     sh[2 * s + 1] = make_float4(q0.z, q1.z, q0.w, q1.w);
                 }
                 __syncthreads();
-#pragma unroll 4
+                PK_UNROLL(PK_NBODY_UNROLL)
                 for (int s = 0; s < kTile / 2; ++s) {
                     const float4 A = sh[2 * s], B = sh[2 * s + 1];
                     const u64 qx = pk2(A.x, A.y), qy = pk2(A.z, A.w), qz = pk2(B.x, B.y), qm = pk2(B.z, B.w);
