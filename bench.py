@@ -142,13 +142,15 @@ class Workload:
         from paper_conf_icppw_matzdf20_b200 import kernels as K
         self.K = K
         if name == "hotspot2d":
-            self.shape = (16384, 16384)
+            # PK_BENCH_ROWS (experiments only): fewer rows, e.g. one SPMD rank's share at N = 8
+            self.shape = (int(os.environ.get("PK_BENCH_ROWS", 16384)), 16384)
             self.host = synth.hotspot_grids(*self.shape)
             self.units_per_iter = self.shape[0] * self.shape[1]
             self.bytes_per_unit = 12          # temp read + power read + temp write
             self.unit, self.metric = "GLUP/s", "hotspot2d_glups"
         elif name == "heat3d":
-            self.shape = (1024, 1024, 1024)
+            # PK_BENCH_PLANES (experiments only): fewer planes, e.g. one SPMD rank's share at N = 8
+            self.shape = (int(os.environ.get("PK_BENCH_PLANES", 1024)), 1024, 1024)
             self.host = (synth.heat_grid(*self.shape),)
             self.units_per_iter = int(np.prod(self.shape))
             self.bytes_per_unit = 8
@@ -178,9 +180,28 @@ class Workload:
             raise SystemExit(f"unknown workload {name}")
         self.scale = getattr(self, "scale", 1e9)
 
+    def block_depth(self):
+        """Rows per tile (Hotspot) / planes per block (Heat) when --tile is not given: the
+        persistent Hotspot grid and the Heat block grid quantise into waves of resident
+        CTAs, which matters once one GPU holds only a slab (SPMD at N = 4, 8).  Measured on
+        one B200 with a rank's share of the grid (PK_BENCH_ROWS / PK_BENCH_PLANES):
+        Hotspot 2048 rows TY 128 / 96 / 64 = 1274 / 1554 / 1536 GLUP/s, 4096 rows 1712 /
+        - / 1729, 16384 rows flat; Heat 128 planes ZC 64 / 24 / 16 = 1121 / 1185 / 1173,
+        256 planes 1154 / - / 1260 (ZC 32: 1234), 1024 planes 1268 / 1255 (24) / 1234."""
+        tile = getattr(self, "tile", 0)
+        if tile:
+            return tile
+        g = max(1, getattr(self, "gpus_used", 1))
+        if self.name == "hotspot2d":
+            # 64 (not the marginally faster 96) keeps the row blocks divisible among 8 slabs
+            return self.K.HOTSPOT_TY if self.shape[0] // g >= 4096 else 64
+        if self.name == "heat3d":
+            return min(64, max(16, (self.shape[0] // g) // 16 // 8 * 8))
+        return 0
+
     def setup(self, ctx):
         K = self.K
-        tile = getattr(self, "tile", 0)
+        tile = self.block_depth()
         if self.name == "hotspot2d":
             self.pr = K.hotspot2d_setup(ctx, *self.host, ty=tile or K.HOTSPOT_TY,
                                         kernel=getattr(self, "variant", None) or "hotspot2d_tbk",
@@ -436,6 +457,7 @@ def main():
         process_model = "one host process drives all partitions"
     base_mode = abi.PK_MODE_PUSH if args.push else 0
     abi.pk_set_mode(ctx, base_mode)
+    w.gpus_used = world if world > 1 else len(devices)
     w.setup(ctx)
     for _ in range(args.warmup):
         w.step()
@@ -529,6 +551,8 @@ def main():
                    "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk",
                                                              "heat3d": "heat3d_tb2"}.get(w.name, w.name),
                    "sweeps_per_launch": getattr(w, "sweeps", 1),
+                   **({"rows_per_tile": w.block_depth()} if w.name == "hotspot2d" and not w.variant else {}),
+                   **({"planes_per_block": w.block_depth()} if w.name == "heat3d" and not w.variant else {}),
                    "partition_shape": list(w.tiles) if w.tiles else "1-D slabs of the slowest grid dim"},
         "gpu_launches": int(st["kernel_launches"] + st["copy_kernels"]),
         "graph_replays": int(st.get("graph_replays", 0)),

@@ -1,0 +1,5 @@
+# one SPMD rank's C3 share at N = 8 / 4 (128 / 256 planes) on one GPU: planes per block
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || tail -5 gpurun_out/build.log
+for pl in 128 256; do for zc in 64 32 16 64; do
+PK_BENCH_PLANES=$pl timeout 300 python bench.py --workload heat3d --tile $zc --steps 5 --warmup 3 --no-e2e --no-cpu-baseline > /tmp/b.log 2>&1; tail -1 /tmp/b.log | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('planes=$pl ZC=$zc', round(d['value'],1), round(d['roofline']['frac'],3), round(d['kernel_ms_avg'],4), d['clocks']['sm_mhz'])" || tail -3 /tmp/b.log
+done; done
