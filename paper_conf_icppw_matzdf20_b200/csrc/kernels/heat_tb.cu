@@ -49,6 +49,9 @@ constexpr int kL1 = kRW + 2;              // sweep-1 rows per warp (one halo row
 constexpr int kNS = PK_HEATTB_NS;         // plane ring depth (3 CTAs x 6 x 10 KB per SM; 7 slots: -2 %)
 constexpr int kSlot = kBoxRows * kCols;   // floats per plane slot (14 KB)
 constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + 2 * kNS * 8 + 128;
+#ifndef PK_HEATTB_PNS
+#define PK_HEATTB_PNS 256
+#endif
 #ifndef PK_HEATTB_MINB
 #define PK_HEATTB_MINB 3
 #endif
@@ -118,7 +121,10 @@ __global__ void __launch_bounds__((kNW + 1) * 32, PK_HEATTB_MINB)
         constexpr uint32_t bytes = (uint32_t)kSlot * 4u;
         for (int q = 0; q < nq; ++q) {
             const int s = q % kNS;
-            ptx::mbar_wait(&empty[s], ((q / kNS) & 1u) ^ 1u);
+            // polls with a 256-ns back-off: 3 producers per SM spinning took issue slots from the
+            // 12 consumer warps (1261-1267 spinning vs 1296-1311 GLUP/s); Hotspot's ring of 4-KB
+            // rows needs prompt refills instead (back-off there: 1810 vs 1900)
+            ptx::mbar_wait_backoff(&empty[s], ((q / kNS) & 1u) ^ 1u, PK_HEATTB_PNS);
             int64_t p = k0 - 2 + q;
             p = p < 0 ? 0 : (p >= D ? D - 1 : p);
             ptx::mbar_arrive_expect_tx(&full[s], bytes);
