@@ -612,16 +612,23 @@ def main():
         # full duplex); every step still uploads its inputs and reads its result back.
         # SPMD ranks, or too little free HBM for a second copy: one context, blocking copies.
         free_b, total_b = torch.cuda.mem_get_info(devices[0])
-        pipelined = (dist is None and free_b > 1.2 * (total_b - free_b) + (8 << 30)
-                     and not os.environ.get("PK_E2E_BLOCKING"))
+        # Contexts in flight: a step's chain (H2D -> kernels -> D2H) must be covered by the others'
+        # copies.  Measured (e2e GLUP/s or TF/s, 2 vs 3 contexts): C3 (4 GiB each way) 482 vs 538,
+        # C2 598 vs 596, C4 170 vs 81 (three concurrent persistent GEMMs contend) -> 3 for C3 only.
+        used_b = total_b - free_b
+        want = 3 if w.name == "heat3d" else 2
+        n_ctx = 1 if dist is not None or os.environ.get("PK_E2E_BLOCKING") else \
+            min(want, 3 if free_b > 2.2 * used_b + (8 << 30) else 2 if free_b > 1.2 * used_b + (8 << 30) else 1)
+        n_ctx = min(n_ctx, int(os.environ.get("PK_E2E_CONTEXTS", n_ctx)))
+        pipelined = n_ctx > 1
         ctxs, ws = [ctx], [w]
-        if pipelined:
-            import copy
-            ctx2 = abi.pk_init(P, part_device=[p % ngpu for p in range(P)])
-            abi.pk_set_mode(ctx2, base_mode)
+        import copy
+        for _ in range(n_ctx - 1):
+            c2 = abi.pk_init(P, part_device=[p % ngpu for p in range(P)])
+            abi.pk_set_mode(c2, base_mode)
             w2 = copy.copy(w)
-            w2.setup(ctx2)
-            ctxs.append(ctx2)
+            w2.setup(c2)
+            ctxs.append(c2)
             ws.append(w2)
         outs = [torch.empty(w.out_shape(), dtype=torch.float32).pin_memory() for _ in ctxs]
         for ws_ in ws:                       # pin (once) before the timed region
@@ -656,9 +663,9 @@ def main():
                          "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
                          "steps": args.e2e_steps,
                          "timing": ("wall clock over all steps: per step pk_copy_from_host_async of the inputs + "
-                                    "launches + pk_sync_to_host_async of the result, steps alternating between two "
-                                    "contexts (H2D of one overlaps kernels + D2H of the other), pinned host buffers, "
-                                    "both contexts synchronised at the end" if pipelined else
+                                    "launches + pk_sync_to_host_async of the result, steps rotating over %d contexts (H2D "
+                                    "of one overlaps kernels + D2H of the others), pinned host buffers, all contexts "
+                                    "synchronised at the end" % len(ctxs) if pipelined else
                                     "wall clock around pk_copy_from_host + launches + pk_sync_to_host per step "
                                     "(pinned host buffers)")}
         for c in ctxs[1:]:
