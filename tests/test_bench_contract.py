@@ -1,0 +1,44 @@
+"""bench.py on a CPU host: the reference arm's JSON line (the oracle timed on the host
+cores) and the launch-configuration choice for the slab one GPU holds."""
+import importlib.util
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _bench_module():
+    spec = importlib.util.spec_from_file_location("bench", os.path.join(ROOT, "bench.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    return m
+
+
+def test_reference_arm_json_line():
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--workload", "jacobi2d",
+                        "--steps", "1", "--warmup", "1"], capture_output=True, text=True, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    line = json.loads(r.stdout.strip().splitlines()[-1])
+    assert line["impl"] == "reference" and line["metric"] == "jacobi2d_glups" and line["unit"] == "GLUP/s"
+    assert line["value"] > 0 and line["higher_is_better"] is True
+    cb = line["cpu_baseline"]
+    assert cb["kind"] == "oracle" and cb["cores"] >= 1 and cb["value"] == line["value"] and cb["sample"]
+    assert line["e2e"] == {"value": line["value"], "unit": "GLUP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
+
+
+def test_block_depth_follows_the_slab_per_gpu():
+    b = _bench_module()
+    from paper_conf_icppw_matzdf20_b200 import kernels as K
+    for name, shape, expect in (("hotspot2d", (16384, 16384), {1: 128, 2: 128, 4: 128, 8: 64}),
+                                ("heat3d", (1024, 1024, 1024), {1: 64, 2: 32, 4: 16, 8: 16})):
+        w = b.Workload.__new__(b.Workload)
+        w.name, w.shape, w.K, w.tile = name, shape, K, 0
+        for g, depth in expect.items():
+            w.gpus_used = g
+            assert w.block_depth() == depth, (name, g)
+            # the slab of each GPU is a whole number of blocks (balanced 1-D partitions)
+            assert (shape[0] // depth) % g == 0
+        w.tile = 40
+        assert w.block_depth() == 40          # --tile wins
