@@ -657,3 +657,26 @@ def test_heat3d_tb2_regions(d, h, w, zc, P):
         ora = _oracle_sets(regions.heat3d_tb2(box, d, h, w, zc, rows=16), {0: 4, 1: 4})   # 120 x 16 x zc blocks
         assert lib == ora
     abi.pk_finalize(ctx)
+
+
+# ------------------------------------------------------------------ degenerate cases
+def test_degenerate_buffers_and_grids():
+    """A zero-element buffer holds no segments; an empty grid launches nothing and moves
+    nothing; a one-block grid at P = 3 leaves two empty partitions (reading Q1), which are
+    not launched, and its stale bytes equal the shadow oracle's."""
+    ctx = host_ctx(3)
+    z = abi.pk_register_buffer(ctx, (0, 16), 4)
+    assert abi.pk_tracker_dump(ctx, z) == []
+    k = abi.pk_builtin_kernel(ctx, "jacobi2d")
+    u = np.arange(16, dtype=np.float32).reshape(4, 4)
+    b0 = abi.pk_register_buffer(ctx, (4, 4), 4, host_init=u)
+    b1 = abi.pk_register_buffer(ctx, (4, 4), 4, host_init=u)
+    abi.pk_launch_partitioned(ctx, k, (0, 1, 1), (32, 8, 1), [b0, b1, 4, 4], [4, 4])
+    st = abi.pk_get_stats(ctx)
+    assert st["kernel_launches"] == 0 and st["stale_bytes"] == 0 and st["moved_bytes"] == 0
+    abi.pk_finalize(ctx)
+    geom = ((1, 1, 1), (32, 8, 1), [4, 4])
+    st_, _ = _run_pair(3, "jacobi2d", {"u0": ((4, 4), 4, True), "u1": ((4, 4), 4, True)},
+                       [["u0", "u1", 4, 4], ["u1", "u0", 4, 4]], geom,
+                       lambda box: regions.jacobi2d(box, (32, 8), 4, 4))
+    assert st_["kernel_launches"] == 2                      # one partition launched per launch
