@@ -28,6 +28,26 @@ def main():
     K.heat3d_iterate(ph, 3)
     ph2 = K.heat3d_setup(ctx, h, zc=8, bdy=8, kernel="heat3d_regs")
     K.heat3d_iterate(ph2, 2)
+    for kern, kw in (("hotspot2d_tb2", {}), ("hotspot2d_tbk", {"sweeps": 4}), ("hotspot2d_tbk", {"sweeps": 8})):
+        pk = K.hotspot2d_setup(ctx, t, p, ty=16, kernel=kern, **kw)
+        K.hotspot2d_iterate(pk, 8 if kw.get("sweeps") == 8 else 4)
+    ph3 = K.heat3d_setup(ctx, h, zc=8, kernel="heat3d_tb2")
+    K.heat3d_iterate(ph3, 4)
+    # asynchronous host copies and the fused halo push
+    import torch
+    tp = torch.from_numpy(t).pin_memory()
+    abi.pk_copy_from_host_async(ctx, pr.tb[0], tp)
+    hb2 = K.hotspot2d_iterate(pr, 3)
+    ho = torch.empty(t.shape, dtype=torch.float32).pin_memory()
+    abi.pk_sync_to_host_async(ctx, hb2, ho)
+    abi.pk_synchronize(ctx)
+    abi.pk_set_mode(ctx, abi.PK_MODE_PUSH)
+    pp = K.hotspot2d_setup(ctx, t, p, ty=16, kernel="hotspot2d_tbk", sweeps=4)
+    K.hotspot2d_iterate(pp, 12)
+    ph4 = K.heat3d_setup(ctx, h, zc=8, kernel="heat3d_tb2")
+    K.heat3d_iterate(ph4, 6)
+    abi.pk_synchronize(ctx)
+    abi.pk_set_mode(ctx, 0)
     pos, vel = synth.nbody_bodies(3000)
     pn = K.nbody_setup(ctx, pos, vel)
     K.nbody_iterate(pn, 2)
