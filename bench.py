@@ -458,6 +458,7 @@ def main():
     base_mode = abi.PK_MODE_PUSH if args.push else 0
     abi.pk_set_mode(ctx, base_mode)
     w.gpus_used = world if world > 1 else len(devices)
+    devices_used = list(range(min(world, torch.cuda.device_count()))) if world > 1 else devices
     w.setup(ctx)
     for _ in range(args.warmup):
         w.step()
@@ -567,6 +568,15 @@ def main():
                       "copies": int(st["copies"]), "strided_copies": int(st["strided_copies"]),
                       "pushed_bytes": int(st["pushed_bytes"]),
                       "halo_copy_kernels": int(st["copy_kernels"])},
+        # inter-GPU bytes (NVLink/NVSwitch when the partitions sit on different GPUs): received
+        # per GPU per step, and that rate averaged over the whole step against 900 GB/s per
+        # direction -- a lower bound of the transfer-phase fraction (copies overlap kernels)
+        "nvlink": ({"bytes_per_gpu_per_step": (st["moved_bytes"] + st["pushed_bytes"]) / len(devices_used)
+                    / args.steps,
+                    "step_avg_frac_of_900GBs": (st["moved_bytes"] + st["pushed_bytes"]) / len(devices_used)
+                    / (elapsed_ms / 1e3) / 900e9,
+                    "note": "moved + pushed bytes between partitions on different GPUs; averaged over the step"}
+                   if len(devices_used) > 1 else None),
         "host_us_per_launch": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"]
                                + st["host_ns_issue"] + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
         "host_us_per_launch_phases": {k: st["host_ns_" + k] / 1e3 / max(1, st["launches"])
