@@ -356,7 +356,10 @@ def run_reference(args, w: Workload, rank):
     # torchrun sets OMP_NUM_THREADS=1 per worker; rank 0 runs the oracle alone on the host
     # cores (the other ranks do no work), so give its OpenMP runtime all of them
     if env_int("WORLD_SIZE", 1) > 1:
-        os.environ["OMP_NUM_THREADS"] = str(len(os.sched_getaffinity(0)))
+        n = len(os.sched_getaffinity(0))
+        os.environ["OMP_NUM_THREADS"] = str(n)
+        from oracle import kernels as ok
+        ok.lib().omp_set_num_threads(n)    # the OpenMP runtime may have read the variable already
     # each step is a bounded sample; warmup steps are run untimed
     for _ in range(args.warmup):
         cpu_oracle_rate(w, budget_s=1.0, max_iters=1)

@@ -42,3 +42,16 @@ def test_block_depth_follows_the_slab_per_gpu():
             assert (shape[0] // depth) % g == 0
         w.tile = 40
         assert w.block_depth() == 40          # --tile wins
+
+
+def test_reference_arm_under_torchrun_uses_all_host_cores():
+    """torchrun sets OMP_NUM_THREADS=1 per worker; rank 0 alone runs the oracle on all cores."""
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29647", os.path.join(ROOT, "bench.py"),
+                        "--gpus", "2", "--impl", "reference", "--workload", "jacobi2d", "--steps", "1",
+                        "--warmup", "1"], capture_output=True, text=True, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.strip().splitlines() if l.startswith("{")]
+    assert len(lines) == 1                     # rank 0 prints the one line
+    line = json.loads(lines[0])
+    assert line["n_gpus"] == 2 and line["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
