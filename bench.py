@@ -474,10 +474,13 @@ def main():
         sampler.start()
         time.sleep(0.3)
     # (1) the timed region.  Kernels of 100 us and more (every config but the latency-bound
-    # C1) are timed live in it: PK_MODE_TIME_KERNELS records CUDA events around every
-    # partition kernel on its own stream.  C1 (microsecond launches) keeps steady-state
-    # graph replay in the timed region and gets its kernel events from a second pass.
-    live = w.name != "jacobi2d"
+    # C1) are timed live in it when there is one partition per process: PK_MODE_TIME_KERNELS
+    # records CUDA events around every partition kernel on its own stream.  C1 (microsecond
+    # launches) keeps steady-state graph replay in the timed region and gets its kernel
+    # events from a second pass.
+    # Single-process P > 1 keeps graph replay (eager + events would add ~130 us of host time per
+    # launch at P = 8) and also takes the events from the second pass.
+    live = w.name != "jacobi2d" and (world > 1 or P == 1)
     if live:
         abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
     abi.pk_synchronize(ctx)
