@@ -52,6 +52,9 @@ constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + 2 * kNS * 8 + 128;
 #ifndef PK_HEATTB_PNS
 #define PK_HEATTB_PNS 256
 #endif
+#ifndef PK_HEATTB_MINB
+#define PK_HEATTB_MINB 3
+#endif
 
 __device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, int32_t z,
                                        uint64_t* bar) {
@@ -86,13 +89,8 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
                                         int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
                                         int lane, int warp, const PushList& push);
 
-// 3 CTAs/SM = 128 registers per thread.  __maxnreg__(136) (15 warps x 17 allocation units)
-// removed most spills but measured slower (1238-1264 vs 1331-1349 GLUP/s, scripts/gpu_run100.sh)
-#ifndef PK_HEATTB_MAXNREG
-#define PK_HEATTB_MAXNREG 128
-#endif
 template <bool PUSH>
-__global__ void __maxnreg__(PK_HEATTB_MAXNREG)
+__global__ void __launch_bounds__((kNW + 1) * 32, PK_HEATTB_MINB)
     k_heat3d_tb2(const __grid_constant__ CUtensorMap tm_u, float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
                  int64_t ZC, pk_partition part, PushList push) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
@@ -152,13 +150,9 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
     const int64_t col0 = c0 - 4 + cx;                 // its grid column
     const bool wclamp = col0 == 0, eclamp = col0 + 4 >= W;
     const bool store_col = lane >= 1 && lane <= 30 && col0 < W;
-    // 32-bit row / plane indices (the launch checks H, D < 2^30): fewer 64-bit compares and
-    // offsets in the loop under the 128-register cap (1331-1349 vs 1305-1307 GLUP/s, gpu_run100.sh)
-    const int Hi = (int)H, Di = (int)D;
-    const int gr1 = (int)y0 + kRW * warp - 1;         // grid row of sweep-1 row j = 0
+    const int64_t gr1 = y0 + kRW * warp - 1;          // grid row of sweep-1 row j = 0
     const int br1 = kRW * warp + 1;                   // box row of sweep-1 row j = 0
     const int64_t HW = H * W;
-    const int64_t rowcol = (int64_t)(gr1 + 1) * W + col0;   // the warp's first own row, the lane's first column
     float4 L1[3][kL1];                                // sweep-1 window, slot = plane sequence mod 3
     ptx::mbar_wait(&full[0], 0);
     ptx::mbar_wait(&full[1], 0);
@@ -178,7 +172,7 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
 #pragma unroll
             for (int j = 0; j < kL1; ++j) {
                 const int br = br1 + j;
-                const int gr = gr1 + j;
+                const int64_t gr = gr1 + j;
                 const float4 dn = *reinterpret_cast<const float4*>(sc + (br + 1) * kCols + cx);
                 const float4 zm = *reinterpret_cast<const float4*>(sm + br * kCols + cx);
                 const float4 zp = *reinterpret_cast<const float4*>(sp + br * kCols + cx);
@@ -191,19 +185,19 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
             // sweep 2 on plane seq q-2 = grid plane k0 + q - 4, own rows j = 1..4
             if (q >= 4) {
                 const int s0 = (2 + u - 2 + 3) % 3, sM = (2 + u - 3 + 3) % 3;
-                const int pz = (int)k0 + q - 4;
-                const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == Di - 1;   // sweep-1 planes outside: clamp
-                float* outp = uout + (int64_t)pz * HW + rowcol;
+                const int64_t pz = k0 + q - 4;
+                const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == D - 1;   // sweep-1 planes outside: clamp
+                float* outp = uout + pz * HW + (y0 + kRW * warp) * W + col0;
 #pragma unroll
                 for (int j = 1; j <= kRW; ++j) {
-                    const int gr = gr1 + j;
+                    const int64_t gr = gr1 + j;
                     const float4 c = L1[s0][j];
                     const float4 zm = zlo ? c : L1[sM][j];
                     const float4 zp = zhi ? c : L1[s1][j];
                     const float4 ym = (EDGE && gr == 0) ? c : L1[s0][j - 1];
-                    const float4 yp = (EDGE && gr == Hi - 1) ? c : L1[s0][j + 1];
+                    const float4 yp = (EDGE && gr == H - 1) ? c : L1[s0][j + 1];
                     const float4 o = sweep(c, zm, zp, ym, yp, wclamp, eclamp);
-                    if (store_col && (!EDGE || gr < Hi)) {   // interior blocks: every own row < H
+                    if (store_col && gr < H) {
                         *reinterpret_cast<float4*>(outp) = o;
                         if (PUSH) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);  // fused halo push
                     }
@@ -247,7 +241,6 @@ cudaError_t launch_heat3d_tb2(const LaunchInfo& li) {
     if (li.nscalars < 4) return cudaErrorInvalidValue;
     int64_t D = li.scalars[0], H = li.scalars[1], W = li.scalars[2], ZC = li.scalars[3];
     if (W % 4 || W < 4 || ZC < 1 || H < 1 || D < 1) return cudaErrorInvalidValue;
-    if (H >= (int64_t)1 << 30 || D >= (int64_t)1 << 30) return cudaErrorInvalidValue;   // 32-bit row/plane indices
     static std::once_flag once;
     static cudaError_t attr_err = cudaSuccess;
     std::call_once(once, [] {

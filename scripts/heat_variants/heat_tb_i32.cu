@@ -52,6 +52,9 @@ constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + 2 * kNS * 8 + 128;
 #ifndef PK_HEATTB_PNS
 #define PK_HEATTB_PNS 256
 #endif
+#ifndef PK_HEATTB_MINB
+#define PK_HEATTB_MINB 3
+#endif
 
 __device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, int32_t z,
                                        uint64_t* bar) {
@@ -86,10 +89,11 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
                                         int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
                                         int lane, int warp, const PushList& push);
 
-// 3 CTAs/SM = 128 registers per thread.  __maxnreg__(136) (15 warps x 17 allocation units)
-// removed most spills but measured slower (1238-1264 vs 1331-1349 GLUP/s, scripts/gpu_run100.sh)
+// 3 CTAs x 5 warps x 136 registers = 255 of the SM's 256 register-allocation units: capping
+// with __maxnreg__ instead of __launch_bounds__(.., 3) (which rounds to 128) removes the
+// consumer's local-memory spills
 #ifndef PK_HEATTB_MAXNREG
-#define PK_HEATTB_MAXNREG 128
+#define PK_HEATTB_MAXNREG 136
 #endif
 template <bool PUSH>
 __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
@@ -152,8 +156,8 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
     const int64_t col0 = c0 - 4 + cx;                 // its grid column
     const bool wclamp = col0 == 0, eclamp = col0 + 4 >= W;
     const bool store_col = lane >= 1 && lane <= 30 && col0 < W;
-    // 32-bit row / plane indices (the launch checks H, D < 2^30): fewer 64-bit compares and
-    // offsets in the loop under the 128-register cap (1331-1349 vs 1305-1307 GLUP/s, gpu_run100.sh)
+    // 32-bit row / plane indices (launch checks H, D < 2^31): 64-bit compares and
+    // offsets here had pushed the consumer past 128 registers into local-memory spills
     const int Hi = (int)H, Di = (int)D;
     const int gr1 = (int)y0 + kRW * warp - 1;         // grid row of sweep-1 row j = 0
     const int br1 = kRW * warp + 1;                   // box row of sweep-1 row j = 0
