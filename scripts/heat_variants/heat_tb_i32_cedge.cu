@@ -81,7 +81,7 @@ __device__ __forceinline__ float4 sweep(const float4& c, const float4& zm, const
     return o;
 }
 
-template <bool PUSH, bool EDGE>
+template <bool PUSH, bool EDGE, bool CEDGE>
 __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint64_t* empty, float* __restrict__ uout,
                                         int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
                                         int lane, int warp, const PushList& push);
@@ -138,19 +138,28 @@ __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
     // ---------------- consumers: blocks touching the grid's first/last row or plane apply
     // the replicate clamp of the intermediate sweep; interior blocks skip the selects
     const bool edge = y0 < 2 || y0 + kRows + 2 > H || k0 < 2 || k0 + ZC + 2 > D;
-    if (edge)
-        consume<PUSH, true>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
-    else
-        consume<PUSH, false>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+    // blocks touching the first/last column apply the x clamp; the others skip its selects
+    const bool cedge = c0 == 0 || c0 + kCols - 4 >= W;
+    if (edge) {
+        if (cedge)
+            consume<PUSH, true, true>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+        else
+            consume<PUSH, true, false>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+    } else {
+        if (cedge)
+            consume<PUSH, false, true>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+        else
+            consume<PUSH, false, false>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+    }
 }
 
-template <bool PUSH, bool EDGE>
+template <bool PUSH, bool EDGE, bool CEDGE>
 __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint64_t* empty, float* __restrict__ uout,
                                         int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
                                         int lane, int warp, const PushList& push) {
     const int cx = 4 * lane;                          // smem column of the lane's first column
     const int64_t col0 = c0 - 4 + cx;                 // its grid column
-    const bool wclamp = col0 == 0, eclamp = col0 + 4 >= W;
+    const bool wclamp = CEDGE && col0 == 0, eclamp = CEDGE && col0 + 4 >= W;
     const bool store_col = lane >= 1 && lane <= 30 && col0 < W;
     // 32-bit row / plane indices (the launch checks H, D < 2^30): fewer 64-bit compares and
     // offsets in the loop under the 128-register cap (1331-1349 vs 1305-1307 GLUP/s, gpu_run100.sh)
@@ -183,7 +192,7 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
                 const float4 zm = *reinterpret_cast<const float4*>(sm + br * kCols + cx);
                 const float4 zp = *reinterpret_cast<const float4*>(sp + br * kCols + cx);
                 const float4 ym = (EDGE && gr == 0) ? cc : up;        // replicate clamp (TMA zero-filled row -1)
-                const float4 yp = (EDGE && gr == H - 1) ? cc : dn;    // ... and row H
+                const float4 yp = (EDGE && gr == Hi - 1) ? cc : dn;   // ... and row H
                 L1[s1][j] = sweep(cc, zm, zp, ym, yp, wclamp, eclamp);
                 up = cc;
                 cc = dn;
