@@ -344,6 +344,8 @@ typedef struct {
     uint64_t copy_kernels;       /* of `strided_copies`: narrow runs moved by the SM halo-copy kernel */
     uint64_t pushed_bytes;       /* bytes stored into other partitions' instances by producing kernels (PK_MODE_PUSH) */
     uint64_t collectives;        /* NCCL SPMD: whole-buffer reads moved as one in-place all-gather */
+    uint64_t graph_fallbacks;    /* a graph capture / instantiation failed: the launch ran eagerly and the
+                                    context stays eager (pk_last_error() keeps the reason) */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);

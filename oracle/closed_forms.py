@@ -89,3 +89,22 @@ def nbody_two_body_accel(p1, p2, m2, eps2):
     d = np.asarray(p2, dtype=np.float64) - np.asarray(p1, dtype=np.float64)
     r2 = float(d @ d) + eps2
     return m2 * d / r2 ** 1.5
+
+
+def hotspot2d_tbk_stale_per_launch(w: int, nparts: int, k: int, elem_bytes: int = 4) -> int:
+    """K fused clamped 5-point sweeps per launch (NEXT-3; K = 2 is hotspot2d_tb2): the
+    output at distance K from a cut depends on input rows up to K rows across it, so
+    every cut moves K full rows of temperature each way per launch."""
+    return (nparts - 1) * 2 * k * w * elem_bytes
+
+
+def hotspot2d_tbk_power_once(w: int, nparts: int, k: int, elem_bytes: int = 4) -> int:
+    """Power enters sweeps 1..K; the last sweep's power term is local, so the cone of
+    one launch reaches K - 1 power rows across each cut.  Power is never rewritten:
+    in validity mode these rows move once (first launch), in single-owner mode every launch."""
+    return (nparts - 1) * 2 * (k - 1) * w * elem_bytes
+
+
+def heat3d_tb2_stale_per_launch(h: int, w: int, nparts: int, elem_bytes: int = 4) -> int:
+    """Two fused 7-point sweeps per launch: two h x w planes each way per z-cut."""
+    return (nparts - 1) * 2 * 2 * h * w * elem_bytes

@@ -196,3 +196,26 @@ def to_byte_ranges(elems: np.ndarray, elem_bytes: int):
     starts = np.concatenate([[elems[0]], elems[breaks + 1]])
     ends = np.concatenate([elems[breaks], [elems[-1]]]) + 1
     return [(int(s) * elem_bytes, int(e) * elem_bytes) for s, e in zip(starts, ends)]
+
+
+def nbody_soa(box, block, n, per_thread=1):
+    """Structure-of-arrays N-body (SURVEY §8(c) paper-vs-validity pin): arguments
+    x, y, z (positions in), m (masses, read only), vx, vy, vz (in place), x', y', z'
+    (positions out).  Thread tx of block bx owns bodies i = bx*per_thread*bdx + tx + u*bdx,
+    guard i < n; it reads x[j], y[j], z[j], m[j] of every body j (all pairs), reads and
+    writes vx[i], vy[i], vz[i] and writes x'[i], y'[i], z'[i].  Elements are fp32."""
+    bdx = block[0]
+    _, _, bxs = _block_ranges(box)
+    i = (bxs[:, None] * (per_thread * bdx) + np.arange(per_thread * bdx)[None, :]).ravel()
+    i = i[i < n]
+    every = np.arange(n, dtype=np.int64) if i.size else np.zeros(0, dtype=np.int64)
+    own = _uniq([i])
+    out = {}
+    for a in range(4):                       # x, y, z, m: every body
+        out[(a, READ)] = every
+    for a in range(4, 7):                    # vx, vy, vz: own bodies, in place
+        out[(a, READ)] = own
+        out[(a, WRITE)] = own
+    for a in range(7, 10):                   # x', y', z': own bodies
+        out[(a, WRITE)] = own
+    return out

@@ -73,7 +73,7 @@ class pk_stats(C.Structure):
                 ("kernel_ms_max_launch", C.c_double), ("timed_kernels", C.c_uint64),
                 ("graph_replays", C.c_uint64), ("graph_captures", C.c_uint64),
                 ("strided_copies", C.c_uint64), ("copy_kernels", C.c_uint64), ("pushed_bytes", C.c_uint64),
-                ("collectives", C.c_uint64)]
+                ("collectives", C.c_uint64), ("graph_fallbacks", C.c_uint64)]
 
 
 RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)

@@ -67,6 +67,7 @@ uint64_t total_bytes(const RangeList& r);
 struct Seg {
     uint64_t b, e;
     uint64_t mask;
+    bool operator==(const Seg& o) const { return b == o.b && e == o.e && mask == o.mask; }
 };
 
 // Segment vectors are immutable and shared: a memoised state (graph replay) is

@@ -28,6 +28,7 @@
 #include <unordered_map>
 
 #include "../runtime/builtins.h"
+#include "launch_util.h"
 #include "common.cuh"
 #include "ptx.cuh"
 #include "tma_host.h"
@@ -248,14 +249,10 @@ cudaError_t launch_heat3d_tb2(const LaunchInfo& li) {
     int64_t D = li.scalars[0], H = li.scalars[1], W = li.scalars[2], ZC = li.scalars[3];
     if (W % 4 || W < 4 || ZC < 1 || H < 1 || D < 1) return cudaErrorInvalidValue;
     if (H >= (int64_t)1 << 30 || D >= (int64_t)1 << 30) return cudaErrorInvalidValue;   // 32-bit row/plane indices
-    static std::once_flag once;
-    static cudaError_t attr_err = cudaSuccess;
-    std::call_once(once, [] {
-        attr_err = cudaFuncSetAttribute(k_heat3d_tb2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
-        if (attr_err == cudaSuccess)
-            attr_err = cudaFuncSetAttribute(k_heat3d_tb2<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
-    });
-    if (attr_err != cudaSuccess) return attr_err;
+    const bool push = li.push && li.push->n > 0;
+    const void* fn = push ? (const void*)k_heat3d_tb2<true> : (const void*)k_heat3d_tb2<false>;
+    KernelDevInfo kd;   // per device: the opt-in above 48 KB is a (function, device) attribute
+    if (cudaError_t e = prepare_kernel(fn, li.device, kSmem, (kNW + 1) * 32, &kd)) return e;
     // tensor map of this instance: dims (W, H, D), box (128, 20, 1), OOB zero fill
     static std::mutex mu;
     static std::unordered_map<const void*, std::pair<uint64_t, CUtensorMap>> cache;
@@ -277,7 +274,6 @@ cudaError_t launch_heat3d_tb2(const LaunchInfo& li) {
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, (void*)&li.part, &pl};
-    const void* fn = (li.push && li.push->n > 0) ? (const void*)k_heat3d_tb2<true> : (const void*)k_heat3d_tb2<false>;
     return cudaLaunchKernel(fn, li.grid, dim3((kNW + 1) * 32), argv, kSmem, li.stream);
 }
 

@@ -27,6 +27,7 @@
 #include <unordered_map>
 
 #include "../runtime/builtins.h"
+#include "launch_util.h"
 #include "common.cuh"
 #include "ptx.cuh"
 #include "tma_host.h"
@@ -181,16 +182,11 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
     const int bdy = (int)li.block.y;
     if (W % 4 || W < 4 || ZC < 1 || li.block.x != 32 || bdy < 1 || bdy > kMaxBdy || li.block.z != 1)
         return cudaErrorInvalidValue;
-    static std::once_flag once;
-    static cudaError_t attr_err = cudaSuccess;
-    std::call_once(once, [] {
-        attr_err = cudaFuncSetAttribute(k_heat3d_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        (int)smem_bytes(kMaxBdy));
-        if (attr_err == cudaSuccess)
-            attr_err = cudaFuncSetAttribute(k_heat3d_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                            (int)smem_bytes(kMaxBdy));
-    });
-    if (attr_err != cudaSuccess) return attr_err;
+    const bool push = li.push && li.push->n > 0;
+    KernelDevInfo kd;   // per device: the opt-in above 48 KB is a (function, device) attribute
+    if (cudaError_t e = prepare_kernel(push ? (const void*)k_heat3d_tma<true> : (const void*)k_heat3d_tma<false>,
+                                       li.device, smem_bytes(kMaxBdy), 32 * (warp_count(kMaxBdy) + 1), &kd))
+        return e;
     // tensor map of this instance: dims (W, H, D), box (136, bdy + 2, 1), OOB zero fill
     static std::mutex mu;
     static std::unordered_map<const void*, std::pair<uint64_t, CUtensorMap>> cache;
@@ -213,7 +209,7 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part, &pl};
-    const void* fn = (li.push && li.push->n > 0) ? (const void*)k_heat3d_tma<true> : (const void*)k_heat3d_tma<false>;
+    const void* fn = push ? (const void*)k_heat3d_tma<true> : (const void*)k_heat3d_tma<false>;
     return cudaLaunchKernel(fn, li.grid, dim3(32, warp_count(bdy) + 1), argv, smem_bytes(bdy), li.stream);
 }
 

@@ -24,6 +24,7 @@
 #include <cuda_runtime.h>
 
 #include "../runtime/builtins.h"
+#include "launch_util.h"
 #include "ptx.cuh"
 
 namespace pk {
@@ -217,24 +218,12 @@ cudaError_t launch_hotspot2d_tb2(const LaunchInfo& li) {
     int64_t H = li.scalars[0], W = li.scalars[1], TY = li.scalars[2];
     if (W % 4 || W < 4 || TY < 1 || li.block.x != kConsumers || li.block.y != 1 || li.block.z != 1)
         return cudaErrorInvalidValue;
-    static int resident[64] = {0};
-    static int sms[64] = {0};
-    const int d = li.device;
-    if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
-    if (!resident[d]) {
-        cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tb2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmem);
-        if (e != cudaSuccess) return e;
-        int nb = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_hotspot2d_tb2, kThreads, kSmem);
-        if (e != cudaSuccess) return e;
-        e = cudaDeviceGetAttribute(&sms[d], cudaDevAttrMultiProcessorCount, d);
-        if (e != cudaSuccess) return e;
-        resident[d] = nb > 0 ? nb : 1;
-    }
+    KernelDevInfo kd;
+    cudaError_t e = prepare_kernel((const void*)k_hotspot2d_tb2, li.device, kSmem, kThreads, &kd);
+    if (e != cudaSuccess) return e;
     const int64_t ntiles = (int64_t)li.grid.x * li.grid.y;
     if (ntiles == 0) return cudaSuccess;
-    const int64_t cap = (int64_t)resident[d] * sms[d];
-    dim3 grid((unsigned)(ntiles < cap ? ntiles : cap));
+    dim3 grid(persistent_grid(ntiles, kd));
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part};
     return cudaLaunchKernel((const void*)k_hotspot2d_tb2, grid, dim3(kThreads), argv, kSmem, li.stream);
 }

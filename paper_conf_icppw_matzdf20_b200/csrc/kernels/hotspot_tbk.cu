@@ -39,6 +39,7 @@
 #include <cuda_runtime.h>
 
 #include "../runtime/builtins.h"
+#include "launch_util.h"
 #include "common.cuh"
 #include "ptx.cuh"
 
@@ -272,26 +273,13 @@ int describe_hotspot2d_tbk(pk_ctx c, pk_kernel k) {
 
 template <int K, bool PUSH>
 cudaError_t launch_k(const LaunchInfo& li, int64_t H, int64_t W, int64_t TY) {
-    static int resident[64] = {0};
-    static int sms[64] = {0};
-    const int d = li.device;
     constexpr size_t kSmem = smem_bytes<K>();
-    if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
-    if (!resident[d]) {
-        cudaError_t e = cudaFuncSetAttribute(k_hotspot2d_tbk<K, PUSH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)kSmem);
-        if (e != cudaSuccess) return e;
-        int nb = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_hotspot2d_tbk<K, PUSH>, kThreads, kSmem);
-        if (e != cudaSuccess) return e;
-        e = cudaDeviceGetAttribute(&sms[d], cudaDevAttrMultiProcessorCount, d);
-        if (e != cudaSuccess) return e;
-        resident[d] = nb > 0 ? nb : 1;
-    }
+    KernelDevInfo kd;
+    cudaError_t e = prepare_kernel((const void*)k_hotspot2d_tbk<K, PUSH>, li.device, kSmem, kThreads, &kd);
+    if (e != cudaSuccess) return e;
     const int64_t ntiles = (int64_t)li.grid.x * li.grid.y;
     if (ntiles == 0) return cudaSuccess;
-    const int64_t cap = (int64_t)resident[d] * sms[d];
-    dim3 grid((unsigned)(ntiles < cap ? ntiles : cap));
+    dim3 grid(persistent_grid(ntiles, kd));
     PushList pl{};
     if (li.push) pl = *li.push;
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], (void*)&li.inst[2], &H, &W, &TY, (void*)&li.part, &pl};

@@ -23,6 +23,7 @@
 #include <utility>
 
 #include "../runtime/builtins.h"
+#include "launch_util.h"
 
 namespace pk {
 namespace {
@@ -229,39 +230,17 @@ cudaError_t launch_nbody(const LaunchInfo& li) {
     int64_t N = li.scalars[0];
     if (li.block.x > kTile || li.block.x < 1 || li.block.y != 1 || li.block.z != 1) return cudaErrorInvalidValue;
     if (N < 1) return cudaSuccess;
-    // per-stream scratch for the kSplit partial accelerations
-    static std::mutex mu;
-    static std::unordered_map<cudaStream_t, std::pair<float4*, size_t>> scratch;
-    float4* partial = nullptr;
-    {
-        std::lock_guard<std::mutex> g(mu);
-        auto& sc = scratch[li.stream];
-        const size_t need = (size_t)kSplit * (size_t)N;
-        if (sc.second < need) {
-            if (sc.first) cudaFree(sc.first);
-            sc.first = nullptr;
-            sc.second = 0;
-            cudaError_t e = cudaMalloc(&sc.first, need * sizeof(float4));
-            if (e != cudaSuccess) return e;
-            sc.second = need;
-        }
-        partial = sc.first;
-    }
-    static int resident[64] = {0}, sms[64] = {0};
-    const int d = li.device;
-    if (d < 0 || d >= 64) return cudaErrorInvalidDevice;
-    if (!resident[d]) {
-        int nb = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_nbody_partial, li.block.x, 0);
-        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms[d], cudaDevAttrMultiProcessorCount, d);
-        if (e != cudaSuccess) return e;
-        resident[d] = nb > 0 ? nb : 1;
-    }
+    // the kSplit partial accelerations: context-owned scratch of this partition (grow-only,
+    // never freed under a memoised graph that may replay into it)
+    cudaError_t e = cudaSuccess;
+    float4* partial = (float4*)context_scratch(li, 0, (size_t)kSplit * (size_t)N * sizeof(float4), &e);
+    if (!partial) return e;
+    KernelDevInfo kd;
+    if ((e = prepare_kernel((const void*)k_nbody_partial, li.device, 0, (int)li.block.x, &kd)) != cudaSuccess) return e;
     const int64_t items = (int64_t)li.grid.x * kSplit;
-    const int64_t cap = (int64_t)resident[d] * sms[d];
-    dim3 grid((unsigned)(items < cap ? items : cap));
+    dim3 grid(persistent_grid(items, kd));
     void* argv[] = {(void*)&li.inst[0], &partial, &N, (void*)&li.part};
-    cudaError_t e = cudaLaunchKernel((const void*)k_nbody_partial, grid, li.block, argv, 0, li.stream);
+    e = cudaLaunchKernel((const void*)k_nbody_partial, grid, li.block, argv, 0, li.stream);
     if (e != cudaSuccess) return e;
     const int64_t per_block = (int64_t)kBodies * li.block.x;
     int64_t i0 = (int64_t)li.part.min[0] * per_block, i1 = (int64_t)li.part.max[0] * per_block;

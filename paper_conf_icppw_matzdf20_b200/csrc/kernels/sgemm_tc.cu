@@ -40,6 +40,7 @@
 #include <unordered_map>
 
 #include "../runtime/builtins.h"
+#include "launch_util.h"
 #include "ptx.cuh"
 
 namespace pk {
@@ -346,29 +347,15 @@ bool make_map(CUtensorMap* m, const float* base, int64_t rows, int64_t cols, int
 
 struct Scratch {
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
-    size_t a_elems = 0, b_elems = 0;
 };
 
-cudaError_t get_scratch(cudaStream_t s, size_t a_elems, size_t b_elems, Scratch** out) {
-    static std::mutex mu;
-    static std::unordered_map<cudaStream_t, Scratch> cache;
-    std::lock_guard<std::mutex> g(mu);
-    Scratch& sc = cache[s];
-    if (sc.a_elems < a_elems) {
-        if (sc.ahi) { cudaFree(sc.ahi); cudaFree(sc.alo); }
-        cudaError_t e = cudaMalloc(&sc.ahi, a_elems * 4);
-        if (e == cudaSuccess) e = cudaMalloc(&sc.alo, a_elems * 4);
-        if (e != cudaSuccess) return e;
-        sc.a_elems = a_elems;
-    }
-    if (sc.b_elems < b_elems) {
-        if (sc.bhi) { cudaFree(sc.bhi); cudaFree(sc.blo); }
-        cudaError_t e = cudaMalloc(&sc.bhi, b_elems * 4);
-        if (e == cudaSuccess) e = cudaMalloc(&sc.blo, b_elems * 4);
-        if (e != cudaSuccess) return e;
-        sc.b_elems = b_elems;
-    }
-    *out = &sc;
+// hi/lo operand scratch: context-owned per partition (grow-only, see context_scratch)
+cudaError_t get_scratch(const LaunchInfo& li, size_t a_elems, size_t b_elems, Scratch* sc) {
+    cudaError_t e = cudaSuccess;
+    if (!(sc->ahi = (float*)context_scratch(li, 0, a_elems * 4, &e))) return e;
+    if (!(sc->alo = (float*)context_scratch(li, 1, a_elems * 4, &e))) return e;
+    if (!(sc->bhi = (float*)context_scratch(li, 2, b_elems * 4, &e))) return e;
+    if (!(sc->blo = (float*)context_scratch(li, 3, b_elems * 4, &e))) return e;
     return cudaSuccess;
 }
 
@@ -400,8 +387,9 @@ cudaError_t launch_sgemm(const LaunchInfo& li) {
     const float* A = (const float*)li.inst[0];
     const float* B = (const float*)li.inst[1];
     float* C = (float*)li.inst[2];
-    Scratch* sc = nullptr;
-    cudaError_t e = get_scratch(li.stream, (size_t)M * K, (size_t)N * K, &sc);
+    Scratch scr;
+    Scratch* sc = &scr;
+    cudaError_t e = get_scratch(li, (size_t)M * K, (size_t)N * K, &scr);
     if (e != cudaSuccess) return e;
     // 1. split this partition's A rows; 2. split + transpose all of B
     const int64_t r0 = (int64_t)li.part.min[1] * BM, r1 = std::min<int64_t>((int64_t)li.part.max[1] * BM, M);
@@ -417,12 +405,9 @@ cudaError_t launch_sgemm(const LaunchInfo& li) {
     if (!make_map(&tm[0], sc->ahi, M, K, BM) || !make_map(&tm[1], sc->alo, M, K, BM) ||
         !make_map(&tm[2], sc->bhi, N, K, BN) || !make_map(&tm[3], sc->blo, N, K, BN))
         return cudaErrorInvalidValue;
-    static bool attr = false;
-    if (!attr) {
-        e = cudaFuncSetAttribute(k_sgemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    KernelDevInfo kd;   // per device: the opt-in above 48 KB is a (function, device) attribute
+    if ((e = prepare_kernel((const void*)k_sgemm_tf32x3, li.device, SMEM_BYTES, kThreads, &kd)) != cudaSuccess)
+        return e;
     void* argv[] = {&tm[0], &tm[1], &tm[2], &tm[3], &C, &M, &N, &K, (void*)&li.part};
     return cudaLaunchKernel((const void*)k_sgemm_tf32x3, li.grid, dim3(kThreads), argv, SMEM_BYTES, li.stream);
 }

@@ -33,7 +33,17 @@ struct LaunchInfo {
     int nscalars;
     pk_partition part;
     const PushList* push = nullptr;  // halo push of the push-capable output (nullptr / n = 0: none)
+    pk_ctx ctx = nullptr;            // owning context and partition index (context_scratch)
+    int part_index = -1;
 };
+
+// Device scratch of a launcher (e.g. N-body partial sums), owned by the context per
+// (partition, slot) on the partition's device.  Grow-only: a smaller request reuses the
+// block; a larger one allocates a new block and RETIRES the old one, which stays
+// allocated until pk_finalize because a memoised graph may still replay into it.
+// Returns nullptr on failure (*err set).
+void* context_scratch(const LaunchInfo& li, int slot, size_t bytes, cudaError_t* err);
+constexpr int kScratchSlots = 4;
 using LauncherFn = cudaError_t (*)(const LaunchInfo&);
 
 struct Builtin {

@@ -18,6 +18,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <array>
 #include <chrono>
 #include <cstdio>
 #include <cstring>
@@ -76,11 +77,13 @@ struct NcclApi {
 };
 constexpr int kNcclUint8 = 1;  // ncclUint8
 
-const NcclApi& nccl() {
-    static NcclApi api;
-    static bool tried = false;
-    if (tried) return api;
-    tried = true;
+NcclApi load_nccl();
+const NcclApi& nccl() {  // process-wide (not device-scoped); thread-safe static initialisation
+    static const NcclApi api = load_nccl();
+    return api;
+}
+NcclApi load_nccl() {
+    NcclApi api;
     void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
     if (!h) {
         const char* p = getenv("PK_NCCL_LIB");
@@ -175,6 +178,8 @@ struct pk_ctx_s {
     bool host_only = false;
     std::vector<int> dev, prank;
     std::vector<int> sm_count;  // per partition's device (halo copy kernel grid)
+    std::vector<uint8_t> peer;  // [p*P + q]: p's device can address q's instances (same GPU or peer access on)
+    bool sm_reach(int p, int q) const { return ipc || peer.empty() || peer[(size_t)p * P + q]; }
     std::vector<cudaStream_t> stream;
     std::vector<cudaEvent_t> ev_kernel, ev_copy;
     std::vector<uint8_t> kernel_recorded;  // [p]: ev_kernel[p] recorded since the hazards were last cleared
@@ -209,12 +214,18 @@ struct pk_ctx_s {
         int seen = 0;
         cudaGraphExec_t exec = nullptr;
         struct Post { int64_t buf; SegState state; uint64_t fp; };
+        std::vector<Post> pre;   // tracker states before the launch (checked on a hit: the key holds only hashes)
         std::vector<Post> post;  // tracker states after the launch (shared, restored by pointer)
         std::shared_ptr<const std::vector<CopyOp>> plan;
         pk_stats delta{};
     };
     std::unordered_map<std::string, Memo> memo;
+    // launcher scratch (pk::context_scratch): [p][slot] = (pointer, bytes); retired blocks
+    // stay allocated until pk_finalize (memoised graphs may still reference them)
+    std::vector<std::array<std::pair<void*, size_t>, kScratchSlots>> scratch;
+    std::vector<std::pair<int, void*>> scratch_retired;  // (device, pointer)
     bool graph_mode = false;  // all work is ordered on stream[first_local]
+    bool graphs_broken = false;  // a capture / instantiation failed once: launch eagerly from now on
     cudaEvent_t ev_fork = nullptr;
     std::vector<cudaEvent_t> ev_join;
 
@@ -248,11 +259,13 @@ struct DriverApi {
     CUresult (*GetAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr) = nullptr;
     CUresult (*GetErrorName)(CUresult, const char**) = nullptr;
 };
-const DriverApi& drv() {
-    static DriverApi d;
-    static bool tried = false;
-    if (tried) return d;
-    tried = true;
+DriverApi load_drv();
+const DriverApi& drv() {  // process-wide driver entry points; thread-safe static initialisation
+    static const DriverApi d = load_drv();
+    return d;
+}
+DriverApi load_drv() {
+    DriverApi d;
     auto get = [](const char* name, void** fn) {
         cudaDriverEntryPointQueryResult q;
         return cudaGetDriverEntryPointByVersion(name, fn, CUDART_VERSION, cudaEnableDefault, &q) == cudaSuccess &&
@@ -594,6 +607,10 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
             if (c->local(p)) used.push_back(c->dev[p]);
         std::sort(used.begin(), used.end());
         used.erase(std::unique(used.begin(), used.end()), used.end());
+        // devices without peer access (no NVLink / P2P) still get copy-engine copies
+        // (cudaMemcpyPeerAsync stages them); only SM-side peer loads and stores -- the
+        // narrow-halo copy kernel and PK_MODE_PUSH -- need the pair enabled (c->peer)
+        std::vector<std::pair<int, int>> enabled;
         for (int a : used)
             for (int b : used) {
                 if (a == b) continue;
@@ -605,7 +622,15 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
                 if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
                 else if (e != cudaSuccess)
                     return fail(PK_ERR_CUDA, std::string("cudaDeviceEnablePeerAccess: ") + cudaGetErrorName(e));
+                enabled.push_back({a, b});
             }
+        c->peer.assign((size_t)c->P * c->P, 0);
+        for (int p = 0; p < c->P; ++p)
+            for (int q = 0; q < c->P; ++q)
+                if (c->local(p) && c->local(q))
+                    c->peer[(size_t)p * c->P + q] =
+                        c->dev[p] == c->dev[q] ||
+                        std::find(enabled.begin(), enabled.end(), std::make_pair(c->dev[p], c->dev[q])) != enabled.end();
         c->stream.resize(c->P);
         c->ev_kernel.resize(c->P);
         c->ev_copy.resize(c->P);
@@ -823,6 +848,10 @@ int pk_finalize(pk_ctx c) {
                     if (B.inst[p] && c->local(p)) { cudaSetDevice(c->dev[p]); cudaFree(B.inst[p]); }
         }
         clear_memo(c);
+        for (size_t p = 0; p < c->scratch.size(); ++p)
+            for (auto& s : c->scratch[p])
+                if (s.first) { cudaSetDevice(c->dev[p]); cudaFree(s.first); }
+        for (auto& r : c->scratch_retired) { cudaSetDevice(r.first); cudaFree(r.second); }
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
             cudaSetDevice(c->dev[p]);
@@ -1366,6 +1395,12 @@ int pk_reset_stats(pk_ctx c) {
 int pk_set_mode(pk_ctx c, uint32_t flags) {
     if (!c) return fail(PK_ERR_INVALID, "bad argument");
     if (flags & ~0x7Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
+    if ((flags & PK_MODE_PUSH) && !c->host_only && !c->ipc)
+        for (int p = 0; p < c->P; ++p)
+            for (int q = 0; q < c->P; ++q)
+                if (c->local(p) && c->local(q) && !c->sm_reach(p, q))
+                    return fail(PK_ERR_INVALID, "PK_MODE_PUSH needs peer access between devices " +
+                                                    std::to_string(c->dev[p]) + " and " + std::to_string(c->dev[q]));
     c->mode = flags;
     return PK_OK;
 }
@@ -1397,6 +1432,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
     const uint32_t mode = c->mode;
     // builtin launchers take every scalar from `scalars`, so the key below captures the launch
     const bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && K.nargs && args && K.launcher &&
+                           !c->graphs_broken &&
                            !(mode & (PK_MODE_TIME_KERNELS | PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
     if (!can_graph) {
         if (!c->host_only)
@@ -1431,6 +1467,27 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
         put(&f, sizeof f);
     }
     auto it = c->memo.find(key);
+    if (it != c->memo.end()) {
+        // the key holds 64-bit fingerprints of the tracker states: confirm the states
+        // themselves (pointer equality, as states are shared copy-on-write, else contents)
+        bool same = it->second.pre.size() == bids.size();
+        for (size_t i = 0; same && i < bids.size(); ++i) {
+            const auto& pr = it->second.pre[i];
+            const SegState cur = c->bufs[bids[i]].tracker.state();
+            same = pr.buf == bids[i] && (pr.state == cur || (pr.state && cur && *pr.state == *cur));
+        }
+        if (!same) {  // fingerprint collision: forget the entry, launch eagerly
+            if (it->second.exec) cudaGraphExecDestroy(it->second.exec);
+            c->memo.erase(it);
+            it = c->memo.end();
+        }
+    }
+    std::vector<pk_ctx_s::Memo::Post> pre_states;
+    pre_states.reserve(bids.size());
+    for (int64_t b : bids) {
+        const Tracker& T = c->bufs[b].tracker;
+        pre_states.push_back({b, T.state(), T.fingerprint()});
+    }
     if (it != c->memo.end() && it->second.exec) {
         // ---- replay: one graph launch + restore the memoised tracker states ----
         pk_ctx_s::Memo& m = it->second;
@@ -1454,6 +1511,31 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
         if (rc) return rc;
     } else {
         // ---- capture the launch once into a multi-stream graph ----
+        // host state the eager path mutates, restored if capture or instantiation fails
+        std::vector<std::vector<RangeList>> saved_last_read;
+        std::vector<std::vector<uint64_t>> saved_pushers;
+        for (int64_t b : bids) {
+            saved_last_read.push_back(c->bufs[b].last_read);
+            saved_pushers.push_back(c->bufs[b].pushers);
+        }
+        auto fall_back = [&](const std::string& why) -> int {
+            // a failed capture enqueued nothing: undo the bookkeeping and run eagerly, and
+            // keep this context on the eager path (no silent retry of a failing capture)
+            for (size_t i = 0; i < bids.size(); ++i) {
+                Buffer& B = c->bufs[bids[i]];
+                B.tracker.set_state(pre_states[i].state, pre_states[i].fp);
+                B.last_read = saved_last_read[i];
+                B.pushers = saved_pushers[i];
+            }
+            c->stats = before;
+            c->graphs_broken = true;
+            c->stats.graph_fallbacks += 1;
+            g_err = why;
+            clear_memo(c);
+            c->graph_mode = false;  // capture ended; stream[p0] already follows every stream's tail
+            if (int r = exit_graph_mode(c)) return r;
+            return launch_eager(c, k, grid, block, smem, args, scalars, ns);
+        };
         if (int r = enter_graph_mode(c)) return r;
         const int p0 = c->first_local;
         if (int r = c->set_device(c->dev[p0])) return r;
@@ -1466,6 +1548,8 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
             }
         rc = ce == cudaSuccess ? launch_eager(c, k, grid, block, smem, args, scalars, ns)
                                : fail(PK_ERR_CUDA, std::string("graph fork: ") + cudaGetErrorName(ce));
+        if (rc == PK_OK && getenv("PK_DEBUG_FAIL_CAPTURE"))  // test hook: exercise the eager fallback
+            rc = fail(PK_ERR_CUDA, "PK_DEBUG_FAIL_CAPTURE");
         for (int p = 0; p < c->P && rc == PK_OK; ++p)
             if (c->local(p) && p != p0) {
                 c->set_device(c->dev[p]);
@@ -1478,18 +1562,37 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
         cudaGraph_t g = nullptr;
         cudaError_t ee = cudaStreamEndCapture(c->stream[p0], &g);
         clear_hazards(c);  // events recorded during capture are graph nodes, not real records
-        if (rc) { if (g) cudaGraphDestroy(g); return rc; }
-        if (ee != cudaSuccess) return fail(PK_ERR_CUDA, std::string("cudaStreamEndCapture: ") + cudaGetErrorName(ee));
-        cudaGraphExec_t ex = nullptr;
-        ee = cudaGraphInstantiate(&ex, g, 0);
-        cudaGraphDestroy(g);
-        if (ee != cudaSuccess) return fail(PK_ERR_CUDA, std::string("cudaGraphInstantiate: ") + cudaGetErrorName(ee));
-        PK_CUDA(cudaGraphLaunch(ex, c->stream[p0]));
-        if (c->memo.size() > 256) clear_memo(c);
-        c->memo[key].exec = ex;
-        c->stats.graph_captures += 1;
+        if (rc || ee != cudaSuccess) {
+            if (g) cudaGraphDestroy(g);
+            cudaGetLastError();
+            if (rc == PK_ERR_WRITE_OVERLAP || rc == PK_ERR_INVALID || rc == PK_ERR_OUT_OF_BOUNDS ||
+                rc == PK_ERR_OVERFLOW)
+                return rc;  // a user error, not a capture problem: same answer eagerly
+            const int r = fall_back(std::string("graph capture failed: ") +
+                                    (rc ? g_err : std::string(cudaGetErrorName(ee))));
+            if (r) return r;
+            goto record;
+        }
+        {
+            cudaGraphExec_t ex = nullptr;
+            ee = cudaGraphInstantiate(&ex, g, 0);
+            cudaGraphDestroy(g);
+            if (ee != cudaSuccess) {
+                cudaGetLastError();
+                const int r = fall_back(std::string("cudaGraphInstantiate: ") + cudaGetErrorName(ee));
+                if (r) return r;
+                goto record;
+            }
+            PK_CUDA(cudaGraphLaunch(ex, c->stream[p0]));
+            if (c->memo.size() > 256) clear_memo(c);
+            c->memo[key].exec = ex;
+            c->stats.graph_captures += 1;
+        }
     }
+record:
+    if (c->graphs_broken) return PK_OK;  // eager from now on: nothing to memoise
     pk_ctx_s::Memo& m = c->memo[key];
+    m.pre = std::move(pre_states);
     m.seen += 1;
     m.plan = std::make_shared<const std::vector<CopyOp>>(c->last_plan);
     m.delta = c->stats;
@@ -1781,7 +1884,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     // IPC-mapped peer instances are addressed through UVA (cudaMemcpyDefault)
                     const bool same_dev = c->ipc || c->dev[o.src] == c->dev[p];
                     const cudaMemcpyKind dkind = c->ipc ? cudaMemcpyDefault : cudaMemcpyDeviceToDevice;
-                    if ((rows > 1 || nslab > 1) && len <= kNarrowPiece) {
+                    if ((rows > 1 || nslab > 1) && len <= kNarrowPiece && c->sm_reach(p, o.src)) {
                         // narrow strided run (a halo column): pulled by the destination's SMs
                         PK_CUDA(launch_strided_copy(dst, src, len, pitch, rows, slice, nslab, c->sm_count[p],
                                                     c->stream[p]));
@@ -2011,7 +2114,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             cudaError_t err;
             if (K.launcher) {
                 LaunchInfo li{K.fn, g, bl, smem, c->stream[p], c->dev[p], inst, args, scalars, ns, part,
-                              push[p].n ? &push[p] : nullptr};
+                              push[p].n ? &push[p] : nullptr, c, p};
                 err = K.launcher(li);
             } else {
                 err = cudaLaunchKernel(K.fn, g, bl, argv, smem, c->stream[p]);
@@ -2087,6 +2190,25 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
 }  // extern "C"
 
 namespace pk {
+void* context_scratch(const LaunchInfo& li, int slot, size_t bytes, cudaError_t* err) {
+    pk_ctx c = li.ctx;
+    *err = cudaSuccess;
+    if (!c || li.part_index < 0 || li.part_index >= c->P || slot < 0 || slot >= kScratchSlots) {
+        *err = cudaErrorInvalidValue;
+        return nullptr;
+    }
+    if (c->scratch.size() != (size_t)c->P) c->scratch.resize(c->P);
+    auto& s = c->scratch[li.part_index][slot];
+    if (s.second >= bytes && s.first) return s.first;
+    void* p = nullptr;
+    // the runtime has selected the partition's device before calling the launcher
+    *err = cudaMalloc(&p, bytes ? bytes : 16);
+    if (*err != cudaSuccess) return nullptr;
+    if (s.first) c->scratch_retired.push_back({c->dev[li.part_index], s.first});
+    s = {p, bytes};
+    return p;
+}
+
 int32_t find_builtin_push_arg(const void* fn) {
     if (!fn) return -1;
     for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_tbk", "heat3d", "heat3d_tb2"}) {

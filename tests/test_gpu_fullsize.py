@@ -92,7 +92,7 @@ def test_c3_heat_fullsize_sampled(kernel):
     del res
     rms = float(np.sqrt(np.mean(g[::8, ::8, ::8].astype(np.float64) ** 2)))
     rng = np.random.default_rng(11)
-    pts = [tuple(int(x) for x in rng.integers(0, 1024, 3)) for _ in range(6)]
+    pts = [tuple(int(x) for x in rng.integers(0, 1024, 3)) for _ in range(60)]
     pts += [(0, 0, 0), (1023, 1023, 1023), (511, 512, 0), (512, 3, 1020)]
     bad = []
     for (z, y, x) in pts:
@@ -120,8 +120,8 @@ def test_c4_sgemm_fullsize_sampled():
     assert np.array_equal(res[1], res[2])
     g = res[1]
     rng = np.random.default_rng(5)
-    rows = rng.integers(0, m, 256)
-    cols = rng.integers(0, n, 256)
+    rows = rng.integers(0, m, 65536)          # >= 65,536 sampled fp64 entries
+    cols = rng.integers(0, n, 65536)
     rows[:4] = [0, 0, m - 1, m - 1]
     cols[:4] = [0, n - 1, 0, n - 1]
     o = ok.gemm_entries(a, b, rows, cols)
@@ -129,6 +129,8 @@ def test_c4_sgemm_fullsize_sampled():
     rms = float(np.sqrt(np.mean(g[::64, ::64].astype(np.float64) ** 2)))
     err = np.abs(gs - o) / np.maximum(np.abs(o), rms)
     assert float(err.max()) <= 1e-4, float(err.max())
+    # every row block and column block of the tile grid is sampled at least once
+    assert len(np.unique(rows // 128)) == m // 128 and len(np.unique(cols // 256)) == n // 256
 
 
 # ------------------------------------------------------------------ C5 N-body 2^20, 10 steps
@@ -162,3 +164,35 @@ def test_c5_nbody_fullsize_sampled_per_step():
     assert np.array_equal(p4, final1[0]) and np.array_equal(v4, final1[1])
     # every step every partition reads all positions: (P-1)/P of the 16 MiB array each
     assert st["stale_bytes"] == st["moved_bytes"] == steps * nb * 16 * 3
+
+
+# ------------------------------------------------------------------ N-body: full 10-step FP64 run, N = 16,384
+def test_nbody_16384_ten_steps_vs_fp64_oracle():
+    """SURVEY §8(c) N-body pin: the whole 10-step trajectory of 16,384 bodies against the
+    fp64 oracle run end to end (no per-step re-seeding).  Positions within 1e-5 (Q18).
+    Velocities: fp32 STORAGE alone (the fp64 oracle with its state rounded to fp32 after
+    every step) already departs by 1.04e-5 on one component of 49,152 (close encounters
+    amplify it; reading Q26), so they are held to 1e-5 normwise and 5e-5 per
+    element.  P = 4 is bit-identical to P = 1."""
+    nb, steps = 16384, 10
+    pos, vel = synth.nbody_bodies(nb)
+    res = {}
+    for P in (1, 4):
+        ctx = gpu_ctx(P)
+        pr = K.nbody_setup(ctx, pos, vel)
+        pb, vb = K.nbody_iterate(pr, steps)
+        res[P] = (fetch(ctx, pb, pos.shape), fetch(ctx, vb, vel.shape))
+        st = abi.pk_get_stats(ctx)
+        abi.pk_finalize(ctx)
+        if P > 1:
+            assert st["stale_bytes"] == st["moved_bytes"] == steps * nb * 16 * (P - 1)
+    assert np.array_equal(res[1][0], res[4][0]) and np.array_equal(res[1][1], res[4][1])
+    gp, gv = res[1]
+    op, ov = ok.nbody(pos, vel, steps)
+    good_x, ex = rel_ok(gp[:, :3], op[:, :3], 1e-5)
+    assert good_x, ex
+    assert np.array_equal(gp[:, 3], pos[:, 3])          # masses untouched
+    dv = gv[:, :3].astype(np.float64) - ov[:, :3]
+    assert np.linalg.norm(dv) <= 1e-5 * np.linalg.norm(ov[:, :3])
+    good_v, evv = rel_ok(gv[:, :3], ov[:, :3], 5e-5)
+    assert good_v, evv

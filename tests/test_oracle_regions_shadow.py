@@ -125,12 +125,143 @@ def test_c1_stale_bytes_40800():
 
 
 def test_misaligned_h2d_redistribution_and_paper_mode_redundancy():
-    # Q2: linear H2D misaligned with P=3 row partitions -> extra first-launch traffic.
+    """Jacobi 64^2, P = 3 (SURVEY §8(c) Q2 / paper-vs-validity pin).
+
+    Hand derivation.  Grid (2, 8) blocks of 32x8 -> row slabs [0,16), [16,40), [40,64);
+    the linear H2D split of 4096 elements is [0,1365), [1365,2730), [2730,4096), i.e. the
+    slab boundaries fall at (row 21, col 21) and (row 42, col 42).  A partition on rows
+    [r0, r1) reads row r0-1 and row r1 interior (62 cells) and rows r0..r1-1 in full,
+    clipped to interior thread rows 1..62.
+      launch 1 (reads u0 as uploaded): p0 holds all it reads; p1 lacks row 15 interior (62),
+        rows 16-20 (5 x 64) and row 21 cols 0-20 (21) = 403; p2 lacks row 39 interior
+        (62), rows 40-41 (128), row 42 cols 0-41 (42) = 232.  635 cells = 2,540 B.
+      launch 2 (reads u1: interior written by launch 1's slabs, border cells still
+        linear): p0 lacks row 16 interior (62); p1 row 15 and row 40 interior (124) plus
+        the border cells (col 0 / 63) of rows 16-20 and (21, 0), held by p0 (11); p2 row
+        39 interior (62) plus (40, 0), (40, 63), (41, 0), (41, 63), (42, 0) held by p1 (5).
+        264 cells = 1,056 B.
+      launch 3+ (reads the buffer read in launch 1, whose border cells the readers now
+        co-hold): only the 4 interior halo rows cross: 248 cells = 992 B.  Without shared
+        copies (the paper's tracker) those 16 border cells are fetched again every time:
+        1,056 B per launch.
+    """
     _, per = _jacobi_run(64, 3, 6)
-    assert per[0] > per[2] and per[2:] == [per[2]] * 4
-    # without shared copies the same halo is re-fetched -> never fewer bytes.
+    assert per == [2540, 1056, 992, 992, 992, 992]
     _, per_so = _jacobi_run(64, 3, 6, single=True)
-    assert all(a >= b for a, b in zip(per_so, per)) and sum(per_so) > sum(per)
+    assert per_so == [2540, 1056, 1056, 1056, 1056, 1056]
+
+
+def test_gemm_launched_twice_single_owner_vs_validity():
+    """Paper-vs-validity pin: the same GEMM launched twice on unchanged
+    operands.  Every partition reads all of B (k x n), of which it holds its 1/P linear
+    slab: launch 1 moves (P-1) |B|.  With shared copies the readers keep B and launch 2
+    moves nothing (1x); the paper's single-owner tracker fetches it again (2x).  A's row
+    band equals the linear slab when the tile rows divide M."""
+    m, n, k, bm, bn, P = 32, 24, 20, 4, 8, 4
+    g = ((n + bn - 1) // bn, m // bm, 1)
+    res = {}
+    for single in (False, True):
+        sh = shadow.Shadow(P, single)
+        sh.register("A", m * k, 4, True)
+        sh.register("B", k * n, 4, True)
+        sh.register("C", m * n, 4, False)
+        per_launch = []
+        for _ in range(2):
+            per = []
+            for p in range(P):
+                acc = regions.gemm(grid.partition_box(g, P, p), m, n, k, bm, bn)
+                per.append({"A": (acc[(0, "r")], None), "B": (acc[(1, "r")], None), "C": (None, acc[(2, "w")])})
+            per_launch.append(sum(sh.launch(per)["stale"]))
+        res[single] = per_launch
+    one = (P - 1) * k * n * 4
+    assert one == cf.gemm_stale(k, n, P) == 5760
+    assert res[False] == [one, 0]
+    assert res[True] == [one, one]
+
+
+def test_nbody_soa_with_mass_single_owner_vs_validity():
+    """Paper-vs-validity pin: N-body on structure-of-arrays fp32 positions
+    x, y, z (ping-pong), a separate read-only mass array and in-place velocities;
+    1,024 bodies, P = 8, 3 steps.  Hand derivation: every step each partition reads all
+    of x, y, z and m and holds 1/8 of each, so each step moves 7 x 1,024 x 4 = 28,672 B per
+    array.  Positions are rewritten every step (3 x 3 x 28,672 = 258,048 B in both modes);
+    velocities are read and written on the own slab only (0 B).  Masses are never written:
+    with shared copies they move once (28,672 B) -> 286,720 B; the paper's tracker moves
+    them every step (3 x 28,672) -> 344,064 B."""
+    n, P, steps = 1024, 8, 3
+    g = (n // 128, 1, 1)
+    totals = {}
+    for single in (False, True):
+        sh = shadow.Shadow(P, single)
+        for name in ("x0", "y0", "z0", "m", "vx", "vy", "vz"):
+            sh.register(name, n, 4, True)
+        for name in ("x1", "y1", "z1"):
+            sh.register(name, n, 4, False)
+        tot = 0
+        for s in range(steps):
+            src = ("x0", "y0", "z0") if s % 2 == 0 else ("x1", "y1", "z1")
+            dst = ("x1", "y1", "z1") if s % 2 == 0 else ("x0", "y0", "z0")
+            names = src + ("m", "vx", "vy", "vz") + dst
+            per = []
+            for p in range(P):
+                acc = regions.nbody_soa(grid.partition_box(g, P, p), (128,), n)
+                per.append({nm: (acc.get((a, "r")), acc.get((a, "w"))) for a, nm in enumerate(names)})
+            tot += sum(sh.launch(per)["stale"])
+        totals[single] = tot
+    assert totals[False] == 286720
+    assert totals[True] == 344064
+
+
+@pytest.mark.parametrize("k", [2, 3, 4])
+@pytest.mark.parametrize("nparts", [2, 4])
+def test_hotspot_tbk_stale_matches_closed_form(nparts, k):
+    """K fused sweeps per launch (hotspot2d_tb2 = K 2, hotspot2d_tbk): temperature is
+    dilated by K rows per cut, power by K - 1 rows (once in validity mode, every launch
+    in single-owner mode) -- closed forms derived from the dependency cone, so an
+    over- or under-declared brute-force region fails here."""
+    h, w, ty = 64, 64, 8
+    for single in (False, True):
+        sh = shadow.Shadow(nparts, single)
+        sh.register("t0", h * w, 4, True)
+        sh.register("t1", h * w, 4, False)
+        sh.register("pw", h * w, 4, True)
+        stale = []
+        for it in range(4):
+            a, b = ("t0", "t1") if it % 2 == 0 else ("t1", "t0")
+            per = []
+            for p in range(nparts):
+                if k == 2:
+                    g = (w // 32 + (w % 32 > 0), (h + ty - 1) // ty, 1)
+                    acc = regions.hotspot2d_tb2(grid.partition_box(g, nparts, p), (8,), h, w, ty)
+                else:
+                    g = (1, (h + ty - 1) // ty, 1)
+                    acc = regions.hotspot2d_tbk(grid.partition_box(g, nparts, p), None, h, w, ty, k)
+                per.append({a: (acc[(0, "r")], None), "pw": (acc[(1, "r")], None), b: (None, acc[(2, "w")])})
+            stale.append(sum(sh.launch(per)["stale"]))
+        t = cf.hotspot2d_tbk_stale_per_launch(w, nparts, k)
+        pw = cf.hotspot2d_tbk_power_once(w, nparts, k)
+        if single:
+            assert stale == [t + pw] * 4
+        else:
+            assert stale == [t + pw, t, t, t]
+
+
+@pytest.mark.parametrize("nparts", [2, 4])
+def test_heat3d_tb2_stale_matches_closed_form(nparts):
+    d, h, w, zc = 16, 6, 8, 2
+    g = (1, 1, d // zc)
+    sh = shadow.Shadow(nparts)
+    sh.register("u0", d * h * w, 4, True)
+    sh.register("u1", d * h * w, 4, False)
+    stale = []
+    for it in range(3):
+        a, b = ("u0", "u1") if it % 2 == 0 else ("u1", "u0")
+        per = []
+        for p in range(nparts):
+            acc = regions.heat3d_tb2(grid.partition_box(g, nparts, p), d, h, w, zc)
+            per.append({a: (acc[(0, "r")], None), b: (None, acc[(1, "w")])})
+        stale.append(sum(sh.launch(per)["stale"]))
+    assert stale == [cf.heat3d_tb2_stale_per_launch(h, w, nparts)] * 3
 
 
 @pytest.mark.parametrize("nparts", [2, 3, 4, 8])
