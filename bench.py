@@ -14,11 +14,14 @@ streams via pk_timer_begin/end) with the inputs resident in HBM; ``e2e`` adds
 the H2D upload (pk_copy_from_host from pinned memory) and the D2H gather
 (pk_sync_to_host) of every step and is wall-clock timed.
 
-Process model: one host process drives every GPU of the box, as
-in the paper.  Under torchrun with N ranks, rank 0 drives N
-partitions on devices 0..N-1 and the other ranks only join the barriers; the
-reported time is the max over ranks.  ``--parts P`` runs P partitions as
-virtual devices on the visible GPUs (transfers then are D2D copies).
+Process model: without torchrun one host process drives every
+partition, as in the paper: ``--gpus N`` puts one partition on each
+of devices 0..N-1.  Under torchrun with N ranks (the driver's multi-GPU launch)
+every rank owns ONE partition on its own GPU (SPMD, NEXT-4): the ranks replay the
+same deterministic plan and pull their stale ranges from the holders' CUDA-IPC-
+mapped instances (``--transport nccl``: NCCL send/recv); the reported time is the
+max over ranks.  ``--parts P`` runs P partitions as virtual devices on the visible
+GPUs (transfers then are D2D copies).
 """
 from __future__ import annotations
 

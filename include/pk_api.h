@@ -346,6 +346,11 @@ typedef struct {
     uint64_t collectives;        /* NCCL SPMD: whole-buffer reads moved as one in-place all-gather */
     uint64_t graph_fallbacks;    /* a graph capture / instantiation failed: the launch ran eagerly and the
                                     context stays eager (pk_last_error() keeps the reason) */
+    double graph_launch_ms;      /* PK_MODE_TIME_KERNELS with graph replay: CUDA events around each replayed
+                                    launch on its stream (copies + partition kernels of that launch) */
+    uint64_t timed_graph_launches;
+    uint64_t host_cpu_ns;        /* thread CPU time spent inside pk_launch_partitioned (excludes time the
+                                    thread is descheduled; a driver spinning on a full launch queue still counts) */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);
@@ -356,7 +361,9 @@ enum {
     PK_MODE_NO_TRANSFERS = 1u << 1,  /* beta of §9.2: resolve + track, do not copy */
     PK_MODE_NO_TRACKING = 1u << 2,   /* gamma of §9.2: no resolution, no tracker, no copies */
     PK_MODE_GLOBAL_BARRIER = 1u << 3,/* literal all_devs_synchronize() between sync and launch (Fig. 4 l. 8) */
-    PK_MODE_TIME_KERNELS = 1u << 4,  /* CUDA events around every partition kernel -> pk_stats.kernel_ms */
+    PK_MODE_TIME_KERNELS = 1u << 4,  /* CUDA events around every eagerly launched partition kernel ->
+                                        pk_stats.kernel_ms, and around every replayed graph launch ->
+                                        pk_stats.graph_launch_ms (graph replay stays on) */
     PK_MODE_NO_GRAPHS = 1u << 5,     /* disable steady-state graph replay (see pk_launch_partitioned) */
     PK_MODE_PUSH = 1u << 6           /* fused halo push, see below */
 };
@@ -381,9 +388,28 @@ enum {
  * the memoised post-launch tracker states instead of re-planning and re-issuing every
  * CUDA call -- the host overhead the paper measures as "patterns".
  * Active for single-process contexts (any number of local partitions, P = 1 included), unless
- * PK_MODE_TIME_KERNELS, PK_MODE_GLOBAL_BARRIER or PK_MODE_NO_GRAPHS is set. */
+ * PK_MODE_GLOBAL_BARRIER or PK_MODE_NO_GRAPHS is set.  If a capture or instantiation
+ * fails, that launch runs eagerly (its bookkeeping rolled back first) and the context
+ * stays eager (pk_stats.graph_fallbacks). */
 int pk_set_mode(pk_ctx ctx, uint32_t flags);
 uint32_t pk_get_mode(pk_ctx ctx);
+
+/* ---------------------------------------------------------------- access recording
+ * The paper requires write maps to be exact and lets read maps over-approximate
+ * (P:L568-571); tools of the VAST kind clone the kernel to mark the memory it touches
+ * (P:L1231-1236).  libpk_trace.so (the same sources built with -DPK_TRACE_ACCESS, see
+ * paper_conf_icppw_matzdf20_b200/build.py) records, at 4-byte granularity, every global
+ * address each builtin kernel FETCHES (plain loads, and the in-bounds part of every TMA
+ * copy -- halo over-fetch included) and every address it STORES, into one bitmap per
+ * (instance, kind); bit w of word w/32 stands for bytes [4w, 4w+4) of the instance.
+ * Single device; tests only.  In libpk.so these calls fail with PK_ERR_STATE. */
+int pk_trace_available(void);                 /* 1 in libpk_trace.so, 0 in libpk.so */
+int pk_trace_reset(pk_ctx ctx);               /* synchronise, clear every bitmap and the stray count */
+/* kind 0 = fetched, 1 = stored; words[ceil(bytes/4/32)] receives the bitmap of instance
+ * `part` of `buf` (synchronises first); PK_ERR_INVALID if nwords is too small. */
+int pk_trace_fetch(pk_ctx ctx, pk_buf buf, int part, int kind, uint32_t* words, uint64_t nwords);
+/* accesses that hit no registered instance or ran past its end (must be 0) */
+int pk_trace_stray(pk_ctx ctx, uint64_t* out);
 
 const char* pk_last_error(void);
 const char* pk_version(void);

@@ -10,7 +10,9 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libpk.so")
+# PK_TRACE_ACCESS=1 selects the access-recording build libpk_trace.so (tests of the
+# declared descriptors against what the kernels touch; pk_trace_* below)
+LIB_PATH = os.path.join(_HERE, "libpk_trace.so" if os.environ.get("PK_TRACE_ACCESS") == "1" else "libpk.so")
 
 PK_OK = 0
 PK_ERR = {-1: "PK_ERR_INVALID", -2: "PK_ERR_CUDA", -3: "PK_ERR_NCCL", -4: "PK_ERR_OOM",
@@ -73,7 +75,8 @@ class pk_stats(C.Structure):
                 ("kernel_ms_max_launch", C.c_double), ("timed_kernels", C.c_uint64),
                 ("graph_replays", C.c_uint64), ("graph_captures", C.c_uint64),
                 ("strided_copies", C.c_uint64), ("copy_kernels", C.c_uint64), ("pushed_bytes", C.c_uint64),
-                ("collectives", C.c_uint64), ("graph_fallbacks", C.c_uint64)]
+                ("collectives", C.c_uint64), ("graph_fallbacks", C.c_uint64),
+                ("graph_launch_ms", C.c_double), ("timed_graph_launches", C.c_uint64), ("host_cpu_ns", C.c_uint64)]
 
 
 RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)
@@ -138,11 +141,16 @@ def lib():
         "pk_get_stats": [C.c_void_p, C.POINTER(pk_stats)],
         "pk_reset_stats": [C.c_void_p],
         "pk_set_mode": [C.c_void_p, C.c_uint32],
+        "pk_trace_reset": [C.c_void_p],
+        "pk_trace_fetch": [C.c_void_p, C.c_int64, C.c_int, C.c_int, C.POINTER(C.c_uint32), C.c_uint64],
+        "pk_trace_stray": [C.c_void_p, C.POINTER(C.c_uint64)],
     }
     for name, args in sig.items():
         f = getattr(L, name)
         f.argtypes = args
         f.restype = C.c_int
+    L.pk_trace_available.argtypes = []
+    L.pk_trace_available.restype = C.c_int
     L.pk_builtin_fn.argtypes = [C.c_char_p]
     L.pk_builtin_fn.restype = C.c_void_p
     L.pk_get_mode.argtypes = [C.c_void_p]
@@ -441,3 +449,30 @@ def affine_access(dims) -> pk_affine_access:
     for i, d in enumerate(dims):
         a.dim[i] = d
     return a
+
+
+# ---------------------------------------------------------------- access recording (libpk_trace.so)
+def pk_trace_available() -> bool:
+    return bool(lib().pk_trace_available())
+
+
+def pk_trace_reset(ctx):
+    _check(lib().pk_trace_reset(ctx), "pk_trace_reset")
+
+
+def pk_trace_fetch(ctx, buf, part, kind, nbytes):
+    """Bitmap of instance `part` of `buf` (kind 0 fetched, 1 stored) as a bool array with
+    one entry per 4-byte word of the instance."""
+    import numpy as np
+    nw = nbytes // 4
+    words = np.zeros((nw + 31) // 32, dtype=np.uint32)
+    _check(lib().pk_trace_fetch(ctx, buf, part, kind, words.ctypes.data_as(C.POINTER(C.c_uint32)), words.size),
+           "pk_trace_fetch")
+    bits = np.unpackbits(words.view(np.uint8), bitorder="little")
+    return bits[:nw].astype(bool)
+
+
+def pk_trace_stray(ctx) -> int:
+    v = C.c_uint64(0)
+    _check(lib().pk_trace_stray(ctx, C.byref(v)), "pk_trace_stray")
+    return int(v.value)

@@ -5,6 +5,7 @@
 #include <stdint.h>
 
 #include "pk_api.h"
+#include "trace.cuh"
 
 namespace pk {
 namespace dev {
@@ -50,12 +51,18 @@ namespace dev {
 __device__ __forceinline__ void push4(const PushList& pl, uint64_t off, const float4& v) {
 #pragma unroll
     for (int i = 0; i < kMaxPush; ++i)
-        if (i < pl.n && off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float4*>(pl.dst[i] + off) = v;
+        if (i < pl.n && off >= pl.lo[i] && off < pl.hi[i]) {
+            *reinterpret_cast<float4*>(pl.dst[i] + off) = v;
+            PK_TRACE_W((const void*)(pl.dst[i] + off), 16);
+        }
 }
 __device__ __forceinline__ void push1(const PushList& pl, uint64_t off, float v) {
 #pragma unroll
     for (int i = 0; i < kMaxPush; ++i)
-        if (i < pl.n && off >= pl.lo[i] && off < pl.hi[i]) *reinterpret_cast<float*>(pl.dst[i] + off) = v;
+        if (i < pl.n && off >= pl.lo[i] && off < pl.hi[i]) {
+            *reinterpret_cast<float*>(pl.dst[i] + off) = v;
+            PK_TRACE_W((const void*)(pl.dst[i] + off), 4);
+        }
 }
 }  // namespace dev
 }  // namespace pk

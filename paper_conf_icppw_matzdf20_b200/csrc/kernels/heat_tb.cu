@@ -29,6 +29,7 @@
 
 #include "../runtime/builtins.h"
 #include "launch_util.h"
+#include "trace.cuh"
 #include "common.cuh"
 #include "ptx.cuh"
 #include "tma_host.h"
@@ -95,7 +96,7 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
 template <bool PUSH>
 __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
     k_heat3d_tb2(const __grid_constant__ CUtensorMap tm_u, float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
-                 int64_t ZC, pk_partition part, PushList push) {
+                 int64_t ZC, pk_partition part, PushList push, const float* uin_trace) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     // 128-B aligned ring; pointer arithmetic on the shared array (not a uintptr_t round
     // trip) keeps the shared address space visible, so the loads below are LDS, not LD
@@ -132,6 +133,7 @@ __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
             p = p < 0 ? 0 : (p >= D ? D - 1 : p);
             ptx::mbar_arrive_expect_tx(&full[s], bytes);
             tma_3d(ring + (size_t)s * kSlot, &tm_u, (int32_t)(c0 - 4), (int32_t)(y0 - 2), (int32_t)p, &full[s]);
+            PK_TRACE_BOX(uin_trace, H, W, c0 - 4, kCols, y0 - 2, kBoxRows, p);
         }
         return;
     }
@@ -206,6 +208,7 @@ __device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint6
                     const float4 o = sweep(c, zm, zp, ym, yp, wclamp, eclamp);
                     if (store_col && (!EDGE || gr < Hi)) {   // interior blocks: every own row < H
                         *reinterpret_cast<float4*>(outp) = o;
+                        PK_TRACE_W(outp, 16);
                         if (PUSH) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);  // fused halo push
                     }
                     outp += W;
@@ -273,7 +276,7 @@ cudaError_t launch_heat3d_tb2(const LaunchInfo& li) {
     }
     PushList pl{};
     if (li.push) pl = *li.push;
-    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, (void*)&li.part, &pl};
+    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, (void*)&li.part, &pl, (void*)&li.inst[0]};
     return cudaLaunchKernel(fn, li.grid, dim3((kNW + 1) * 32), argv, kSmem, li.stream);
 }
 

@@ -28,6 +28,7 @@
 
 #include "../runtime/builtins.h"
 #include "launch_util.h"
+#include "trace.cuh"
 #include "common.cuh"
 #include "ptx.cuh"
 #include "tma_host.h"
@@ -61,7 +62,8 @@ __device__ __forceinline__ void tma_3d(void* dst, const CUtensorMap* map, int32_
 template <bool PUSH>
 __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUtensorMap tm_u,
                                                     float* __restrict__ uout, int64_t D, int64_t H, int64_t W,
-                                                    int64_t ZC, int bdy, pk_partition part, PushList push) {
+                                                    int64_t ZC, int bdy, pk_partition part, PushList push,
+                                                    const float* uin_trace) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
     // bdy = logical rows per block; warps 0..nw-1 consume (kRPW rows each), warp nw produces
@@ -98,6 +100,7 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUt
             p = p < 0 ? 0 : (p >= D ? D - 1 : p);
             ptx::mbar_arrive_expect_tx(&full[s], bytes);
             tma_3d(smem + (size_t)s * sb, &tm_u, (int32_t)(c0 - kHalo), (int32_t)(i0 - 1), (int32_t)p, &full[s]);
+            PK_TRACE_BOX(uin_trace, H, W, c0 - kHalo, kRowF, i0 - 1, bdy + 2, p);
         }
         return;
     }
@@ -143,6 +146,7 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUt
             o.z = c.z + kAlpha * ((zm.z + zp.z + ym.z + yp.z + c.y + c.w) - 6.0f * c.z);
             o.w = c.w + kAlpha * ((zm.w + zp.w + ym.w + yp.w + c.z + ev) - 6.0f * c.w);
             *reinterpret_cast<float4*>(uout + kout + i * W + j0) = o;
+            PK_TRACE_W(uout + kout + i * W + j0, 16);
             if (PUSH) dev::push4(push, (uint64_t)(kout + i * W + j0) * 4u, o);  // fused halo push
         }
         __syncwarp();
@@ -208,7 +212,7 @@ cudaError_t launch_heat3d_tma(const LaunchInfo& li) {
     int bdy_arg = bdy;
     PushList pl{};
     if (li.push) pl = *li.push;
-    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part, &pl};
+    void* argv[] = {&tm, (void*)&li.inst[1], &D, &H, &W, &ZC, &bdy_arg, (void*)&li.part, &pl, (void*)&li.inst[0]};
     const void* fn = push ? (const void*)k_heat3d_tma<true> : (const void*)k_heat3d_tma<false>;
     return cudaLaunchKernel(fn, li.grid, dim3(32, warp_count(bdy) + 1), argv, smem_bytes(bdy), li.stream);
 }

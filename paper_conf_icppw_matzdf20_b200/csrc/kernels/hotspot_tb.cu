@@ -25,6 +25,7 @@
 
 #include "../runtime/builtins.h"
 #include "launch_util.h"
+#include "trace.cuh"
 #include "ptx.cuh"
 
 namespace pk {
@@ -88,6 +89,8 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
                 ptx::mbar_arrive_expect_tx(&full[s], 2u * bytes);
                 ptx::bulk_g2s(st + toff, tin + row * W + tlo, bytes, &full[s]);
                 ptx::bulk_g2s(st + kRowF + toff, pw + row * W + tlo, bytes, &full[s]);
+                PK_TRACE_R(tin + row * W + tlo, bytes);
+                PK_TRACE_R(pw + row * W + tlo, bytes);
             }
         }
         return;
@@ -174,7 +177,10 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tb2(const float* __restr
                 o.y = hs(s1B.y, n4.y, s4.y, s1B.z, s1B.x, pA.y);
                 o.z = hs(s1B.z, n4.z, s4.z, s1B.w, s1B.y, pA.z);
                 o.w = hs(s1B.w, n4.w, s4.w, e2, s1B.z, pA.w);
-                if (active) *reinterpret_cast<float4*>(outp) = o;
+                if (active) {
+                    *reinterpret_cast<float4*>(outp) = o;
+                    PK_TRACE_W(outp, 16);
+                }
                 outp += dW;
             }
             // ---- rotate the register windows; stage seq t-2 is no longer read by this warp

@@ -154,6 +154,7 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
                 } else if (t >= 2 * K) {
                     if (store) {
                         *reinterpret_cast<float4*>(outp) = o;
+                        PK_TRACE_W(outp, 16);
                         if (PUSH) dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
                     }
                     outp += dW;
@@ -214,6 +215,8 @@ __global__ void __launch_bounds__(kThreads, K <= 4 ? PK_TBK_MINB : PK_TBK8_MINB)
                 ptx::mbar_arrive_expect_tx(&full[s], 2u * bytes);
                 ptx::bulk_g2s(st + toff, tin + row * W + tlo, bytes, &full[s]);
                 ptx::bulk_g2s(st + G::RowF + toff, pw + row * W + tlo, bytes, &full[s]);
+                PK_TRACE_R(tin + row * W + tlo, bytes);
+                PK_TRACE_R(pw + row * W + tlo, bytes);
             }
         }
         return;

@@ -86,7 +86,11 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restr
                 float* st = ring + (size_t)s * kStageFloats;
                 ptx::mbar_arrive_expect_tx(&full[s], tbytes + (need_p ? pbytes : 0u));
                 ptx::bulk_g2s(st + toff, tin + row * W + tlo, tbytes, &full[s]);
-                if (need_p) ptx::bulk_g2s(st + kTRow, pw + row * W + c0, pbytes, &full[s]);
+                PK_TRACE_R(tin + row * W + tlo, tbytes);
+                if (need_p) {
+                    ptx::bulk_g2s(st + kTRow, pw + row * W + c0, pbytes, &full[s]);
+                    PK_TRACE_R(pw + row * W + c0, pbytes);
+                }
             }
         }
         return;
@@ -128,6 +132,7 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restr
                 o.w = hs(c.w, a.w, b.w, ev, c.z, p.w);
                 const int64_t row = down ? r0 - 1 + t : rend - t;
                 *reinterpret_cast<float4*>(tout + row * W + j0) = o;
+                PK_TRACE_W(tout + row * W + j0, 16);
                 if (PUSH) dev::push4(push, (uint64_t)(row * W + j0) * 4u, o);  // fused halo push
             }
             __syncwarp();

@@ -24,6 +24,7 @@
 
 #include "../runtime/builtins.h"
 #include "launch_util.h"
+#include "trace.cuh"
 
 namespace pk {
 namespace {
@@ -129,6 +130,7 @@ __global__ void __launch_bounds__(256, PK_NBODY_MINB) k_nbody_partial(const floa
         for (int u = 0; u < kBodies; ++u) {
             const int64_t i = base + threadIdx.x + u * (int64_t)blockDim.x;
             const float4 p = i < N ? pin[i] : make_float4(0.f, 0.f, 0.f, 0.f);
+            if (i < N) PK_TRACE_R(pin + i, 16);
             px[u] = pk2(p.x, p.x);  // broadcast pairs: ptxas uses the scalar .F32 operand form
             py[u] = pk2(p.y, p.y);
             pz[u] = pk2(p.z, p.z);
@@ -147,6 +149,8 @@ __global__ void __launch_bounds__(256, PK_NBODY_MINB) k_nbody_partial(const floa
                     const int64_t j = t0 + 2 * s;
                     const float4 q0 = j < c1 ? pin[j] : make_float4(0.f, 0.f, 0.f, 0.f);  // m = 0 pads add 0
                     const float4 q1 = j + 1 < c1 ? pin[j + 1] : make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (j < c1) PK_TRACE_R(pin + j, 16);
+                    if (j + 1 < c1) PK_TRACE_R(pin + j + 1, 16);
                     sh[2 * s] = make_float4(q0.x, q1.x, q0.y, q1.y);
                     sh[2 * s + 1] = make_float4(q0.z, q1.z, q0.w, q1.w);
                 }
@@ -204,11 +208,15 @@ __global__ void __launch_bounds__(256) k_nbody_final(const float4* __restrict__ 
     }
     const float4 p = pin[i];
     float4 v = vel[i];
+    PK_TRACE_R(pin + i, 16);
+    PK_TRACE_R(vel + i, 16);
     v.x = fmaf(a.x, kDt, v.x);
     v.y = fmaf(a.y, kDt, v.y);
     v.z = fmaf(a.z, kDt, v.z);
     vel[i] = v;
     pout[i] = make_float4(fmaf(v.x, kDt, p.x), fmaf(v.y, kDt, p.y), fmaf(v.z, kDt, p.z), p.w);
+    PK_TRACE_W(vel + i, 16);
+    PK_TRACE_W(pout + i, 16);
 }
 
 int describe_nbody(pk_ctx c, pk_kernel k) {

@@ -41,6 +41,7 @@
 
 #include "../runtime/builtins.h"
 #include "launch_util.h"
+#include "trace.cuh"
 #include "ptx.cuh"
 
 namespace pk {
@@ -72,27 +73,32 @@ __global__ void k_split_rows(const float* __restrict__ x, float* __restrict__ hi
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         float h, l;
         split_tf32(x[base + i], h, l);
+        PK_TRACE_R(x + base + i, 4);
         hi[base + i] = h;
         lo[base + i] = l;
     }
 }
 
-// B (K x N, row-major) -> Bt_hi, Bt_lo (N x K, row-major) via 32 x 32 smem tiles
+// B (K x N, row-major) -> Bt_hi, Bt_lo (N x K, row-major) via 32 x 32 smem tiles, for the
+// column band [nb0, nb1) the partition's C tiles read (n0 = nb0 + 32 blockIdx.x)
 __global__ void k_split_transp(const float* __restrict__ b, float* __restrict__ bthi, float* __restrict__ btlo,
-                               int64_t K, int64_t N) {
+                               int64_t K, int64_t N, int64_t nb0, int64_t nb1) {
     __shared__ float th[32][33], tl[32][33];
-    const int64_t k0 = blockIdx.y * 32, n0 = blockIdx.x * 32;
+    const int64_t k0 = blockIdx.y * 32, n0 = nb0 + blockIdx.x * 32;
     for (int r = threadIdx.y; r < 32; r += blockDim.y) {
         const int64_t k = k0 + r, n = n0 + threadIdx.x;
         float h = 0.f, l = 0.f;
-        if (k < K && n < N) split_tf32(b[k * N + n], h, l);
+        if (k < K && n < nb1) {
+            split_tf32(b[k * N + n], h, l);
+            PK_TRACE_R(b + k * N + n, 4);
+        }
         th[r][threadIdx.x] = h;
         tl[r][threadIdx.x] = l;
     }
     __syncthreads();
     for (int r = threadIdx.y; r < 32; r += blockDim.y) {
         const int64_t n = n0 + r, k = k0 + threadIdx.x;
-        if (k < K && n < N) {
+        if (k < K && n < nb1) {
             bthi[n * K + k] = th[threadIdx.x][r];
             btlo[n * K + k] = tl[threadIdx.x][r];
         }
@@ -300,9 +306,13 @@ __global__ void __launch_bounds__(kThreads, 1)
             for (int c = 0; c < EPI_COLS; c += 4) {
                 if (c0 + c + 4 <= N && (N % 4) == 0) {
                     *reinterpret_cast<float4*>(dst + c) = make_float4(sum[c], sum[c + 1], sum[c + 2], sum[c + 3]);
+                    PK_TRACE_W(dst + c, 16);
                 } else {
                     for (int i = 0; i < 4; ++i)
-                        if (c0 + c + i < N) dst[c + i] = sum[c + i];
+                        if (c0 + c + i < N) {
+                            dst[c + i] = sum[c + i];
+                            PK_TRACE_W(dst + c + i, 4);
+                        }
                 }
             }
         }
@@ -397,8 +407,10 @@ cudaError_t launch_sgemm(const LaunchInfo& li) {
         k_split_rows<<<1184, 256, 0, li.stream>>>(A, sc->ahi, sc->alo, r0, r1, K);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
-    dim3 tg((unsigned)((N + 31) / 32), (unsigned)((K + 31) / 32));
-    k_split_transp<<<tg, dim3(32, 8), 0, li.stream>>>(B, sc->bhi, sc->blo, K, N);
+    // only the B column band of this partition's C tiles (tile partitions split N too)
+    const int64_t nb0 = (int64_t)li.part.min[0] * BN, nb1 = std::min<int64_t>((int64_t)li.part.max[0] * BN, N);
+    dim3 tg((unsigned)((nb1 - nb0 + 31) / 32), (unsigned)((K + 31) / 32));
+    if (nb1 > nb0) k_split_transp<<<tg, dim3(32, 8), 0, li.stream>>>(B, sc->bhi, sc->blo, K, N, nb0, nb1);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     // 3. tensor-core GEMM over the partition's C tiles
     CUtensorMap tm[4];

@@ -36,8 +36,13 @@ __global__ void __launch_bounds__(256) k_jacobi2d(const float* __restrict__ in, 
     if (i < 1 || i > H - 2 || j < 1 || j > W - 2) return;
     const float n = in[(i - 1) * W + j], s = in[(i + 1) * W + j];
     const float w = in[i * W + j - 1], e = in[i * W + j + 1];
+    PK_TRACE_R(in + (i - 1) * W + j, 4);
+    PK_TRACE_R(in + (i + 1) * W + j, 4);
+    PK_TRACE_R(in + i * W + j - 1, 4);
+    PK_TRACE_R(in + i * W + j + 1, 4);
     const float v = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(__fadd_rn(n, s), w), e));
     out[i * W + j] = v;
+    PK_TRACE_W(out + i * W + j, 4);
     if (PUSH) dev::push1(push, (uint64_t)(i * W + j) * 4u, v);  // fused halo push
 }
 
@@ -78,13 +83,18 @@ struct Row4 {
     float w, e; // column j0-1 (lane 0 only) and j0+4 (lane 31 only), clamped
 };
 
+// we = the row will be a centre row (its W/E halo columns are used); halo rows above and
+// below the block are only read straight up / down (no diagonal reads, as declared)
 __device__ __forceinline__ Row4 load_row(const float* __restrict__ t, int64_t r, int64_t W, int64_t jl,
-                                         int64_t jw, int64_t je, int lane) {
+                                         int64_t jw, int64_t je, int lane, bool we) {
     Row4 x;
     const float* row = t + r * W;
     x.c = ld_stream4(row + jl);
-    x.w = lane == 0 ? ld_nc(row + jw) : 0.f;
-    x.e = lane == 31 ? ld_nc(row + je) : 0.f;
+    x.w = we && lane == 0 ? ld_nc(row + jw) : 0.f;
+    x.e = we && lane == 31 ? ld_nc(row + je) : 0.f;
+    PK_TRACE_R(row + jl, 16);
+    if (we && lane == 0) PK_TRACE_R(row + jw, 4);
+    if (we && lane == 31) PK_TRACE_R(row + je, 4);
     return x;
 }
 
@@ -110,17 +120,19 @@ __global__ void __launch_bounds__(128) k_hotspot2d(const float* __restrict__ tin
     const int64_t jw = jl > 0 ? jl - 1 : 0, je = jl + 4 < W ? jl + 4 : W - 1;
     const bool west_edge = jl == 0, east_edge = jl + 4 >= W;
 
-    Row4 N = load_row(tin, r0 > 0 ? r0 - 1 : 0, W, jl, jw, je, lane);
-    Row4 C = load_row(tin, r0, W, jl, jw, je, lane);
-    Row4 S = load_row(tin, r0 + 1 < H ? r0 + 1 : H - 1, W, jl, jw, je, lane);
+    Row4 N = load_row(tin, r0 > 0 ? r0 - 1 : 0, W, jl, jw, je, lane, false);
+    Row4 C = load_row(tin, r0, W, jl, jw, je, lane, true);
+    Row4 S = load_row(tin, r0 + 1 < H ? r0 + 1 : H - 1, W, jl, jw, je, lane, r0 + 1 < r1);
     float4 P = ld_stream4(pw + r0 * W + jl);
+    PK_TRACE_R(pw + r0 * W + jl, 16);
     for (int64_t r = r0; r < r1; ++r) {
         // prefetch the row after next and the next power row
         Row4 S2 = S;
         float4 P2 = P;
         if (r + 1 < r1) {
-            S2 = load_row(tin, r + 2 < H ? r + 2 : H - 1, W, jl, jw, je, lane);
+            S2 = load_row(tin, r + 2 < H ? r + 2 : H - 1, W, jl, jw, je, lane, r + 2 < r1);
             P2 = ld_stream4(pw + (r + 1) * W + jl);
+            PK_TRACE_R(pw + (r + 1) * W + jl, 16);
         }
         float wv = __shfl_up_sync(0xffffffffu, C.c.w, 1);
         float ev = __shfl_down_sync(0xffffffffu, C.c.x, 1);
@@ -133,7 +145,10 @@ __global__ void __launch_bounds__(128) k_hotspot2d(const float* __restrict__ tin
         o.y = hs(C.c.y, N.c.y, S.c.y, C.c.z, C.c.x, P.y);
         o.z = hs(C.c.z, N.c.z, S.c.z, C.c.w, C.c.y, P.z);
         o.w = hs(C.c.w, N.c.w, S.c.w, ev, C.c.z, P.w);
-        if (active) st4(tout + r * W + j0, o);
+        if (active) {
+            st4(tout + r * W + j0, o);
+            PK_TRACE_W(tout + r * W + j0, 16);
+        }
         N = C;
         C = S;
         S = S2;
@@ -183,6 +198,9 @@ __device__ __forceinline__ Pl4 load_pl(const float* __restrict__ u, int64_t off,
     x.c = ld_stream4(u + off + jl);
     x.w = lane == 0 ? ld_nc(u + off + jw) : 0.f;
     x.e = lane == 31 ? ld_nc(u + off + je) : 0.f;
+    PK_TRACE_R(u + off + jl, 16);
+    if (lane == 0) PK_TRACE_R(u + off + jw, 4);
+    if (lane == 31) PK_TRACE_R(u + off + je, 4);
     return x;
 }
 
@@ -222,14 +240,20 @@ __global__ void __launch_bounds__(1024) k_heat3d(const float* __restrict__ uin, 
     Pl4 Zc = load_pl(uin, k0 * HW + rowc, jl, jw, je, lane);
     Pl4 Zp = load_pl(uin, (k0 + 1 < D ? k0 + 1 : D - 1) * HW + rowc, jl, jw, je, lane);
     float4 Hr = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (halo_lo || halo_hi) Hr = ld_stream4(uin + k0 * HW + rowh + jl);
+    if (halo_lo || halo_hi) {
+        Hr = ld_stream4(uin + k0 * HW + rowh + jl);
+        PK_TRACE_R(uin + k0 * HW + rowh + jl, 16);
+    }
     int buf = 0;
     for (int64_t k = k0; k < k1; ++k) {
         Pl4 Zn = Zp;
         float4 Hn = Hr;
         if (k + 1 < k1) {
             Zn = load_pl(uin, (k + 2 < D ? k + 2 : D - 1) * HW + rowc, jl, jw, je, lane);
-            if (halo_lo || halo_hi) Hn = ld_stream4(uin + (k + 1) * HW + rowh + jl);
+            if (halo_lo || halo_hi) {
+                Hn = ld_stream4(uin + (k + 1) * HW + rowh + jl);
+                PK_TRACE_R(uin + (k + 1) * HW + rowh + jl, 16);
+            }
         }
         ysh[buf][ty + 1][lane] = Zc.c;
         if (halo_lo) ysh[buf][0][lane] = Hr;
@@ -250,7 +274,10 @@ __global__ void __launch_bounds__(1024) k_heat3d(const float* __restrict__ uin, 
         o.y = c.y + kAlpha * ((Zm.c.y + Zp.c.y + Ym.y + Yp.y + c.x + c.z) - 6.0f * c.y);
         o.z = c.z + kAlpha * ((Zm.c.z + Zp.c.z + Ym.z + Yp.z + c.y + c.w) - 6.0f * c.z);
         o.w = c.w + kAlpha * ((Zm.c.w + Zp.c.w + Ym.w + Yp.w + c.z + ev) - 6.0f * c.w);
-        if (active) st4(uout + k * HW + rowc + j0, o);
+        if (active) {
+            st4(uout + k * HW + rowc + j0, o);
+            PK_TRACE_W(uout + k * HW + rowc + j0, 16);
+        }
         Zm = Zc;
         Zc = Zp;
         Zp = Zn;

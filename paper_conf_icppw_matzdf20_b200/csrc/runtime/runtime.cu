@@ -20,6 +20,8 @@
 #include <algorithm>
 #include <array>
 #include <chrono>
+#include <ctime>
+#include <cstddef>
 #include <cstdio>
 #include <cstring>
 #include <memory>
@@ -27,11 +29,66 @@
 #include <unordered_map>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../core/host_core.h"
+#include "../kernels/trace.cuh"
 #include "builtins.h"
 #include "pk_api.h"
 
 using namespace pk;
+
+// ---- access recording (libpk_trace.so only; kernels/trace.cuh) ----
+#ifdef PK_TRACE_ACCESS
+#include <mutex>
+__device__ pk::trace::Table g_pk_trace;
+namespace {
+struct TraceInst {
+    const void* base;
+    uint64_t bytes;
+    uint32_t* bits[2];
+};
+std::mutex g_trace_mu;
+std::vector<TraceInst> g_trace;  // every registered instance of every context (one device)
+cudaError_t trace_upload() {
+    pk::trace::Table t{};
+    t.n = (int32_t)g_trace.size();
+    for (size_t i = 0; i < g_trace.size(); ++i) {
+        t.base[i] = (uint64_t)(uintptr_t)g_trace[i].base;
+        t.bytes[i] = g_trace[i].bytes;
+        t.bits[i][0] = g_trace[i].bits[0];
+        t.bits[i][1] = g_trace[i].bits[1];
+    }
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(g_pk_trace, &t, sizeof t);
+    return e;
+}
+cudaError_t trace_add(const void* base, uint64_t bytes) {
+    std::lock_guard<std::mutex> g(g_trace_mu);
+    if (g_trace.size() >= (size_t)pk::trace::kMaxInst) return cudaErrorMemoryAllocation;
+    TraceInst ti{base, bytes, {nullptr, nullptr}};
+    const size_t wb = ((bytes / 4 + 31) / 32) * 4;
+    for (int k = 0; k < 2; ++k) {
+        cudaError_t e = cudaMalloc(&ti.bits[k], wb ? wb : 4);
+        if (e == cudaSuccess) e = cudaMemset(ti.bits[k], 0, wb ? wb : 4);
+        if (e != cudaSuccess) return e;
+    }
+    g_trace.push_back(ti);
+    return trace_upload();
+}
+void trace_remove(const void* base) {
+    std::lock_guard<std::mutex> g(g_trace_mu);
+    for (size_t i = 0; i < g_trace.size(); ++i)
+        if (g_trace[i].base == base) {
+            cudaFree(g_trace[i].bits[0]);
+            cudaFree(g_trace[i].bits[1]);
+            g_trace.erase(g_trace.begin() + i);
+            trace_upload();
+            return;
+        }
+}
+}  // namespace
+#endif
 
 namespace {
 
@@ -50,6 +107,27 @@ int fail(const Status& s) { return fail(s.code, s.msg); }
             return fail(PK_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorName(e_) + \
                                          " (" + cudaGetErrorString(e_) + ")");          \
     } while (0)
+
+// NVTX ranges per phase of the launch replacement (SURVEY.md §5 tracing): visible in
+// Nsight Systems / ncu --nvtx; NVTX v3 is header-only and costs a branch without a tool.
+struct NvtxPhase {
+    bool open = false;
+    explicit NvtxPhase(const char* name) { next(name); }
+    void next(const char* name) {
+        if (open) nvtxRangePop();
+        nvtxRangePushA(name);
+        open = true;
+    }
+    ~NvtxPhase() {
+        if (open) nvtxRangePop();
+    }
+};
+
+uint64_t thread_cpu_ns() {
+    timespec ts;
+    clock_gettime(CLOCK_THREAD_CPUTIME_ID, &ts);
+    return (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+}
 
 uint64_t now_ns() {
     return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
@@ -166,6 +244,7 @@ struct TimedLaunch {
     cudaEvent_t start, stop;
     int part;
     uint64_t launch_id;
+    bool graph = false;  // events around a replayed graph launch (whole launch), not one kernel
 };
 
 }  // namespace
@@ -226,6 +305,7 @@ struct pk_ctx_s {
     std::vector<std::pair<int, void*>> scratch_retired;  // (device, pointer)
     bool graph_mode = false;  // all work is ordered on stream[first_local]
     bool graphs_broken = false;  // a capture / instantiation failed once: launch eagerly from now on
+    bool capturing = false;      // inside a stream capture (no timing events: they would be graph nodes)
     cudaEvent_t ev_fork = nullptr;
     std::vector<cudaEvent_t> ev_join;
 
@@ -806,14 +886,20 @@ static int drain_timing(pk_ctx c) {
         PK_CUDA(cudaEventSynchronize(t.stop));
         float ms = 0.f;
         PK_CUDA(cudaEventElapsedTime(&ms, t.start, t.stop));
-        c->stats.kernel_ms += ms;
-        c->stats.timed_kernels += 1;
+        if (t.graph) {
+            c->stats.graph_launch_ms += ms;
+            c->stats.timed_graph_launches += 1;
+        } else {
+            c->stats.kernel_ms += ms;
+            c->stats.timed_kernels += 1;
+        }
         c->event_pool[t.part].push_back(t.start);
         c->event_pool[t.part].push_back(t.stop);
     }
     // per launch: max over partitions
     std::unordered_map<uint64_t, double> mx;
     for (TimedLaunch& t : c->pending_timing) {
+        if (t.graph) continue;
         float ms = 0.f;
         cudaEventElapsedTime(&ms, t.start, t.stop);
         double& v = mx[t.launch_id];
@@ -841,6 +927,12 @@ int pk_finalize(pk_ctx c) {
             ipc_barrier(c);
             if (c->flag_local) { cudaSetDevice(c->dev[c->first_local]); cudaFree(c->flag_local); }
         }
+#ifdef PK_TRACE_ACCESS
+        for (Buffer& B : c->bufs)
+            if (B.alive)
+                for (int p = 0; p < c->P; ++p)
+                    if (B.inst[p] && c->local(p)) trace_remove(B.inst[p]);
+#endif
         for (size_t b = 0; b < c->bufs.size(); ++b) {
             Buffer& B = c->bufs[b];
             if (B.alive && B.owned)
@@ -955,6 +1047,14 @@ int pk_register_buffer(pk_ctx c, int ndim, const int64_t* shape, int elem_bytes,
             B.inst[q] = (char*)m + x.off;
         }
     }
+#ifdef PK_TRACE_ACCESS
+    if (!c->host_only)
+        for (int p = 0; p < c->P; ++p)
+            if (c->local(p) && B.inst[p] && B.bytes) {
+                if (int r = c->set_device(c->dev[p])) return r;
+                PK_CUDA(trace_add(B.inst[p], B.bytes));
+            }
+#endif
     B.alive = true;
     c->bufs.push_back(std::move(B));
     *out = (pk_buf)(c->bufs.size() - 1);
@@ -985,6 +1085,10 @@ int pk_unregister_buffer(pk_ctx c, pk_buf b) {
             if (B.ipc_base[q]) { ipc_close(c, B.ipc_base[q]); B.ipc_base[q] = nullptr; B.inst[q] = nullptr; }
         if (int r = ipc_barrier(c)) return r;
     }
+#ifdef PK_TRACE_ACCESS
+    for (int p = 0; p < c->P; ++p)
+        if (B.inst[p] && c->local(p)) trace_remove(B.inst[p]);
+#endif
     if (!c->host_only && B.owned) {
         for (int p = 0; p < c->P; ++p)
             if (B.inst[p] && c->local(p)) {
@@ -1008,6 +1112,7 @@ static int wait_readers(pk_ctx c, Buffer& B, int p) {
 }
 
 int pk_copy_from_host(pk_ctx c, pk_buf b, const void* host, size_t bytes) {
+    NvtxPhase nv("pk a8 H2D 1:n linear");
     if (!valid_buf(c, b) || !host) return fail(PK_ERR_INVALID, "bad argument");
     Buffer& B = c->bufs[b];
     if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (H2D copies the whole virtual buffer)");
@@ -1227,6 +1332,7 @@ static int sync_to_host_ipc(pk_ctx c, Buffer& B, void* host) {
 }
 
 static int sync_to_host(pk_ctx c, pk_buf b, void* host, size_t bytes, bool async) {
+    NvtxPhase nv("pk a8 D2H n:1 gather");
     if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "bad argument");
     Buffer& B = c->bufs[b];
     if (bytes != B.bytes) return fail(PK_ERR_INVALID, "size mismatch (D2H gathers the whole virtual buffer)");
@@ -1427,13 +1533,17 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
 int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
                           const void* const* args, const int64_t* scalars, int ns) {
     if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
+    struct CpuTime {  // thread CPU time of this call -> pk_stats.host_cpu_ns
+        pk_ctx c;
+        uint64_t t0 = thread_cpu_ns();
+        ~CpuTime() { c->stats.host_cpu_ns += thread_cpu_ns() - t0; }
+    } cpu_time{c};
     if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
     const Kernel& K = c->kernels[k];
     const uint32_t mode = c->mode;
     // builtin launchers take every scalar from `scalars`, so the key below captures the launch
     const bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && K.nargs && args && K.launcher &&
-                           !c->graphs_broken &&
-                           !(mode & (PK_MODE_TIME_KERNELS | PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
+                           !c->graphs_broken && !(mode & (PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
     if (!can_graph) {
         if (!c->host_only)
             if (int r = exit_graph_mode(c)) return r;
@@ -1449,7 +1559,8 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
     put(grid, 12);
     put(block, 12);
     put(&smem, sizeof smem);
-    put(&mode, sizeof mode);
+    const uint32_t kmode = mode & ~(uint32_t)PK_MODE_TIME_KERNELS;  // timing events sit outside the graph
+    put(&kmode, sizeof kmode);
     put(&ns, sizeof ns);
     if (ns) put(scalars, sizeof(int64_t) * ns);
     std::vector<int64_t> bids;
@@ -1490,10 +1601,27 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
     }
     if (it != c->memo.end() && it->second.exec) {
         // ---- replay: one graph launch + restore the memoised tracker states ----
+        NvtxPhase nv("pk graph replay");
         pk_ctx_s::Memo& m = it->second;
         if (int r = enter_graph_mode(c)) return r;
-        if (int r = c->set_device(c->dev[c->first_local])) return r;
-        PK_CUDA(cudaGraphLaunch(m.exec, c->stream[c->first_local]));
+        const int p0 = c->first_local;
+        if (int r = c->set_device(c->dev[p0])) return r;
+        cudaEvent_t e0 = nullptr, e1 = nullptr;
+        if (mode & PK_MODE_TIME_KERNELS) {  // the whole replayed launch, on the stream it runs on
+            auto& pool = c->event_pool[p0];
+            for (cudaEvent_t* e : {&e0, &e1}) {
+                if (!pool.empty()) { *e = pool.back(); pool.pop_back(); }
+                else PK_CUDA(cudaEventCreate(e));
+            }
+            PK_CUDA(cudaEventRecord(e0, c->stream[p0]));
+        }
+        PK_CUDA(cudaGraphLaunch(m.exec, c->stream[p0]));
+        if (mode & PK_MODE_TIME_KERNELS) {
+            PK_CUDA(cudaEventRecord(e1, c->stream[p0]));
+            TimedLaunch tl{e0, e1, p0, c->launch_counter};
+            tl.graph = true;
+            c->pending_timing.push_back(tl);
+        }
         for (auto& ps : m.post) c->bufs[ps.buf].tracker.set_state(ps.state, ps.fp);
         c->replay_plan = m.plan;
         add_stats(c->stats, m.delta, 1);
@@ -1546,8 +1674,10 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
                 c->set_device(c->dev[p]);
                 ce = cudaStreamWaitEvent(c->stream[p], c->ev_fork, 0);
             }
+        c->capturing = true;
         rc = ce == cudaSuccess ? launch_eager(c, k, grid, block, smem, args, scalars, ns)
                                : fail(PK_ERR_CUDA, std::string("graph fork: ") + cudaGetErrorName(ce));
+        c->capturing = false;
         if (rc == PK_OK && getenv("PK_DEBUG_FAIL_CAPTURE"))  // test hook: exercise the eager fallback
             rc = fail(PK_ERR_CUDA, "PK_DEBUG_FAIL_CAPTURE");
         for (int p = 0; p < c->P && rc == PK_OK; ++p)
@@ -1631,6 +1761,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     const bool transfer = track && !(mode & PK_MODE_NO_TRANSFERS);
     const bool single_owner = mode & PK_MODE_SINGLE_OWNER;
     uint64_t t0 = now_ns();
+    NvtxPhase nv("pk a1+a2 partition, regions");
 
     // ---- a1 + a2: partition boxes and regions (cached) ----
     std::shared_ptr<std::vector<Regions>> regs;
@@ -1661,6 +1792,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     c->stats.host_ns_partition += t1 - t0;
     uint64_t t2 = now_ns();
     c->stats.host_ns_regions += t2 - t1;
+    nv.next("pk a3 stale detection, plan");
 
     // per (partition, distinct buffer): merged read / write sets
     struct BufSets { int64_t b; RangeList r, w; };
@@ -1774,6 +1906,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
 
     uint64_t t3 = now_ns();
     c->stats.host_ns_plan += t3 - t2;
+    nv.next("pk a4+a5 transfers, ordering");
     c->stats.launches += 1;
     const uint64_t launch_id = c->launch_counter++;
     const uint64_t E = c->ipc ? ++c->epoch : 0;  // replicated: identical on every rank
@@ -2018,6 +2151,8 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         }
     }
     uint64_t t4 = now_ns();
+    nv.next("pk a6 partitioned launches");
+    const bool time_k = (mode & PK_MODE_TIME_KERNELS) && !c->capturing;
 
     // ---- a6: partitioned launches (Eq. 8-10) ----
     bool writes_arg[PK_MAX_ARGS] = {};
@@ -2103,7 +2238,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             dim3 g(part.max[0] - part.min[0], part.max[1] - part.min[1], part.max[2] - part.min[2]);
             dim3 bl(block[0], block[1], block[2]);
             cudaEvent_t e0 = nullptr, e1 = nullptr;
-            if (mode & PK_MODE_TIME_KERNELS) {
+            if (time_k) {
                 auto& pool = c->event_pool[p];
                 for (cudaEvent_t* e : {&e0, &e1}) {
                     if (!pool.empty()) { *e = pool.back(); pool.pop_back(); }
@@ -2122,7 +2257,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             if (err != cudaSuccess)
                 return fail(PK_ERR_CUDA, "launch of '" + K.name + "' on partition " + std::to_string(p) + ": " +
                                              cudaGetErrorName(err) + " (" + cudaGetErrorString(err) + ")");
-            if (mode & PK_MODE_TIME_KERNELS) {
+            if (time_k) {
                 PK_CUDA(cudaEventRecord(e1, c->stream[p]));
                 c->pending_timing.push_back(TimedLaunch{e0, e1, p, launch_id});
             }
@@ -2160,6 +2295,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     }
     uint64_t t5 = now_ns();
     c->stats.host_ns_issue += (t4 - t3) + (t5 - t4);
+    nv.next("pk a7 tracker update");
 
     // ---- a7: tracker update with the write sets, kernels running ----
     if (track)
@@ -2185,6 +2321,66 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 }
     c->stats.host_ns_update += now_ns() - t5;
     return PK_OK;
+}
+
+// ---- access recording (PK_TRACE_ACCESS build) ----
+int pk_trace_available(void) {
+#ifdef PK_TRACE_ACCESS
+    return 1;
+#else
+    return 0;
+#endif
+}
+
+int pk_trace_reset(pk_ctx c) {
+#ifdef PK_TRACE_ACCESS
+    if (!c || c->host_only) return fail(PK_ERR_INVALID, "bad context");
+    if (int r = pk_synchronize(c)) return r;
+    std::lock_guard<std::mutex> g(g_trace_mu);
+    for (const TraceInst& t : g_trace)
+        for (int k = 0; k < 2; ++k) PK_CUDA(cudaMemset(t.bits[k], 0, ((t.bytes / 4 + 31) / 32) * 4));
+    unsigned long long z = 0;
+    PK_CUDA(cudaMemcpyToSymbol(g_pk_trace, &z, sizeof z, offsetof(pk::trace::Table, stray)));
+    return PK_OK;
+#else
+    (void)c;
+    return fail(PK_ERR_STATE, "library built without PK_TRACE_ACCESS (load libpk_trace.so)");
+#endif
+}
+
+int pk_trace_fetch(pk_ctx c, pk_buf b, int part, int kind, uint32_t* words, uint64_t nwords) {
+#ifdef PK_TRACE_ACCESS
+    if (!valid_buf(c, b) || part < 0 || part >= c->P || kind < 0 || kind > 1 || (nwords && !words))
+        return fail(PK_ERR_INVALID, "bad argument");
+    if (int r = pk_synchronize(c)) return r;
+    const Buffer& B = c->bufs[b];
+    std::lock_guard<std::mutex> g(g_trace_mu);
+    for (const TraceInst& t : g_trace)
+        if (t.base == B.inst[part]) {
+            const uint64_t n = (t.bytes / 4 + 31) / 32;
+            if (nwords < n) return fail(PK_ERR_INVALID, "bitmap needs " + std::to_string(n) + " words");
+            PK_CUDA(cudaMemcpy(words, t.bits[kind], n * 4, cudaMemcpyDeviceToHost));
+            return PK_OK;
+        }
+    return fail(PK_ERR_STATE, "instance is not traced");
+#else
+    (void)c; (void)b; (void)part; (void)kind; (void)words; (void)nwords;
+    return fail(PK_ERR_STATE, "library built without PK_TRACE_ACCESS (load libpk_trace.so)");
+#endif
+}
+
+int pk_trace_stray(pk_ctx c, uint64_t* out) {
+#ifdef PK_TRACE_ACCESS
+    if (!c || !out) return fail(PK_ERR_INVALID, "bad argument");
+    if (int r = pk_synchronize(c)) return r;
+    unsigned long long v = 0;
+    PK_CUDA(cudaMemcpyFromSymbol(&v, g_pk_trace, sizeof v, offsetof(pk::trace::Table, stray)));
+    *out = v;
+    return PK_OK;
+#else
+    (void)c; (void)out;
+    return fail(PK_ERR_STATE, "library built without PK_TRACE_ACCESS (load libpk_trace.so)");
+#endif
 }
 
 }  // extern "C"
