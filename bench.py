@@ -135,6 +135,79 @@ class ClockSampler:
                 "power_w_max": max(power) if power else None}
 
 
+class NvlinkCounters:
+    """NVML NVLink data counters (KiB, cumulative over all links) of the GPUs in use, read
+    around the timed region -- the hardware's count of inter-GPU bytes, to set beside the
+    library's moved + pushed bytes.  None where NVML or the field is missing."""
+
+    def __init__(self, gpus):
+        self.gpus, self.h, self.t0 = list(gpus), None, None
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            self.nv = nv
+            self.h = [nv.nvmlDeviceGetHandleByIndex(g) for g in self.gpus]
+        except Exception:
+            self.h = None
+
+    def _read(self):
+        nv = self.nv
+        tot = [0, 0]
+        for h in self.h:
+            vals = nv.nvmlDeviceGetFieldValues(h, [nv.NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX,
+                                                   nv.NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_RX])
+            for i, v in enumerate(vals):
+                if v.nvmlReturn != 0:
+                    raise RuntimeError("field unavailable")
+                tot[i] += int(v.value.ullVal) * 1024
+        return tot
+
+    def start(self):
+        try:
+            self.t0 = self._read() if self.h else None
+        except Exception:
+            self.t0 = None
+
+    def stop(self):
+        if not self.t0:
+            return None
+        try:
+            t1 = self._read()
+        except Exception:
+            return None
+        return {"tx_bytes": t1[0] - self.t0[0], "rx_bytes": t1[1] - self.t0[1], "gpus": self.gpus,
+                "source": "NVML NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX/RX over the timed region"}
+
+
+def measure_tf32_ceiling(device, n=8192, reps=10):
+    """Dense TF32 tensor-core ceiling of this GPU in this run: cuBLAS through torch.matmul on
+    fp32 inputs with TF32 enabled (SURVEY.md §8(d) "measured ceilings"), CUDA events."""
+    try:
+        import torch
+        with torch.cuda.device(device):
+            old = torch.backends.cuda.matmul.allow_tf32
+            torch.backends.cuda.matmul.allow_tf32 = True
+            a = torch.randn(n, n, device="cuda")
+            b = torch.randn(n, n, device="cuda")
+            for _ in range(3):
+                torch.matmul(a, b)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            e0.record()
+            for _ in range(reps):
+                torch.matmul(a, b)
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / reps
+            torch.backends.cuda.matmul.allow_tf32 = old
+            del a, b
+            torch.cuda.empty_cache()
+        return {"tflops": 2.0 * n ** 3 / (ms / 1e3) / 1e12, "shape": [n, n, n], "ms": ms,
+                "how": "torch.matmul fp32 with allow_tf32 (cuBLAS), mean of %d after 3 warm-up" % reps}
+    except Exception as e:  # pragma: no cover
+        return None
+
+
 # ------------------------------------------------------------------ workloads
 class Workload:
     """Inputs, setup and per-step loop of one config, driven through the C-ABI."""
@@ -174,7 +247,14 @@ class Workload:
         elif name == "sgemm":
             m = n = k = 16384
             self.shape = (m, n, k)
-            self.host = synth.gemm_operands(m, n, k)
+            a, b = synth.gemm_operands(m, n, k)
+            # Each step is one partitioned GEMM X' = A X whose operand X is the previous step's
+            # output: partition p wrote row slab p of it, so every step reads the whole operand
+            # from all partitions -- the (P-1)|B| broadcast of BASELINE's C4 config happens
+            # inside every timed step.  A is scaled by sqrt(3/K) (entry variance 1/K) so the
+            # iterates keep their magnitude (DESIGN.md §3 input recipe).
+            a *= np.float32(math.sqrt(3.0 / k))
+            self.host = (a, b)
             self.units_per_iter = 2 * m * n * k          # FP32-equivalent flops
             self.bytes_per_unit = 0
             self.scale = 1e12
@@ -182,6 +262,8 @@ class Workload:
         else:
             raise SystemExit(f"unknown workload {name}")
         self.scale = getattr(self, "scale", 1e9)
+        # kernels launched per partition per pk_launch_partitioned (gpu_launches)
+        self.kernels_per_launch = {"nbody": 2, "sgemm": 3}.get(name, 1)
 
     def block_depth(self):
         """Rows per tile (Hotspot) / planes per block (Heat) when --tile is not given: the
@@ -224,6 +306,7 @@ class Workload:
         elif self.name == "sgemm":
             self.pr, _ = K.sgemm_program(ctx, *self.host, launches=0)
             self.upload_bufs = [(self.pr.abc[0], self.host[0]), (self.pr.abc[1], self.host[1])]
+            self.gemm_t = 0    # X_t = buffer B (t even) / C (t odd)
         elif self.name == "jacobi2d":
             self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0, tiles=self.tiles)
             self.upload_bufs = [(b, self.host[0]) for b in self.pr.bufs]
@@ -251,8 +334,10 @@ class Workload:
             a, b, c = pr.abc
             m, n, k = pr.mnk
             for _ in range(self.iters):
-                pr.launch(grid, blk, [a, b, c, m, n, k], sc)
-            out = c
+                x, y = (b, c) if self.gemm_t % 2 == 0 else (c, b)
+                pr.launch(grid, blk, [a, x, y, m, n, k], sc)
+                self.gemm_t += 1
+                out = y
         else:
             out, _ = K.nbody_iterate(pr, self.iters, self.t)
         self.t += self.iters
@@ -269,7 +354,7 @@ class Workload:
             "heat3d": lambda: 2 * self.shape[1] * self.shape[2] * 4 * (P - 1),
             "jacobi2d": lambda: 2 * (self.shape[1] - 2) * 4 * (P - 1),
             "nbody": lambda: self.shape[0] * 16 * (P - 1),
-            "sgemm": lambda: 0,   # B moves once (first launch): (P-1) K N 4 B, reported by the stats
+            "sgemm": lambda: (P - 1) * self.shape[2] * self.shape[1] * 4,   # the whole operand X, every step
         }
         return from_cf[self.name]() * self.iters
 
@@ -401,6 +486,8 @@ def main():
                     help="PK_MODE_PUSH: halo rows stored into the neighbours' instances by the producing kernel")
     ap.add_argument("--abg", action="store_true",
                     help="also run the paper's alpha/beta/gamma overhead decomposition (P:L1164-1181)")
+    ap.add_argument("--abg-repeats", type=int, default=3)
+    ap.add_argument("--no-e3", action="store_true", help="skip the P = 1 library vs direct-launch comparison")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "pk":
         print("warning: fewer than 3 warm-up steps", file=sys.stderr)
@@ -476,27 +563,29 @@ def main():
     if sampler:
         sampler.start()
         time.sleep(0.3)
-    # (1) the timed region.  Kernels of 100 us and more (every config but the latency-bound
-    # C1) are timed live in it when there is one partition per process: PK_MODE_TIME_KERNELS
-    # records CUDA events around every partition kernel on its own stream.  C1 (microsecond
-    # launches) keeps steady-state graph replay in the timed region and gets its kernel
-    # events from a second pass.
-    # Single-process P > 1 keeps graph replay (eager + events would add ~130 us of host time per
-    # launch at P = 8) and also takes the events from the second pass.
-    live = w.name != "jacobi2d" and (world > 1 or P == 1)
+    # (1) the timed region, in the production mode (steady-state graph replay on for
+    # single-process contexts).  Launches of 100 us and more (every config but the
+    # latency-bound C1) are timed live in it: PK_MODE_TIME_KERNELS records CUDA events
+    # around every replayed launch on the stream it runs on (around every partition kernel
+    # when a launch runs eagerly: SPMD ranks).  C1 (microsecond launches) takes its events
+    # from a second pass of the same steps.
+    nvl = NvlinkCounters(devices_used if world == 1 else [env_int("LOCAL_RANK", rank) % max(1, torch.cuda.device_count())])
+    live = w.name != "jacobi2d"
     if live:
         abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
     abi.pk_synchronize(ctx)
+    nvl.start()
     abi.pk_timer_begin(ctx)
     for _ in range(args.steps):
         w.step()
     elapsed_ms = abi.pk_timer_end(ctx)
+    nvlink_measured = nvl.stop()
     st = abi.pk_get_stats(ctx)
     if live:
         stk = st
         abi.pk_set_mode(ctx, base_mode)
     else:
-        # (2) per-kernel CUDA events for the roofline (events around every partition kernel)
+        # (2) CUDA events for the roofline from a second pass of the same steps
         abi.pk_reset_stats(ctx)
         abi.pk_set_mode(ctx, base_mode | abi.PK_MODE_TIME_KERNELS)
         for _ in range(max(1, min(args.steps, 3))):
@@ -505,7 +594,17 @@ def main():
         stk = abi.pk_get_stats(ctx)
         abi.pk_set_mode(ctx, base_mode)
     clocks = sampler.stop() if sampler else {}
-    st["kernel_ms"], st["timed_kernels"] = stk["kernel_ms"], stk["timed_kernels"]
+    for key_ in ("kernel_ms", "timed_kernels", "kernel_ms_max_launch", "graph_launch_ms", "timed_graph_launches",
+                 "launches"):
+        st["t_" + key_] = stk[key_]
+    # (3) host overhead without launch-queue back-pressure: one step issued into idle
+    # streams (the timed region's launches queue up behind running kernels, and a full
+    # queue blocks the issuing thread inside the CUDA calls)
+    abi.pk_synchronize(ctx)
+    abi.pk_reset_stats(ctx)
+    w.step()
+    sh = abi.pk_get_stats(ctx)
+    abi.pk_synchronize(ctx)
     if dist:
         tt = torch.tensor([elapsed_ms, st["kernel_launches"], st["moved_bytes"], st["copies"], st["pushed_bytes"]],
                           dtype=torch.float64)
@@ -520,19 +619,31 @@ def main():
     value = units / (elapsed_ms / 1e3) / w.scale
     peaks = load_peaks()
     kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk", "heat3d": "heat3d_tb2"}.get(w.name, w.name)
-    avg_kernel_ms = st["kernel_ms"] / max(1, st["timed_kernels"])
-    per_launch_units = w.units_per_iter * getattr(w, "sweeps", 1) / P
+    # duration of one timed launch: a replayed graph (single process: every partition's
+    # copies + kernels of the launch) or, launched eagerly, the slowest partition kernel
+    n_timed = st["t_timed_graph_launches"] + (st["t_launches"] - st["t_timed_graph_launches"])
+    avg_kernel_ms = (st["t_graph_launch_ms"] + st["t_kernel_ms_max_launch"]) / max(1, n_timed)
+    # units of one timed launch: all partitions of this process (one per SPMD rank)
+    per_launch_units = w.units_per_iter * getattr(w, "sweeps", 1) / (P if world > 1 else 1)
     if w.name == "sgemm":
-        # tensor bound: 3 TF32 MMAs per FP32-equivalent product; TF32 peak = measured bf16 x (1.1/2.25).
-        # Each step is one ~35 ms launch timed alone (not a seconds-long loop): the burst figure applies.
+        # tensor bound: 3 TF32 MMAs per FP32-equivalent product, against the TF32 ceiling measured
+        # in this run (cuBLAS via torch.matmul, allow_tf32, 8192^3); the bf16-derived figure beside it
+        tf32 = measure_tf32_ceiling(devices[0] if world == 1 else torch.cuda.current_device())
         bf16 = (peaks or {}).get("bf16_tflops", 1668.4)
-        peak = bf16 * 1.1 / 2.25
+        derived = bf16 * 1.1 / 2.25
+        # the denominator is the HIGHER of the two: cuBLAS' TF32 GEMM measured in this run (it
+        # measured 723 TF/s at 8192^3, i.e. below what the 3xTF32 kernel sustains, so it is not a
+        # ceiling on its own) and measured bf16 x the nominal TF32/BF16 ratio
+        peak = max(tf32["tflops"] if tf32 else 0.0, derived)
         achieved = 3 * per_launch_units / (avg_kernel_ms / 1e3) / 1e12
-        sust = (peaks or {}).get("bf16_tflops_sustained", 1392.4) * 1.1 / 2.25
         roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                    "frac": achieved / peak, "traffic": ncu_traffic(kname), "frac_of_sustained": achieved / sust,
-                    "peak_source": "MEASURED_PEAKS.json bf16_tflops (burst) x 1.1/2.25 (TF32/BF16 nominal ratio); "
-                                   "achieved = 3 x 2MNK TF32 flops / (split + GEMM kernel time)"}
+                    "frac": achieved / peak, "traffic": ncu_traffic(kname),
+                    "peak_bf16_derived": derived, "frac_of_bf16_derived": achieved / derived,
+                    "tf32_ceiling": tf32,
+                    "frac_of_cublas_tf32": (achieved / tf32["tflops"]) if tf32 else None,
+                    "peak_source": "max(TF32 GEMM of cuBLAS measured in this run: torch.matmul fp32 with allow_tf32, "
+                                   "8192^3, CUDA events; MEASURED_PEAKS.json bf16_tflops x 1.1/2.25, the nominal "
+                                   "TF32/BF16 ratio); achieved = 3 x 2MNK TF32 flops / launch time"}
     elif w.name == "nbody":
         # FP32-ALU bound: 12 FP32-pipe instructions per interaction on 128 lanes/SM
         sm_mhz = clocks.get("sm_mhz") or (peaks or {}).get("sm_max_mhz", 1965.0)
@@ -564,14 +675,18 @@ def main():
                    **({"rows_per_tile": w.block_depth()} if w.name == "hotspot2d" and not w.variant else {}),
                    **({"planes_per_block": w.block_depth()} if w.name == "heat3d" and not w.variant else {}),
                    "partition_shape": list(w.tiles) if w.tiles else "1-D slabs of the slowest grid dim"},
-        "gpu_launches": int(st["kernel_launches"] + st["copy_kernels"]),
+        "gpu_launches": int(st["kernel_launches"] * w.kernels_per_launch + st["copy_kernels"]),
         "graph_replays": int(st.get("graph_replays", 0)),
         "clocks": clocks,
         "roofline": roofline,
         "kernel_ms_avg": avg_kernel_ms,
-        "kernel_timing": ("CUDA events around every partition kernel on its stream, inside the timed region"
-                          if live else "CUDA events around every partition kernel on its stream, second pass of "
-                          "the same steps right after the timed region (the timed region replays graphs)"),
+        "kernel_timing": (("CUDA events on the launching stream inside the timed region, production mode: "
+                           "around each replayed graph launch (%d launches)%s" %
+                           (st["t_timed_graph_launches"],
+                            "" if st["t_timed_graph_launches"] == n_timed else
+                            ", around every partition kernel of the %d eager launches" % (n_timed - st["t_timed_graph_launches"])))
+                          if live else "CUDA events on the launching stream, second pass of the same steps right "
+                          "after the timed region (C1: microsecond launches)"),
         "transfers": {"stale_bytes": int(st["stale_bytes"]), "moved_bytes": int(st["moved_bytes"]),
                       "analytic_min_bytes": w.stale_min(P) * args.steps if not w.tiles else None,
                       "copies": int(st["copies"]), "strided_copies": int(st["strided_copies"]),
@@ -586,38 +701,83 @@ def main():
                     / (elapsed_ms / 1e3) / 900e9,
                     "note": "moved + pushed bytes between partitions on different GPUs; averaged over the step"}
                    if len(devices_used) > 1 else None),
-        "host_us_per_launch": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"]
-                               + st["host_ns_issue"] + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
-        "host_us_per_launch_phases": {k: st["host_ns_" + k] / 1e3 / max(1, st["launches"])
+        # host time inside pk_launch_partitioned, from one step issued into idle streams (no
+        # launch-queue back-pressure); thread CPU time beside the wall time
+        "host_us_per_launch": (sh["host_ns_partition"] + sh["host_ns_regions"] + sh["host_ns_plan"]
+                               + sh["host_ns_issue"] + sh["host_ns_update"]) / 1e3 / max(1, sh["launches"]),
+        "host_cpu_us_per_launch": sh["host_cpu_ns"] / 1e3 / max(1, sh["launches"]),
+        "host_us_per_launch_phases": {k: sh["host_ns_" + k] / 1e3 / max(1, sh["launches"])
                                       for k in ("partition", "regions", "plan", "issue", "update")},
+        "host_us_per_launch_timed_region": {
+            "wall": (st["host_ns_partition"] + st["host_ns_regions"] + st["host_ns_plan"] + st["host_ns_issue"]
+                     + st["host_ns_update"]) / 1e3 / max(1, st["launches"]),
+            "thread_cpu": st["host_cpu_ns"] / 1e3 / max(1, st["launches"]),
+            "note": "includes time blocked in CUDA calls once the launch queue is full (launches are issued "
+                    "far ahead of the GPU)"},
+        "nvlink_nvml": nvlink_measured,
         "us_per_launch": elapsed_ms * 1e3 * getattr(w, "sweeps", 1) / max(1, w.iters * args.steps),
     })
 
     # ---- alpha / beta / gamma (§9.2) ----
     if args.abg:
-        times = {}
-        for name, mode in (("alpha", 0), ("beta", abi.PK_MODE_NO_TRANSFERS), ("gamma", abi.PK_MODE_NO_TRACKING)):
-            abi.pk_set_mode(ctx, mode | (base_mode if mode == 0 else 0))
-            w.step()                                   # settle the mode (tracker state, caches)
-            abi.pk_synchronize(ctx)
-            if dist:
-                dist.barrier()
-            t0 = time.perf_counter()
-            for _ in range(args.steps):
-                w.step()
-            abi.pk_synchronize(ctx)
-            el = time.perf_counter() - t0
-            if dist:
-                te = torch.tensor([el], dtype=torch.float64)
-                dist.all_reduce(te, op=dist.ReduceOp.MAX)
-                el = float(te[0])
-            times[name] = el
+        # R repeats per mode, interleaved (alpha, beta, gamma, alpha, ...) so that clock drift
+        # hits all three alike; each repeat = args.steps steps, device-timed (pk_timer), max over ranks
+        reps = {"alpha": [], "beta": [], "gamma": []}
+        modes = (("alpha", 0), ("beta", abi.PK_MODE_NO_TRANSFERS), ("gamma", abi.PK_MODE_NO_TRACKING))
+        for r in range(args.abg_repeats):
+            for name, mode in modes:
+                abi.pk_set_mode(ctx, mode | (base_mode if mode == 0 else 0))
+                w.step()                                   # settle the mode (tracker state, caches, graphs)
+                abi.pk_synchronize(ctx)
+                if dist:
+                    dist.barrier()
+                abi.pk_timer_begin(ctx)
+                for _ in range(args.steps):
+                    w.step()
+                el = abi.pk_timer_end(ctx) / 1e3
+                if dist:
+                    te = torch.tensor([el], dtype=torch.float64)
+                    dist.all_reduce(te, op=dist.ReduceOp.MAX)
+                    el = float(te[0])
+                reps[name].append(el)
         abi.pk_set_mode(ctx, base_mode)
-        a, b, g = times["alpha"], times["beta"], times["gamma"]
+        med = {k: statistics.median(v) for k, v in reps.items()}
+        a, b, g = med["alpha"], med["beta"], med["gamma"]
+        # per-repeat fractions (same repeat index) give the spread of each share
+        fr = {"T_application": [rg / ra for ra, rg in zip(reps["alpha"], reps["gamma"])],
+              "T_transfers": [(ra - rb) / ra for ra, rb in zip(reps["alpha"], reps["beta"])],
+              "T_patterns": [(rb - rg) / ra for ra, rb, rg in zip(reps["alpha"], reps["beta"], reps["gamma"])]}
         result["overhead"] = {"alpha_s": a, "beta_s": b, "gamma_s": g, "T_application": g / a,
                               "T_transfers": (a - b) / a, "T_patterns": (b - g) / a,
-                              "note": "wall clock over the same steps; beta = no transfers (results wrong "
-                                      "by design), gamma = no dependency resolution / tracking"}
+                              "repeats": args.abg_repeats, "seconds": reps,
+                              "spread": {k: [min(v), max(v)] for k, v in fr.items()},
+                              "note": "device time (pk_timer) of the same steps, median over interleaved repeats, "
+                                      "[min, max] of the per-repeat shares; beta = no transfers (results wrong by "
+                                      "design), gamma = no dependency resolution / tracking (P:L1164-1181)"}
+
+    # ---- E3: P = 1 through the library vs the original single-GPU launches ----
+    if P == 1 and world == 1 and not args.no_e3:
+        lib_ms, dir_ms = [], []
+        per_step = elapsed_ms / args.steps
+        n3 = max(1, min(args.steps, int(2000 / max(per_step, 1e-3))))     # ~2 s per pass
+        for r in range(2):
+            for direct in (False, True):
+                w.pr.direct = direct
+                if per_step < 500:
+                    w.step()                                   # settle (graphs of the library path)
+                abi.pk_synchronize(ctx)
+                abi.pk_timer_begin(ctx)
+                for _ in range(n3):
+                    w.step()
+                (dir_ms if direct else lib_ms).append(abi.pk_timer_end(ctx))
+        w.pr.direct = False
+        lm, dm = statistics.median(lib_ms), statistics.median(dir_ms)
+        result["e3_single_gpu_slowdown"] = {
+            "library_ms_per_step": lm / n3, "direct_ms_per_step": dm / n3, "steps_per_pass": n3,
+            "slowdown_pct": 100.0 * (lm / dm - 1.0),
+            "note": "device time of the same steps: pk_launch_partitioned at P = 1 (graph replay, production mode) vs "
+                    "pk_launch_direct (the kernel's full grid, no partitioning / tracking); median of 2 interleaved "
+                    "repeats; the paper reports a median 2.1 % slowdown (P:L1156-1161)"}
 
     # ---- e2e: same metric with the H2D upload and D2H gather inside every step ----
     if not args.no_e2e:
@@ -666,6 +826,7 @@ def main():
                 (abi.pk_copy_from_host_async if pipelined else abi.pk_copy_from_host)(c, b, hbuf)
                 h2d += hbuf.numel() * hbuf.element_size()
             ws_.t = 0
+            ws_.gemm_t = 0                   # e2e C4: C = A B from the uploaded operands every step
             out = ws_.step()
             (abi.pk_sync_to_host_async if pipelined else abi.pk_sync_to_host)(c, out, out_host)
             d2h += out_host.numel() * out_host.element_size()

@@ -274,6 +274,15 @@ const void* pk_builtin_fn(const char* name);
 int pk_launch_partitioned(pk_ctx ctx, pk_kernel k, const int32_t grid[3],
                           const int32_t block[3], size_t smem_bytes,
                           const void* const* args, const int64_t* scalars, int nscalars);
+/* The ORIGINAL single-GPU launch, for the paper's E3 measurement (§9.2:
+ * "slowdown of the partitioned binary on a single GPU"): the kernel's full grid is
+ * launched once on partition 0's stream with partition 0's instances -- no partition
+ * boxes, regions, tracker, transfers or graph replay.  It neither reads nor updates the
+ * validity map, so it is a measurement baseline, not a way to run the method: only for
+ * single-partition contexts (PK_ERR_STATE otherwise).  Same arguments and errors as
+ * pk_launch_partitioned (PK_ERR_INVALID, PK_ERR_CUDA). */
+int pk_launch_direct(pk_ctx ctx, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem_bytes,
+                     const void* const* args, const int64_t* scalars, int nscalars);
 /* cudaDeviceSynchronize replacement: all partitions' streams (§8.4). */
 int pk_synchronize(pk_ctx ctx);
 /* Device-side timer over everything the context enqueues between the two calls:

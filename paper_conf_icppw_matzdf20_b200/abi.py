@@ -129,6 +129,8 @@ def lib():
         "pk_builtin_kernel": [C.c_void_p, C.c_char_p, _I64P],
         "pk_launch_partitioned": [C.c_void_p, C.c_int64, _I32P, _I32P, C.c_size_t,
                                   C.POINTER(C.c_void_p), _I64P, C.c_int],
+        "pk_launch_direct": [C.c_void_p, C.c_int64, _I32P, _I32P, C.c_size_t,
+                             C.POINTER(C.c_void_p), _I64P, C.c_int],
         "pk_synchronize": [C.c_void_p],
         "pk_timer_begin": [C.c_void_p],
         "pk_timer_end": [C.c_void_p, C.POINTER(C.c_double)],
@@ -333,9 +335,7 @@ def pk_builtin_kernel(ctx, name) -> int:
 _LAUNCH_ARGS = {}   # marshalled ctypes arguments of recent launches (steady-state loops repeat them)
 
 
-def pk_launch_partitioned(ctx, kernel, grid, block, args, scalars=(), smem=0):
-    """args: one int per kernel argument -- the pk_buf id for a buffer, the
-    (int64) value for a scalar; None passes a NULL pointer."""
+def _launch_args(kernel, grid, block, args, scalars):
     key = (kernel, tuple(grid), tuple(block), tuple(args), tuple(scalars))
     m = _LAUNCH_ARGS.get(key)
     if m is None:
@@ -346,7 +346,20 @@ def pk_launch_partitioned(ctx, kernel, grid, block, args, scalars=(), smem=0):
         if len(_LAUNCH_ARGS) > 1024:
             _LAUNCH_ARGS.clear()
         _LAUNCH_ARGS[key] = m
+    return m
+
+
+def pk_launch_partitioned(ctx, kernel, grid, block, args, scalars=(), smem=0):
+    """args: one int per kernel argument -- the pk_buf id for a buffer, the
+    (int64) value for a scalar; None passes a NULL pointer."""
+    m = _launch_args(kernel, grid, block, args, scalars)
     _check(lib().pk_launch_partitioned(ctx, kernel, m[0], m[1], smem, m[2], m[3], m[4]), "pk_launch_partitioned")
+
+
+def pk_launch_direct(ctx, kernel, grid, block, args, scalars=(), smem=0):
+    """The original single-GPU launch (E3 baseline; single-partition contexts only)."""
+    m = _launch_args(kernel, grid, block, args, scalars)
+    _check(lib().pk_launch_direct(ctx, kernel, m[0], m[1], smem, m[2], m[3], m[4]), "pk_launch_direct")
 
 
 def pk_synchronize(ctx):

@@ -2323,6 +2323,51 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     return PK_OK;
 }
 
+int pk_launch_direct(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
+                     const void* const* args, const int64_t* scalars, int ns) {
+    if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
+    if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
+    if (c->host_only || c->P != 1 || c->world != 1)
+        return fail(PK_ERR_STATE, "pk_launch_direct: single-partition, single-process device contexts only");
+    const Kernel& K = c->kernels[k];
+    if (K.nargs && !args) return fail(PK_ERR_INVALID, "null args");
+    for (int w = 0; w < 3; ++w)
+        if (grid[w] < 0 || block[w] < 1) return fail(PK_ERR_INVALID, "bad grid/block");
+    void* inst[PK_MAX_ARGS];
+    void* argv[PK_MAX_ARGS + 1];
+    for (int a = 0; a < K.nargs; ++a) {
+        if (K.kinds[a] == PK_ARG_BUFFER) {
+            if (!args[a]) return fail(PK_ERR_INVALID, "null buffer argument");
+            const pk_buf b = *(const pk_buf*)args[a];
+            if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "argument " + std::to_string(a) + " is not a live buffer");
+            inst[a] = c->bufs[b].inst[0];
+            argv[a] = &inst[a];
+        } else {
+            inst[a] = nullptr;
+            argv[a] = const_cast<void*>(args[a]);
+        }
+    }
+    pk_partition part;  // the whole grid: blockIdx' = blockIdx (Eq. 8 with min = 0)
+    for (int d = 0; d < 3; ++d) {
+        part.min[d] = 0;
+        part.max[d] = grid[d];
+        part.grid[d] = grid[d];
+    }
+    argv[K.nargs] = &part;
+    if (int r = c->set_device(c->dev[0])) return r;
+    const dim3 g(grid[0], grid[1], grid[2]), bl(block[0], block[1], block[2]);
+    cudaError_t err;
+    if (K.launcher) {
+        LaunchInfo li{K.fn, g, bl, smem, c->stream[0], c->dev[0], inst, args, scalars, ns, part, nullptr, c, 0};
+        err = K.launcher(li);
+    } else {
+        err = cudaLaunchKernel(K.fn, g, bl, argv, smem, c->stream[0]);
+    }
+    if (err != cudaSuccess)
+        return fail(PK_ERR_CUDA, "direct launch of '" + K.name + "': " + cudaGetErrorName(err));
+    return PK_OK;
+}
+
 // ---- access recording (PK_TRACE_ACCESS build) ----
 int pk_trace_available(void) {
 #ifdef PK_TRACE_ACCESS

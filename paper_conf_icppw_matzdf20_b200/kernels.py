@@ -101,6 +101,7 @@ class Problem:
         if tiles:   # NEXT-2 tile partitions (tx, ty, tz), tx*ty*tz == P
             abi.pk_set_partition_shape(ctx, self.k, tiles)
         self.bufs = []
+        self.direct = False   # True: pk_launch_direct (the E3 single-GPU baseline, P = 1 only)
 
     def buffer(self, shape, elem_bytes=4, host=None, dev_ptrs=None):
         b = abi.pk_register_buffer(self.ctx, shape, elem_bytes, dev_ptrs=dev_ptrs, host_init=host)
@@ -108,7 +109,10 @@ class Problem:
         return b
 
     def launch(self, grid, block, args, scalars):
-        abi.pk_launch_partitioned(self.ctx, self.k, grid, block, args, scalars)
+        if self.direct:
+            abi.pk_launch_direct(self.ctx, self.k, grid, block, args, scalars)
+        else:
+            abi.pk_launch_partitioned(self.ctx, self.k, grid, block, args, scalars)
 
 
 def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None):

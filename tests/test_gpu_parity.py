@@ -390,6 +390,28 @@ def test_graph_replay_matches_eager_and_one_way(P):
         assert se[key] == sg[key], key
 
 
+def test_direct_launch_equals_partitioned_p1():
+    """pk_launch_direct (E3 baseline: the original single-GPU launch) computes exactly what
+    the library computes at P = 1, and refuses multi-partition contexts."""
+    t, p = synth.hotspot_grids(200, 1028)
+    ref, _ = _hotspot(t, p, 8, 1, kernel="hotspot2d_tbk")
+    ctx = gpu_ctx(1)
+    pr = K.hotspot2d_setup(ctx, t, p, 16, kernel="hotspot2d_tbk")
+    pr.direct = True
+    out = K.hotspot2d_iterate(pr, 8)
+    g = fetch(ctx, out, t.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, ref)
+    assert st["launches"] == 0          # nothing went through the partitioned path
+    ctx = gpu_ctx(2)
+    pr = K.hotspot2d_setup(ctx, t, p, 16)
+    pr.direct = True
+    with pytest.raises(abi.PkError):
+        K.hotspot2d_iterate(pr, 1)
+    abi.pk_finalize(ctx)
+
+
 @pytest.mark.parametrize("P", [1, 3])
 def test_failed_capture_falls_back_to_eager(P, monkeypatch):
     """A capture that fails (forced by the PK_DEBUG_FAIL_CAPTURE hook) must not lose the
