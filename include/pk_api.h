@@ -360,6 +360,8 @@ typedef struct {
     uint64_t timed_graph_launches;
     uint64_t host_cpu_ns;        /* thread CPU time spent inside pk_launch_partitioned (excludes time the
                                     thread is descheduled; a driver spinning on a full launch queue still counts) */
+    uint64_t streamed_bytes;     /* of moved_bytes: copied on a side stream while the consuming kernel ran */
+    uint64_t timed_eager_launches; /* launches whose partition kernels were timed (kernel_ms_max_launch) */
 } pk_stats;
 int pk_get_stats(pk_ctx ctx, pk_stats* out);   /* drains pending kernel timings */
 int pk_reset_stats(pk_ctx ctx);
@@ -374,8 +376,23 @@ enum {
                                         pk_stats.kernel_ms, and around every replayed graph launch ->
                                         pk_stats.graph_launch_ms (graph replay stays on) */
     PK_MODE_NO_GRAPHS = 1u << 5,     /* disable steady-state graph replay (see pk_launch_partitioned) */
-    PK_MODE_PUSH = 1u << 6           /* fused halo push, see below */
+    PK_MODE_PUSH = 1u << 6,          /* fused halo push, see below */
+    PK_MODE_NO_OVERLAP = 1u << 7     /* streamed operands are copied before the kernel instead (see below) */
 };
+/* Streamed operands -- the transfer overlapped with the kernel it feeds (B200 design; the
+ * paper synchronises every read before the launch, Fig. 4 l. 2-8).  A builtin may name one
+ * input argument it can consume while its copies are in flight (sgemm_tf32x3: B, the
+ * operand every row partition reads whole).  Its stale ranges for partition p
+ * are then copied on a side stream of p, granule by granule (copy engine: no SM), starting
+ * after p's own linear slab, each granule followed by a stream-front-end store of an
+ * arrival flag; p's kernel starts right away and its TMA producer polls the flag of a
+ * granule before loading it.  The side stream forks from p's stream after every hazard
+ * wait (so the copies only wait for data that is ready) and rejoins it behind the kernel.
+ * Counted in pk_stats.streamed_bytes (also in moved_bytes).  Single-process contexts;
+ * off with PK_MODE_GLOBAL_BARRIER and PK_MODE_NO_OVERLAP.  Only pieces pulled from ANOTHER
+ * GPU are streamed (a same-device D2D copy needs SMs the consuming kernel is holding;
+ * measured on a B200 it crawls); PK_STREAM_SAME_DEVICE=1 in the environment at pk_init
+ * streams virtual partitions' copies too (functional tests on one GPU). */
 /* PK_MODE_PUSH -- the transfer fused into the producing kernel (B200 design; the paper
  * only pulls).  For a kernel whose builtin can push its output (jacobi2d,
  * hotspot2d, hotspot2d_tbk, heat3d), the library predicts that the next reader of the

@@ -30,6 +30,7 @@ PK_MODE_GLOBAL_BARRIER = 1 << 3
 PK_MODE_TIME_KERNELS = 1 << 4
 PK_MODE_NO_GRAPHS = 1 << 5
 PK_MODE_PUSH = 1 << 6
+PK_MODE_NO_OVERLAP = 1 << 7
 
 
 class PkError(RuntimeError):
@@ -76,7 +77,8 @@ class pk_stats(C.Structure):
                 ("graph_replays", C.c_uint64), ("graph_captures", C.c_uint64),
                 ("strided_copies", C.c_uint64), ("copy_kernels", C.c_uint64), ("pushed_bytes", C.c_uint64),
                 ("collectives", C.c_uint64), ("graph_fallbacks", C.c_uint64),
-                ("graph_launch_ms", C.c_double), ("timed_graph_launches", C.c_uint64), ("host_cpu_ns", C.c_uint64)]
+                ("graph_launch_ms", C.c_double), ("timed_graph_launches", C.c_uint64), ("host_cpu_ns", C.c_uint64),
+                ("streamed_bytes", C.c_uint64), ("timed_eager_launches", C.c_uint64)]
 
 
 RANGE_CB = C.CFUNCTYPE(None, C.c_void_p, C.c_uint64, C.c_uint64)

@@ -7,7 +7,7 @@
 
 namespace pk {
 
-cudaError_t prepare_kernel(const void* fn, int dev, size_t smem, int threads, KernelDevInfo* out) {
+cudaError_t prepare_kernel(const void* fn, int dev, size_t smem, int threads, KernelDevInfo* out, bool occupancy) {
     static std::mutex mu;
     static std::map<std::tuple<const void*, int, size_t, int>, KernelDevInfo> done;
     std::lock_guard<std::mutex> g(mu);
@@ -26,8 +26,11 @@ cudaError_t prepare_kernel(const void* fn, int dev, size_t smem, int threads, Ke
         if (e != cudaSuccess) return e;
     }
     KernelDevInfo k;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k.resident, fn, threads, smem);
-    if (e != cudaSuccess) return e;
+    k.resident = 1;
+    if (occupancy) {
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&k.resident, fn, threads, smem);
+        if (e != cudaSuccess) return e;
+    }
     e = cudaDeviceGetAttribute(&k.sms, cudaDevAttrMultiProcessorCount, dev);
     if (e != cudaSuccess) return e;
     if (k.resident < 1) return cudaErrorInvalidConfiguration;  // cannot be resident at all

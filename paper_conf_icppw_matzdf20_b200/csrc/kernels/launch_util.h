@@ -19,7 +19,9 @@ struct KernelDevInfo {
 // launcher; `dev` must name it): raise fn's dynamic shared memory limit to `smem`
 // (when above the 48 KB default) and compute its residency, once per (fn, dev, smem,
 // threads).  Thread-safe.  Returns the first error of the attribute / occupancy calls.
-cudaError_t prepare_kernel(const void* fn, int dev, size_t smem, int threads, KernelDevInfo* out);
+// occupancy = false: only the attribute (cluster kernels, launched one tile per CTA).
+cudaError_t prepare_kernel(const void* fn, int dev, size_t smem, int threads, KernelDevInfo* out,
+                           bool occupancy = true);
 
 // Persistent grid size: min(work items, resident CTAs x SMs).
 inline unsigned persistent_grid(long long items, const KernelDevInfo& k) {

@@ -19,6 +19,19 @@ struct PushList {
     uint64_t dst[kMaxPush];
 };
 
+// Streamed operand (Builtin::stream_arg): the copies that make that argument valid on
+// the partition run on a side stream WHILE the kernel runs -- the transfer overlapped
+// with the computation it feeds (the B operand broadcast of C4).  The copy
+// of granule g (bytes [g * granule, (g + 1) * granule) of the instance) stores 1 into
+// flags[g] when it has landed; bit g of `wait` tells the kernel to poll flags[g]
+// (acquire) before it reads that granule.  wait == 0: nothing is in flight.
+constexpr int kMaxGranules = 64;
+struct Arrival {
+    const uint32_t* flags;   // device words [kMaxGranules] of this partition
+    uint64_t wait;
+    uint64_t granule;        // bytes
+};
+
 // Everything a launcher needs for one partition (Fig. 4 lines 10-19).
 struct LaunchInfo {
     const void* fn;
@@ -35,6 +48,7 @@ struct LaunchInfo {
     const PushList* push = nullptr;  // halo push of the push-capable output (nullptr / n = 0: none)
     pk_ctx ctx = nullptr;            // owning context and partition index (context_scratch)
     int part_index = -1;
+    Arrival arrival = {nullptr, 0, 0};  // streamed operand (Builtin::stream_arg), if any
 };
 
 // Device scratch of a launcher (e.g. N-body partial sums), owned by the context per
@@ -56,9 +70,14 @@ struct Builtin {
     int (*describe)(pk_ctx, pk_kernel);
     LauncherFn launcher;       // nullptr = generic cudaLaunchKernel
     int32_t push_arg = -1;     // output buffer argument the kernel can halo-push (LaunchInfo::push), -1: none
+    // input argument the kernel can consume while its copies are in flight (LaunchInfo::arrival),
+    // -1: none; stream_granule(scalars) = the granule in bytes (<= kMaxGranules granules per buffer)
+    int32_t stream_arg = -1;
+    uint64_t (*stream_granule)(const int64_t* scalars, int nscalars) = nullptr;
 };
 
 const Builtin* find_builtin(const char* name);
+const Builtin* find_builtin_by_fn(const void* fn);
 LauncherFn find_builtin_launcher(const void* fn);
 int32_t find_builtin_push_arg(const void* fn);
 

@@ -222,6 +222,8 @@ struct Kernel {
     std::vector<Tap> taps;
     LauncherFn launcher = nullptr;
     int32_t push_arg = -1;  // output buffer argument the kernel can halo-push (builtin capability)
+    int32_t stream_arg = -1;  // input argument consumed while its copies are in flight (builtin capability)
+    uint64_t (*stream_granule)(const int64_t*, int) = nullptr;
     uint64_t version = 0;  // bumps when taps change (region cache key)
 };
 
@@ -308,6 +310,15 @@ struct pk_ctx_s {
     bool capturing = false;      // inside a stream capture (no timing events: they would be graph nodes)
     cudaEvent_t ev_fork = nullptr;
     std::vector<cudaEvent_t> ev_join;
+    // streamed operands (Builtin::stream_arg): per partition a side stream for the copies
+    // that overlap the kernel, its fork/join events and kMaxGranules arrival flag words
+    std::vector<cudaStream_t> side;
+    std::vector<cudaEvent_t> ev_side_fork, ev_side_done;
+    std::vector<uint32_t*> arrive_flags;
+    // stream pieces whose source shares the destination's GPU too (off by default: measured on
+    // a B200, a same-device D2D copy crawls while the consuming kernel holds every SM, whereas a
+    // peer copy runs on the NVLink copy engines; PK_STREAM_SAME_DEVICE=1 at pk_init, for tests)
+    bool stream_same_dev = false;
 
     bool local(int p) const { return prank[p] == rank; }
     int set_device(int d) {
@@ -336,6 +347,7 @@ struct DriverApi {
     bool ok = false;
     CUresult (*WaitValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned) = nullptr;
     CUresult (*WriteValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned) = nullptr;
+    CUresult (*WriteValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned) = nullptr;
     CUresult (*GetAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr) = nullptr;
     CUresult (*GetErrorName)(CUresult, const char**) = nullptr;
 };
@@ -352,6 +364,7 @@ DriverApi load_drv() {
                q == cudaDriverEntryPointSuccess && *fn;
     };
     d.ok = get("cuStreamWaitValue64", (void**)&d.WaitValue64) && get("cuStreamWriteValue64", (void**)&d.WriteValue64) &&
+           get("cuStreamWriteValue32", (void**)&d.WriteValue32) &&
            get("cuMemGetAddressRange", (void**)&d.GetAddressRange) && get("cuGetErrorName", (void**)&d.GetErrorName);
     return d;
 }
@@ -636,6 +649,7 @@ static int init_impl(const pk_init_params* prm, const void* nccl_id, pk_host_all
     c->rank = prm->my_rank;
     c->world = prm->world_size;
     c->init_flags = prm->flags;
+    c->stream_same_dev = getenv("PK_STREAM_SAME_DEVICE") != nullptr;
     c->host_only = prm->flags & PK_INIT_HOST_ONLY;
     c->ipc = ag != nullptr && c->world > 1;
     c->allgather = ag;
@@ -906,6 +920,7 @@ static int drain_timing(pk_ctx c) {
         v = std::max(v, (double)ms);
     }
     for (auto& kv : mx) c->stats.kernel_ms_max_launch += kv.second;
+    c->stats.timed_eager_launches += mx.size();
     c->pending_timing.clear();
     return PK_OK;
 }
@@ -944,6 +959,14 @@ int pk_finalize(pk_ctx c) {
             for (auto& s : c->scratch[p])
                 if (s.first) { cudaSetDevice(c->dev[p]); cudaFree(s.first); }
         for (auto& r : c->scratch_retired) { cudaSetDevice(r.first); cudaFree(r.second); }
+        for (size_t p = 0; p < c->side.size(); ++p)
+            if (c->side[p]) {
+                cudaSetDevice(c->dev[p]);
+                cudaStreamDestroy(c->side[p]);
+                cudaEventDestroy(c->ev_side_fork[p]);
+                cudaEventDestroy(c->ev_side_done[p]);
+                cudaFree(c->arrive_flags[p]);
+            }
         for (int p = 0; p < c->P; ++p) {
             if (!c->local(p)) continue;
             cudaSetDevice(c->dev[p]);
@@ -1389,6 +1412,10 @@ int pk_register_kernel(pk_ctx c, const char* name, const void* fn, int nargs, co
     k.fn = fn;
     k.launcher = find_builtin_launcher(fn);  // a builtin __global__ keeps its own launch geometry
     k.push_arg = find_builtin_push_arg(fn);
+    if (const Builtin* bi = find_builtin_by_fn(fn)) {
+        k.stream_arg = bi->stream_arg;
+        k.stream_granule = bi->stream_granule;
+    }
     k.nargs = nargs;
     k.partition_dim = partition_dim;
     for (int i = 0; i < nargs; ++i) {
@@ -1500,7 +1527,7 @@ int pk_reset_stats(pk_ctx c) {
 
 int pk_set_mode(pk_ctx c, uint32_t flags) {
     if (!c) return fail(PK_ERR_INVALID, "bad argument");
-    if (flags & ~0x7Fu) return fail(PK_ERR_INVALID, "unknown mode flag");
+    if (flags & ~0xFFu) return fail(PK_ERR_INVALID, "unknown mode flag");
     if ((flags & PK_MODE_PUSH) && !c->host_only && !c->ipc)
         for (int p = 0; p < c->P; ++p)
             for (int q = 0; q < c->P; ++q)
@@ -1526,6 +1553,7 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
     a.moved_bytes += sign * d.moved_bytes;
     a.pushed_bytes += sign * d.pushed_bytes;
     a.collectives += sign * d.collectives;
+    a.streamed_bytes += sign * d.streamed_bytes;
     for (int i = 0; i < 16; ++i)
         for (int j = 0; j < 16; ++j) a.pair_bytes[i][j] += sign * d.pair_bytes[i][j];
 }
@@ -1736,6 +1764,71 @@ record:
     return PK_OK;
 }
 
+// Streamed operand (Builtin::stream_arg): the stale ranges of buffer `b` bound for partition
+// p are copied on p's side stream, granule by granule, while p's kernel runs; after the
+// last piece of granule g the stream front end stores 1 into flag g (cuStreamWriteValue32:
+// no SM is needed, so a kernel that occupies every SM while it polls cannot starve it).
+// The flags are reset on p's stream before the fork, i.e. after p's previous kernel.
+// Granules go in the order the consumer needs them: starting after p's own linear slab
+// (a row partition of the GEMM starts its K loop on the chunks it holds, see sgemm_tc.cu).
+static int issue_streamed(pk_ctx c, int p, int64_t b, const std::vector<CopyOp>& ops, uint64_t granule,
+                          Arrival* out) {
+    Buffer& B = c->bufs[b];
+    if (c->side.empty()) {
+        c->side.assign(c->P, nullptr);
+        c->ev_side_fork.assign(c->P, nullptr);
+        c->ev_side_done.assign(c->P, nullptr);
+        c->arrive_flags.assign(c->P, nullptr);
+    }
+    if (!c->side[p]) {
+        PK_CUDA(cudaStreamCreateWithFlags(&c->side[p], cudaStreamNonBlocking));
+        PK_CUDA(cudaEventCreateWithFlags(&c->ev_side_fork[p], cudaEventDisableTiming));
+        PK_CUDA(cudaEventCreateWithFlags(&c->ev_side_done[p], cudaEventDisableTiming));
+        PK_CUDA(cudaMalloc((void**)&c->arrive_flags[p], kMaxGranules * sizeof(uint32_t)));
+        PK_CUDA(cudaMemset(c->arrive_flags[p], 0, kMaxGranules * sizeof(uint32_t)));
+    }
+    uint32_t* flags = c->arrive_flags[p];
+    const uint64_t ng = (B.bytes + granule - 1) / granule;
+    struct Piece { uint64_t g, b, e; int src; };
+    std::vector<Piece> pieces;
+    uint64_t need = 0;
+    for (const CopyOp& o : ops)
+        for (uint64_t x = o.b; x < o.e;) {
+            const uint64_t g = x / granule, y = std::min(o.e, (g + 1) * granule);
+            pieces.push_back({g, x, y, o.src});
+            need |= 1ull << g;
+            x = y;
+        }
+    const uint64_t g0 = std::min<uint64_t>(ng - 1, (uint64_t)(p + 1) * B.bytes / c->P / granule);
+    std::stable_sort(pieces.begin(), pieces.end(), [&](const Piece& x, const Piece& y) {
+        const uint64_t rx = (x.g + ng - g0) % ng, ry = (y.g + ng - g0) % ng;
+        return rx != ry ? rx < ry : x.b < y.b;
+    });
+    for (uint64_t m = need; m; m &= m - 1)  // granules this launch copies: not arrived yet
+        PK_CU(WriteValue32((CUstream)c->stream[p], (CUdeviceptr)(flags + __builtin_ctzll(m)), 0u,
+                           CU_STREAM_WRITE_VALUE_DEFAULT));
+    PK_CUDA(cudaEventRecord(c->ev_side_fork[p], c->stream[p]));  // after every hazard wait on stream[p]
+    PK_CUDA(cudaStreamWaitEvent(c->side[p], c->ev_side_fork[p], 0));
+    for (size_t i = 0; i < pieces.size(); ++i) {
+        const Piece& x = pieces[i];
+        char* dst = (char*)B.inst[p] + x.b;
+        const char* src = (const char*)B.inst[x.src] + x.b;
+        if (c->dev[x.src] == c->dev[p])
+            PK_CUDA(cudaMemcpyAsync(dst, src, x.e - x.b, cudaMemcpyDeviceToDevice, c->side[p]));
+        else
+            PK_CUDA(cudaMemcpyPeerAsync(dst, c->dev[p], src, c->dev[x.src], x.e - x.b, c->side[p]));
+        c->stats.copies += 1;
+        c->stats.moved_bytes += x.e - x.b;
+        c->stats.streamed_bytes += x.e - x.b;
+        if (x.src < 16 && p < 16) c->stats.pair_bytes[x.src][p] += x.e - x.b;
+        if (i + 1 == pieces.size() || pieces[i + 1].g != x.g)  // granule complete
+            PK_CU(WriteValue32((CUstream)c->side[p], (CUdeviceptr)(flags + x.g), 1u, CU_STREAM_WRITE_VALUE_DEFAULT));
+    }
+    PK_CUDA(cudaEventRecord(c->ev_copy[p], c->side[p]));
+    *out = Arrival{flags, need, granule};
+    return PK_OK;
+}
+
 static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
                         const void* const* args, const int64_t* scalars, int ns) {
     if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
@@ -1912,6 +2005,18 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
     const uint64_t E = c->ipc ? ++c->epoch : 0;  // replicated: identical on every rank
 
     // ---- a4 + a5: transfers, pulled on the destination stream ----
+    // streamed operand: the copies of the kernel's stream_arg buffer overlap its kernel
+    std::vector<Arrival> arrival(P, Arrival{nullptr, 0, 0});
+    std::vector<uint8_t> side_pending(P, 0);
+    int64_t sbuf = -1;
+    uint64_t granule = 0;
+    if (!c->host_only && transfer && K.stream_arg >= 0 && K.stream_arg < K.nargs && bound[K.stream_arg] &&
+        K.stream_granule && c->world == 1 && !c->ipc && drv().ok &&
+        !(mode & (PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_OVERLAP))) {
+        granule = K.stream_granule(scalars, ns);
+        const Buffer& SB = *bound[K.stream_arg];
+        if (granule && (SB.bytes + granule - 1) / granule <= (uint64_t)kMaxGranules) sbuf = bid[K.stream_arg];
+    }
     if (!c->host_only) {
         if (transfer && !c->last_plan.empty()) {
             std::vector<size_t> order;
@@ -1982,9 +2087,15 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                         ++u;
                     return u;
                 };
+                std::vector<CopyOp> side_ops;
                 for (size_t t = 0; t < order.size();) {
                     const CopyOp& o = c->last_plan[order[t]];
                     if (!c->local(o.src) && !c->ipc) { ++t; continue; }
+                    if (o.buf == sbuf && (c->stream_same_dev || c->dev[o.src] != c->dev[p])) {
+                        side_ops.push_back(o);  // streamed: copied on the side stream under the kernel
+                        ++t;
+                        continue;
+                    }
                     const uint64_t len = o.e - o.b;
                     uint64_t pitch = 0;
                     size_t u = run2d(t, &pitch);
@@ -2063,7 +2174,12 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     if (o.src < 16 && p < 16) c->stats.pair_bytes[o.src][p] += moved;
                     t = u;
                 }
-                PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
+                if (!side_ops.empty()) {  // records ev_copy[p] on the side stream
+                    if (int r = issue_streamed(c, p, sbuf, side_ops, granule, &arrival[p])) return r;
+                    side_pending[p] = 1;
+                } else {
+                    PK_CUDA(cudaEventRecord(c->ev_copy[p], c->stream[p]));
+                }
                 if (c->ipc)
                     if (int r = ipc_signal(c, p, kFlagCopied, E)) return r;
                 for (size_t t = i; t < j; ++t) {
@@ -2250,6 +2366,7 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
             if (K.launcher) {
                 LaunchInfo li{K.fn, g, bl, smem, c->stream[p], c->dev[p], inst, args, scalars, ns, part,
                               push[p].n ? &push[p] : nullptr, c, p};
+                li.arrival = arrival[p];
                 err = K.launcher(li);
             } else {
                 err = cudaLaunchKernel(K.fn, g, bl, argv, smem, c->stream[p]);
@@ -2276,6 +2393,14 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     if (writes || !track) c->bufs[bid[a]].last_writer[p] = (P > 1) ? W_KERNEL : W_NONE;
                 }
         }
+        // streamed copies rejoin their partition's stream behind its kernel, so everything
+        // later on that stream (and a graph's join) is ordered after them
+        for (int p = 0; p < P; ++p)
+            if (side_pending[p]) {
+                if (int r = c->set_device(c->dev[p])) return r;
+                PK_CUDA(cudaEventRecord(c->ev_side_done[p], c->side[p]));
+                PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_side_done[p], 0));
+            }
     } else {
         for (int p = 0; p < P; ++p)
             if (!(*regs)[p].empty && c->local(p)) c->stats.kernel_launches += 1;
@@ -2448,6 +2573,16 @@ void* context_scratch(const LaunchInfo& li, int slot, size_t bytes, cudaError_t*
     if (s.first) c->scratch_retired.push_back({c->dev[li.part_index], s.first});
     s = {p, bytes};
     return p;
+}
+
+const Builtin* find_builtin_by_fn(const void* fn) {
+    if (!fn) return nullptr;
+    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk", "heat3d",
+                          "heat3d_regs", "heat3d_tb2", "nbody", "sgemm_tf32x3"}) {
+        const Builtin* b = find_builtin(n);
+        if (b && b->fn == fn) return b;
+    }
+    return nullptr;
 }
 
 int32_t find_builtin_push_arg(const void* fn) {

@@ -1,0 +1,10 @@
+# round 2, call 12: GEMM v3 (CTA pairs, cta_group::2): correctness first, then bench + ncu
+timeout 300 python scripts/gemm_debug.py 256x256x512 384x512x1024 640x520x2048 2048x2048x16384
+timeout 900 python -m pytest tests -m gpu -q -x -k "gemm or sgemm or c4" > gpurun_out/r02_12_gemm.log 2>&1; echo "gemm tests: $(tail -1 gpurun_out/r02_12_gemm.log)"
+grep -E "^E |FAILED" gpurun_out/r02_12_gemm.log | head -20
+for P in 1 4; do
+timeout 300 python bench.py --workload sgemm --parts $P --steps 6 --no-e2e --no-cpu-baseline --no-e3 > /tmp/s.json 2> /tmp/s.err
+tail -1 /tmp/s.json | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('sgemm P$P', round(d['value'],1), round(d['ms_per_step'],2), 'frac', round(d['roofline']['frac'],3), d['transfers']['moved_bytes'], d['clocks']['sm_mhz'], d['clocks']['reasons'])" || tail -5 /tmp/s.err
+done
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_sgemm -c 1 -o gpurun_out/r02_sgemm_v3 python scripts/gemm_debug.py 4096x4096x16384 > gpurun_out/r02_12_ncu.log 2>&1; tail -1 gpurun_out/r02_12_ncu.log
+python scripts/ncu_summary.py gpurun_out/r02_sgemm_v3.ncu-rep | grep -E "time|tensor|dram__bytes|issue"

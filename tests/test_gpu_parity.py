@@ -357,6 +357,51 @@ def test_gemm_oracle_and_bitwise(m, n, k):
         assert st["moved_bytes"] == st["stale_bytes"]
 
 
+def _gemm_chain(a, b, P, launches, mode=0):
+    """X_{t+1} = A X_t (the bench's C4 step): every launch reads the operand the previous
+    launch wrote in row slabs, so every launch broadcasts (P-1)/P of it."""
+    m, k = a.shape
+    n = b.shape[1]
+    ctx = gpu_ctx(P, mode)
+    pr, _ = K.sgemm_program(ctx, a, b, launches=0)
+    grid, blk, sc = pr.geom
+    ab, bb, cb = pr.abc
+    out = cb
+    for t in range(launches):
+        x, y = (bb, cb) if t % 2 == 0 else (cb, bb)
+        pr.launch(grid, blk, [ab, x, y, m, n, k], sc)
+        out = y
+    g = fetch(ctx, out, (m, n))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return g, st
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_gemm_streamed_operand_overlap(P, monkeypatch):
+    """Streamed B (the operand broadcast overlapped with the GEMM, pk_api.h): bit-identical to
+    the copy-before-kernel path (PK_MODE_NO_OVERLAP) and to 1-way, every stale byte of the
+    operand moved on the side stream, graphs captured and replayed without a fallback."""
+    monkeypatch.setenv("PK_STREAM_SAME_DEVICE", "1")   # virtual partitions: stream the D2D copies too
+    m = k = n = 1024
+    a, b = synth.gemm_operands(m, n, k)
+    a *= np.float32((3.0 / k) ** 0.5)
+    launches = 6
+    g1, _ = _gemm_chain(a, b, 1, launches)
+    gs, ss = _gemm_chain(a, b, P, launches)
+    gn, sn = _gemm_chain(a, b, P, launches, abi.PK_MODE_NO_OVERLAP)
+    assert np.array_equal(gs, g1) and np.array_equal(gn, g1)
+    per = (P - 1) * k * n * 4     # the operand X, every launch (A moves only where its linear
+    assert ss["streamed_bytes"] == launches * per     # H2D split misses the tile rows: P = 3)
+    assert ss["stale_bytes"] == ss["moved_bytes"] == sn["moved_bytes"] == sn["stale_bytes"]
+    assert sn["streamed_bytes"] == 0
+    assert ss["graph_fallbacks"] == 0 and ss["graph_replays"] >= 1
+    # the chain against the oracle: the same X_t from the fp64 product of the GPU's own X_{t-1}
+    ref = ok.gemm(a, _gemm_chain(a, b, 1, launches - 1)[0])
+    good, err = rel_ok(gs, ref, 1e-4)
+    assert good, err
+
+
 def test_gemm_read_pattern_placement_moves_nothing():
     """NEXT-1: operands uploaded where the launch reads them (pk_copy_from_host_for)."""
     m, n, k = 768, 512, 256
