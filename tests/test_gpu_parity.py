@@ -42,6 +42,44 @@ def test_c1_jacobi_512_p2_oracle_stale_and_bitwise():
     assert s2["kernel_launches"] == 20 and s2["pair_bytes"][0][1] == s2["pair_bytes"][1][0] == 20400
 
 
+@pytest.mark.parametrize("single", [False, True])
+def test_paper_vs_validity_tracker_measured_on_gpu(single):
+    """SURVEY NEXT-1 / §8(c) paper-vs-validity pins, measured through the library on the GPU
+    (the hand derivations are in tests/test_oracle_regions_shadow.py): Jacobi 64^2 at P = 3
+    moves exactly 2,540 / 1,056 / 992... B per launch with shared copies, 1,056 B per launch
+    from the second on without them; the same GEMM launched twice moves (P-1)|B|
+    once vs twice.  Results bit-identical to 1-way in both modes."""
+    mode = abi.PK_MODE_SINGLE_OWNER if single else 0
+    u = synth.uniform((64, 64), 0, 1, seed=64)
+    ref, _ = _jacobi(u, 6, 1)
+    ctx = gpu_ctx(3, mode)
+    pr = K.Problem(ctx, "jacobi2d")
+    b0, b1 = pr.buffer((64, 64), 4, host=u), pr.buffer((64, 64), 4, host=u)
+    grid, blk, sc = K.jacobi2d_launch(64, 64)
+    per = []
+    for t in range(6):
+        a, b = (b0, b1) if t % 2 == 0 else (b1, b0)
+        abi.pk_reset_stats(ctx)
+        pr.launch(grid, blk, [a, b, 64, 64], sc)
+        st = abi.pk_get_stats(ctx)
+        assert st["moved_bytes"] == st["stale_bytes"]
+        per.append(st["moved_bytes"])
+    g = fetch(ctx, b0, (64, 64))
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, ref)
+    assert per == ([2540, 1056, 1056, 1056, 1056, 1056] if single else [2540, 1056, 992, 992, 992, 992])
+    m, n, k = 512, 512, 192           # 4 tile rows: one per partition, A's linear slabs aligned
+    a_, b_ = synth.gemm_operands(m, n, k)
+    g1, _ = _gemm(a_, b_, 1)
+    ctx = gpu_ctx(4, mode)
+    pr, cb = K.sgemm_program(ctx, a_, b_, launches=2)
+    g = fetch(ctx, cb, (m, n))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, g1)
+    assert st["moved_bytes"] == st["stale_bytes"] == (2 if single else 1) * 3 * k * n * 4
+
+
 def test_c1_harmonic_fixed_point_bit_exact_on_gpu():
     n = 512
     i = np.arange(n, dtype=np.float32)[:, None]
@@ -419,6 +457,8 @@ def test_gemm_read_pattern_placement_moves_nothing():
     abi.pk_finalize(ctx)
     assert np.array_equal(g, ref)
     assert st["stale_bytes"] == 0 == st["moved_bytes"]
+    good, err = rel_ok(g, ok.gemm(a, b), 1e-4)     # and the oracle, not only the 1-way run
+    assert good, err
 
 
 # ------------------------------------------------------------------ steady-state graph replay
