@@ -179,6 +179,24 @@ class NvlinkCounters:
                 "source": "NVML NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX/RX over the timed region"}
 
 
+def nvlink_check(measured, st, P, part_dev, world):
+    """Set NVML's NVLink byte counters beside the library's inter-GPU bytes (moved + pushed
+    between partitions on different GPUs): on an NVSwitch box the NVML RX bytes must cover them
+    (protocol overhead and other traffic only add)."""
+    if measured is None:
+        return None
+    if world > 1:
+        lib = st["moved_bytes"] + st["pushed_bytes"]        # SPMD: every cross-rank byte crosses GPUs
+    else:
+        devs = [part_dev[p % len(part_dev)] for p in range(P)] if part_dev else [0] * P
+        lib = sum(st["pair_bytes"][q][p] for q in range(min(P, 16)) for p in range(min(P, 16))
+                  if devs[q] != devs[p]) + (st["pushed_bytes"] if len(set(devs)) > 1 else 0)
+    out = dict(measured)
+    out["library_interdevice_bytes"] = int(lib)
+    out["rx_covers_library_bytes"] = (measured["rx_bytes"] >= lib) if lib else None
+    return out
+
+
 def measure_tf32_ceiling(device, n=8192, reps=10):
     """Dense TF32 tensor-core ceiling of this GPU in this run: cuBLAS through torch.matmul on
     fp32 inputs with TF32 enabled (SURVEY.md §8(d) "measured ceilings"), CUDA events."""
@@ -730,7 +748,7 @@ def main():
             "thread_cpu": st["host_cpu_ns"] / 1e3 / max(1, st["launches"]),
             "note": "includes time blocked in CUDA calls once the launch queue is full (launches are issued "
                     "far ahead of the GPU)"},
-        "nvlink_nvml": nvlink_measured,
+        "nvlink_nvml": nvlink_check(nvlink_measured, st, P, devices if world == 1 else None, world),
         "us_per_launch": elapsed_ms * 1e3 * getattr(w, "sweeps", 1) / max(1, w.iters * args.steps),
     })
 
