@@ -296,11 +296,24 @@ class Workload:
             return tile
         g = max(1, getattr(self, "gpus_used", 1))
         if self.name == "hotspot2d":
-            # 64 (not the marginally faster 96) keeps the row blocks divisible among 8 slabs
-            return self.K.HOTSPOT_TY if self.shape[0] // g >= 4096 else 64
+            if getattr(self, "variant", None):
+                return self.K.HOTSPOT_TY
+            # the partitions of the full grid one process runs: one per rank (SPMD) or all (one process)
+            parts = g if g > 1 else 1
+            return self.K.hotspot2d_tbk_rows(self.shape[0], self.shape[1], getattr(self, "sweeps_arg", 4), parts,
+                                             self.ctas())
         if self.name == "heat3d":
             return min(64, max(16, (self.shape[0] // g) // 16 // 8 * 8))
         return 0
+
+    def ctas(self):
+        """Persistent CTAs of hotspot2d_tbk on this GPU: 3 per SM (2 for K > 4)."""
+        try:
+            import torch
+            sms = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+        except Exception:
+            sms = 148
+        return sms * (3 if getattr(self, "sweeps_arg", 4) <= 4 else 2)
 
     def setup(self, ctx):
         K = self.K

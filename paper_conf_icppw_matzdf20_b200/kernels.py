@@ -41,6 +41,28 @@ def tbk_cols(k):
 TBK_COLS = tbk_cols(4)
 
 
+def hotspot2d_tbk_rows(h, w, k=4, parts=1, ctas=444, lo=48, hi=136):
+    """Rows per logical block of "hotspot2d_tbk" for an h x w grid split into `parts` row
+    slabs, run by a persistent grid of `ctas` CTAs (148 SMs x 3): the tiles of one partition
+    are processed in ceil(tiles / ctas) rounds, and a tile of TY rows costs about
+    TY + 2K (halo rows recomputed) + a fixed overhead, so TY minimises rounds x (TY + 2K + 8).
+    Measured on one B200 (`scripts/r02/gpu_20.sh`): 16384 rows TY 128 / 131 = 1998 / 2013
+    GLUP/s (4480 vs 4410 tiles: 11 vs 10 rounds); 2048 rows (a rank's share at N = 8) TY 64 /
+    54 = 1541 / 1626; larger TY than the model's range measured slower (146 / 164 / 218 at
+    16384 rows: 1982 / 1924 / 1860)."""
+    ncb = _cdiv(w, tbk_cols(k))
+    best = None
+    for ty in range(lo, hi + 1):
+        per = _cdiv(_cdiv(h, ty), parts)          # row blocks of the largest partition
+        rounds = _cdiv(per * ncb, ctas)
+        if rounds < 3 and ty > lo:
+            continue                              # <= 2 tiles per CTA measured poorly (TY 103 at 2048 rows)
+        cost = rounds * (ty + 2 * k + 8)
+        if best is None or cost < best[0] or (cost == best[0] and ty > best[1]):
+            best = (cost, ty)
+    return best[1]
+
+
 def hotspot2d_tbk_launch(h, w, ty=HOTSPOT_TY, k=4):
     """Logical block = tbk_cols(k) columns x ty rows, k sweeps per launch (scalar 3,
     K in 2, 3, 4, 6, 8); scalar 4 = the block's column count."""

@@ -31,17 +31,24 @@ def test_reference_arm_json_line():
 def test_block_depth_follows_the_slab_per_gpu():
     b = _bench_module()
     from paper_conf_icppw_matzdf20_b200 import kernels as K
-    for name, shape, expect in (("hotspot2d", (16384, 16384), {1: 128, 2: 128, 4: 128, 8: 64}),
-                                ("heat3d", (1024, 1024, 1024), {1: 64, 2: 32, 4: 16, 8: 16})):
-        w = b.Workload.__new__(b.Workload)
-        w.name, w.shape, w.K, w.tile = name, shape, K, 0
-        for g, depth in expect.items():
-            w.gpus_used = g
-            assert w.block_depth() == depth, (name, g)
-            # the slab of each GPU is a whole number of blocks (balanced 1-D partitions)
-            assert (shape[0] // depth) % g == 0
-        w.tile = 40
-        assert w.block_depth() == 40          # --tile wins
+    w = b.Workload.__new__(b.Workload)
+    w.name, w.shape, w.K, w.tile = "heat3d", (1024, 1024, 1024), K, 0
+    for g, depth in {1: 64, 2: 32, 4: 16, 8: 16}.items():
+        w.gpus_used = g
+        assert w.block_depth() == depth, g
+        assert (1024 // depth) % g == 0       # the slab of each GPU is a whole number of blocks
+    w.tile = 40
+    assert w.block_depth() == 40              # --tile wins
+    # Hotspot: rows per tile from the persistent grid's rounds (444 CTAs)
+    assert K.hotspot2d_tbk_rows(16384, 16384) == 131       # 126 x 35 tiles: 10 rounds (128 rows: 11)
+    assert K.hotspot2d_tbk_rows(16384, 16384, parts=8) == 54   # a rank's 38 x 35 tiles: 3 rounds
+    for h, parts in ((16384, 1), (16384, 2), (16384, 4), (16384, 8), (2048, 1), (300, 1)):
+        ty = K.hotspot2d_tbk_rows(h, 16384, parts=parts)
+        ncb = -(-16384 // K.tbk_cols(4))
+        cost = lambda t: -(-(-(-(-(-h // t)) // parts)) * ncb // 444) * (t + 16)
+        rounds = lambda t: -(-(-(-(-(-h // t)) // parts)) * ncb // 444)
+        ok_t = [t for t in range(48, 137) if rounds(t) >= 3] or [48]
+        assert 48 <= ty <= 136 and all(cost(ty) <= cost(t) for t in ok_t)
 
 
 def test_reference_arm_under_torchrun_uses_all_host_cores():

@@ -45,7 +45,8 @@ def _tol_ok(g, o, rms, rtol):
 # ------------------------------------------------------------------ C2 Hotspot 16384^2, 100 it
 def test_c2_hotspot_fullsize_tbk_sampled():
     h = w = 16384
-    iters, k, ty = 100, 4, K.HOTSPOT_TY       # bench default: hotspot2d_tbk, K = 4, TY = 128
+    # the bench default: hotspot2d_tbk, K = 4, TY from the persistent grid's rounds (131 at 16384 rows)
+    iters, k, ty = 100, 4, K.hotspot2d_tbk_rows(16384, 16384)
     t, p = synth.hotspot_grids(h, w)
     res = {}
     for P in (1, 4):
@@ -55,9 +56,21 @@ def test_c2_hotspot_fullsize_tbk_sampled():
         st = abi.pk_get_stats(ctx)
         abi.pk_finalize(ctx)
         if P > 1:
-            # temp: K halo rows each way per cut per launch; power: K-1 rows once (linear H2D is row-aligned)
+            # launch 1 reads temp (K halo rows) and power (K - 1 rows) around each partition's rows as
+            # uploaded (linear slabs of H / P rows, which 131-row blocks need not match); every later
+            # launch moves K temperature rows each way per cut
             row = w * 4
-            assert st["stale_bytes"] == st["moved_bytes"] == (iters * 2 + 2 * (k - 1)) * row * (P - 1)
+            nb = -(-h // ty)
+            first = 0
+            for q in range(P):
+                r0, r1 = q * nb // P * ty, min(h, (q + 1) * nb // P * ty)      # partition rows (Q1)
+                s0, s1 = q * h // P, (q + 1) * h // P                           # linear H2D slab (Q2)
+                for dil in (k, k - 1):
+                    a, b = max(0, r0 - dil), min(h, r1 + dil)
+                    first += (b - a) - max(0, min(b, s1) - max(a, s0))
+            launches = iters // k
+            want = first * row + (launches - 1) * 2 * k * row * (P - 1)
+            assert st["stale_bytes"] == st["moved_bytes"] == want
     assert np.array_equal(res[1], res[4])
     g = res[1]
     rms = float(np.sqrt(np.mean(g.astype(np.float64) ** 2)))
