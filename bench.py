@@ -186,7 +186,8 @@ def nvlink_check(measured, st, P, part_dev, world):
     if measured is None:
         return None
     if world > 1:
-        lib = st["moved_bytes"] + st["pushed_bytes"]        # SPMD: every cross-rank byte crosses GPUs
+        # SPMD (rank 0's view): the bytes rank 0 pulled; with one GPU per rank they all crossed NVLink
+        lib = st["moved_bytes"] + st["pushed_bytes"]
     else:
         devs = [part_dev[p % len(part_dev)] for p in range(P)] if part_dev else [0] * P
         lib = sum(st["pair_bytes"][q][p] for q in range(min(P, 16)) for p in range(min(P, 16))
@@ -647,6 +648,7 @@ def main():
     w.step()
     sh = abi.pk_get_stats(ctx)
     abi.pk_synchronize(ctx)
+    st_local = dict(st)        # this rank's own counters (its GPU's NVLink bytes are what NVML sees here)
     if dist:
         tt = torch.tensor([elapsed_ms, st["kernel_launches"], st["moved_bytes"], st["copies"], st["pushed_bytes"]],
                           dtype=torch.float64)
@@ -761,7 +763,7 @@ def main():
             "thread_cpu": st["host_cpu_ns"] / 1e3 / max(1, st["launches"]),
             "note": "includes time blocked in CUDA calls once the launch queue is full (launches are issued "
                     "far ahead of the GPU)"},
-        "nvlink_nvml": nvlink_check(nvlink_measured, st, P, devices if world == 1 else None, world),
+        "nvlink_nvml": nvlink_check(nvlink_measured, st_local, P, devices if world == 1 else None, world),
         "us_per_launch": elapsed_ms * 1e3 * getattr(w, "sweeps", 1) / max(1, w.iters * args.steps),
     })
 
