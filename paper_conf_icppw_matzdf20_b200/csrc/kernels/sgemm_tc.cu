@@ -72,6 +72,9 @@
 namespace pk {
 namespace {
 
+#ifndef PK_SGEMM_DIAG
+#define PK_SGEMM_DIAG 8
+#endif
 constexpr int BM = 128, BN = 256, BK = 16, STAGES = 6;  // BM: rows per CTA (256 per pair)
 constexpr int BNH = BN / 2;                         // B columns held by each CTA of the pair
 constexpr int A_TILE = BM * BK * 4;                 // 8 KB
@@ -208,9 +211,12 @@ __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
     return v;
 }
 
-// chunk of K processed j-th by a tile in tile row `rt` (of `nrt`): diagonal start, wrap
+// chunk of K processed j-th by a tile in tile row `rt` (of `nrt`): diagonal start, wrap.  The
+// start is quantised to eighths of K (the row slabs of up to 8 partitions): the pairs running
+// at the same time then mostly stream the same B k-slices, which L2 serves once
+constexpr int kDiagSlabs = PK_SGEMM_DIAG;
 __device__ __forceinline__ int chunk_at(int j, int64_t rt, int64_t nrt, int nchunks) {
-    const int c0 = (int)((rt * nchunks) / nrt);  // rt / nrt: tile-row pair / pairs of the full grid
+    const int c0 = (int)(((rt * kDiagSlabs) / nrt) * nchunks / kDiagSlabs);  // rt / nrt: pair / pairs of the grid
     const int c = c0 + j;
     return c >= nchunks ? c - nchunks : c;
 }
