@@ -2015,7 +2015,11 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         !(mode & (PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_OVERLAP))) {
         granule = K.stream_granule(scalars, ns);
         const Buffer& SB = *bound[K.stream_arg];
-        if (granule && (SB.bytes + granule - 1) / granule <= (uint64_t)kMaxGranules) sbuf = bid[K.stream_arg];
+        bool alone = true;  // the buffer bound to another argument too (C = A A): those reads do not poll
+        for (int a = 0; a < K.nargs; ++a)
+            if (a != K.stream_arg && bound[a] && bid[a] == bid[K.stream_arg]) alone = false;
+        if (alone && granule && (SB.bytes + granule - 1) / granule <= (uint64_t)kMaxGranules)
+            sbuf = bid[K.stream_arg];
     }
     if (!c->host_only) {
         if (transfer && !c->last_plan.empty()) {

@@ -440,6 +440,26 @@ def test_gemm_streamed_operand_overlap(P, monkeypatch):
     assert good, err
 
 
+def test_gemm_operand_aliased_is_not_streamed(monkeypatch):
+    """C = A A: the streamed argument's buffer is also the A operand, whose loads do not poll the
+    arrival flags, so its copies must land before the kernel (no streaming)."""
+    monkeypatch.setenv("PK_STREAM_SAME_DEVICE", "1")
+    n = 512
+    a, _ = synth.gemm_operands(n, n, n)
+    ref = ok.gemm(a, a)
+    ctx = gpu_ctx(3)
+    pr = K.Problem(ctx, "sgemm_tf32x3")
+    ab, cb = pr.buffer((n, n), 4, host=a), pr.buffer((n, n), 4)
+    grid, blk, sc = K.sgemm_launch(n, n, n)
+    pr.launch(grid, blk, [ab, ab, cb, n, n, n], sc)
+    g = fetch(ctx, cb, (n, n))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    assert st["streamed_bytes"] == 0 and st["moved_bytes"] == st["stale_bytes"] > 0
+    good, err = rel_ok(g, ref, 1e-4)
+    assert good, err
+
+
 def test_gemm_read_pattern_placement_moves_nothing():
     """NEXT-1: operands uploaded where the launch reads them (pk_copy_from_host_for)."""
     m, n, k = 768, 512, 256
