@@ -22,7 +22,7 @@ from paper_conf_icppw_matzdf20_b200 import abi
 from paper_conf_icppw_matzdf20_b200 import kernels as K
 
 
-def _pingpong(kid, geom, a, b, extra, n):
+def _pingpong(geom, a, b, extra, n):
     grid, blk, sc = geom
     out = []
     for t in range(n):
@@ -36,7 +36,7 @@ def jacobi2d(ctx, make, h=72, w=100):
     kid = abi.pk_builtin_kernel(ctx, "jacobi2d")
     u0, u1 = make((h, w), 4, u), make((h, w), 4, u)
     geom = K.jacobi2d_launch(h, w)
-    return kid, _pingpong(kid, geom, u0, u1, ([], [h, w]), 2), {u0: ((h, w), 4), u1: ((h, w), 4)}
+    return kid, _pingpong(geom, u0, u1, ([], [h, w]), 2), {u0: ((h, w), 4), u1: ((h, w), 4)}
 
 
 def _hotspot(name, ctx, make, h, w, ty, k=4, bdx=K.HOTSPOT_BDX):
