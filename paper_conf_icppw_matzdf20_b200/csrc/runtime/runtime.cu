@@ -2579,39 +2579,28 @@ void* context_scratch(const LaunchInfo& li, int slot, size_t bytes, cudaError_t*
     return p;
 }
 
+// the one registry of builtin kernels (kernels/*.cu)
+static const Builtin* const kAllBuiltins[] = {
+    &kBuiltinJacobi2d,     &kBuiltinHotspot2dTma, &kBuiltinHotspot2d, &kBuiltinHotspot2dTb2, &kBuiltinHotspot2dTbk,
+    &kBuiltinHeat3dTma,    &kBuiltinHeat3d,       &kBuiltinHeat3dTb2, &kBuiltinNbody,        &kBuiltinSgemm};
+
 const Builtin* find_builtin_by_fn(const void* fn) {
     if (!fn) return nullptr;
-    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk", "heat3d",
-                          "heat3d_regs", "heat3d_tb2", "nbody", "sgemm_tf32x3"}) {
-        const Builtin* b = find_builtin(n);
-        if (b && b->fn == fn) return b;
-    }
+    for (const Builtin* b : kAllBuiltins)
+        if (b->fn == fn) return b;
     return nullptr;
 }
-
 int32_t find_builtin_push_arg(const void* fn) {
-    if (!fn) return -1;
-    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_tbk", "heat3d", "heat3d_tb2"}) {
-        const Builtin* b = find_builtin(n);
-        if (b && b->fn == fn) return b->push_arg;
-    }
-    return -1;
+    const Builtin* b = find_builtin_by_fn(fn);
+    return b ? b->push_arg : -1;
 }
 LauncherFn find_builtin_launcher(const void* fn) {
-    if (!fn) return nullptr;
-    for (const char* n : {"jacobi2d", "hotspot2d", "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk", "heat3d", "heat3d_regs", "heat3d_tb2",
-                          "nbody", "sgemm_tf32x3"}) {
-        const Builtin* b = find_builtin(n);
-        if (b && b->fn == fn) return b->launcher;
-    }
-    return nullptr;
+    const Builtin* b = find_builtin_by_fn(fn);
+    return b ? b->launcher : nullptr;
 }
 const Builtin* find_builtin(const char* name) {
     if (!name) return nullptr;
-    static const Builtin* all[] = {&kBuiltinJacobi2d, &kBuiltinHotspot2dTma, &kBuiltinHotspot2d, &kBuiltinHotspot2dTb2,
-                                   &kBuiltinHotspot2dTbk, &kBuiltinHeat3dTma, &kBuiltinHeat3d, &kBuiltinHeat3dTb2, &kBuiltinNbody,
-                                   &kBuiltinSgemm};
-    for (const Builtin* b : all)
+    for (const Builtin* b : kAllBuiltins)
         if (std::strcmp(b->name, name) == 0) return b;
     return nullptr;
 }
