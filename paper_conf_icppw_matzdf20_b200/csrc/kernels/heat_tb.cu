@@ -13,14 +13,15 @@
 // 20 rows [y0-2, y0+18) x 1 plane, out-of-grid columns/rows zero-filled, the plane
 // index clamped -- into a 6-slot mbarrier ring, 3 CTAs/SM.  4 consumer warps march z; warp w
 // owns rows y0+4w .. +3, a lane owns 4 columns.  Per input plane q a warp computes
-// sweep 1 of plane q-1 on its 4 rows plus one halo row above and below (6 rows,
-// inputs from shared memory) into a register window of 3 planes x 6 rows, and
-// sweep 2 of plane q-2 on its own 4 rows from that window, which it stores.
-// x neighbours are warp shuffles; lanes 0 and 31 are halo lanes whose outer
-// column is wrong after each sweep (shuffle wrap), so lanes 1..30 store: 120
-// owned columns.  Halo rows, columns and planes of sweep 1 are recomputed by the
-// blocks that need them from identical inputs in identical order, so P-way
-// launches are bit-identical to 1-way; no barrier among consumers.
+// sweep 1 of plane q-1 on its 4 rows (warp 0 also the block's halo row above, warp 3
+// the one below; inputs from shared memory) into a register window of 3 planes x 4
+// rows, hands its top and bottom sweep-1 rows to its neighbours through shared memory
+// (one named barrier among the consumer warps per plane), and computes sweep 2 of
+// plane q-2 on its own 4 rows, which it stores.  x neighbours are warp shuffles;
+// lanes 0 and 31 are halo lanes whose outer column is wrong after each sweep (shuffle
+// wrap), so lanes 1..30 store: 120 owned columns.  Halo rows, columns and planes of
+// sweep 1 are recomputed by the blocks that need them from identical inputs in
+// identical order, so P-way launches are bit-identical to 1-way.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -44,13 +45,16 @@ constexpr int kRW = 4;                    // owned rows per consumer warp
 constexpr int kNW = 4;                    // consumer warps (3 CTAs/SM; measured 6 warps x 2 CTAs: -4 %)
 constexpr int kRows = kRW * kNW;          // owned rows per block (16)
 constexpr int kBoxRows = kRows + 4;       // rows y0-2 .. y0+kRows+1
-constexpr int kL1 = kRW + 2;              // sweep-1 rows per warp (one halo row each side)
 #ifndef PK_HEATTB_NS
 #define PK_HEATTB_NS 6
 #endif
 constexpr int kNS = PK_HEATTB_NS;         // plane ring depth (3 CTAs x 6 x 10 KB per SM; 7 slots: -2 %)
 constexpr int kSlot = kBoxRows * kCols;   // floats per plane slot (14 KB)
-constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + 2 * kNS * 8 + 128;
+// sweep-1 rows shared between warps: per plane, each warp's top and bottom own row plus the
+// block's two halo rows (10 rows), double-buffered by plane parity
+constexpr int kXRows = 2 * kNW + 2;
+constexpr size_t kXBytes = (size_t)2 * kXRows * kCols * 4;
+constexpr size_t kSmem = (size_t)kNS * kSlot * 4 + kXBytes + 2 * kNS * 8 + 128;
 #ifndef PK_HEATTB_PNS
 #define PK_HEATTB_PNS 256
 #endif
@@ -84,9 +88,9 @@ __device__ __forceinline__ float4 sweep(const float4& c, const float4& zm, const
 }
 
 template <bool PUSH, bool EDGE>
-__device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint64_t* empty, float* __restrict__ uout,
-                                        int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
-                                        int lane, int warp, const PushList& push);
+__device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t* full, uint64_t* empty,
+                                        float* __restrict__ uout, int64_t D, int64_t H, int64_t W, int64_t c0,
+                                        int64_t y0, int64_t k0, int nq, int lane, int warp, const PushList& push);
 
 // 3 CTAs/SM = 128 registers per thread.  __maxnreg__(136) (15 warps x 17 allocation units)
 // removed most spills but measured slower (1238-1264 vs 1331-1349 GLUP/s, scripts/gpu_run100.sh)
@@ -101,7 +105,8 @@ __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
     // 128-B aligned ring; pointer arithmetic on the shared array (not a uintptr_t round
     // trip) keeps the shared address space visible, so the loads below are LDS, not LD
     float* ring = reinterpret_cast<float*>(smem_raw + ((128u - ((uint32_t)(uintptr_t)smem_raw & 127u)) & 127u));
-    uint64_t* full = reinterpret_cast<uint64_t*>(ring + (size_t)kNS * kSlot);
+    float* xbuf = ring + (size_t)kNS * kSlot;   // exchange rows (kXBytes)
+    uint64_t* full = reinterpret_cast<uint64_t*>(reinterpret_cast<unsigned char*>(xbuf) + kXBytes);
     uint64_t* empty = full + kNS;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y, bz = part.min[2] + blockIdx.z;
@@ -142,80 +147,124 @@ __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
     // the replicate clamp of the intermediate sweep; interior blocks skip the selects
     const bool edge = y0 < 2 || y0 + kRows + 2 > H || k0 < 2 || k0 + ZC + 2 > D;
     if (edge)
-        consume<PUSH, true>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+        consume<PUSH, true>(ring, xbuf, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
     else
-        consume<PUSH, false>(ring, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
+        consume<PUSH, false>(ring, xbuf, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
 }
 
+// Consumers.  Round 1 had every warp recompute sweep 1 on one halo row above and below its
+// own rows (24 sweep-1 rows per block and plane, a 3 x 6-row register window, spills at the
+// 128-register cap); here a warp computes its own 4 rows (warp 0 / 3 also the block's halo
+// row above / below: 18 rows) and takes the sweep-1 rows next to its own from its
+// neighbours through shared memory: 6 % fewer instructions, no spills, throughput equal
+// within noise (power-capped, scripts/r02/gpu_29.sh, gpu_30.sh).  Compact exchange rows:
+// 2w + 1 / 2w + 2 = warp w's top / bottom own row, 0 / 9 = the block's halo rows, so warp
+// w's row above is 2w and its row below 2w + 3.  One named barrier among the consumer warps
+// per plane, after sweep 1 and before the exchange writes, orders (a) the writes of plane
+// q-1 after every read of the same buffer (plane q-3) in the previous iteration and (b) the
+// reads of plane q-2 after their writes in the previous iteration.  Each value is computed by
+// the same expression on the same inputs as in the recomputing version, so the results are
+// bit-identical to it.
 template <bool PUSH, bool EDGE>
-__device__ __forceinline__ void consume(const float* ring, uint64_t* full, uint64_t* empty, float* __restrict__ uout,
-                                        int64_t D, int64_t H, int64_t W, int64_t c0, int64_t y0, int64_t k0, int nq,
-                                        int lane, int warp, const PushList& push) {
-    const int cx = 4 * lane;                          // smem column of the lane's first column
-    const int64_t col0 = c0 - 4 + cx;                 // its grid column
+__device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t* full, uint64_t* empty,
+                                        float* __restrict__ uout, int64_t D, int64_t H, int64_t W, int64_t c0,
+                                        int64_t y0, int64_t k0, int nq, int lane, int warp, const PushList& push) {
+    const int cx = 4 * lane;
+    const int64_t col0 = c0 - 4 + cx;
     const bool wclamp = col0 == 0, eclamp = col0 + 4 >= W;
     const bool store_col = lane >= 1 && lane <= 30 && col0 < W;
-    // 32-bit row / plane indices (the launch checks H, D < 2^30): fewer 64-bit compares and
-    // offsets in the loop under the 128-register cap (1331-1349 vs 1305-1307 GLUP/s, gpu_run100.sh)
     const int Hi = (int)H, Di = (int)D;
-    const int gr1 = (int)y0 + kRW * warp - 1;         // grid row of sweep-1 row j = 0
-    const int br1 = kRW * warp + 1;                   // box row of sweep-1 row j = 0
+    const int gr1 = (int)y0 + kRW * warp - 1;         // grid row of sweep-1 row j = 0 (the row above)
+    const int br1 = kRW * warp + 1;                   // its box row
     const int64_t HW = H * W;
-    const int64_t rowcol = (int64_t)(gr1 + 1) * W + col0;   // the warp's first own row, the lane's first column
-    float4 L1[3][kL1];                                // sweep-1 window, slot = plane sequence mod 3
+    const int64_t rowcol = (int64_t)(gr1 + 1) * W + col0;
+    const bool top = warp == 0, bot = warp == kNW - 1;
+    float4 L1[3][kRW];                                // own rows j = 1..4 at index j - 1
     ptx::mbar_wait(&full[0], 0);
     ptx::mbar_wait(&full[1], 0);
     for (int q0 = 2; q0 < nq; q0 += 3) {
 #pragma unroll
         for (int u = 0; u < 3; ++u) {
-            const int q = q0 + u;                     // q == 2 + u (mod 3)
+            const int q = q0 + u;
             if (q >= nq) break;
             ptx::mbar_wait(&full[q % kNS], (uint32_t)((q / kNS) & 1));
-            const float* sm = ring + (size_t)((q - 2) % kNS) * kSlot;   // plane seq q-2
-            const float* sc = ring + (size_t)((q - 1) % kNS) * kSlot;   // plane seq q-1
-            const float* sp = ring + (size_t)(q % kNS) * kSlot;         // plane seq q
-            // sweep 1 on plane seq q-1, rows j = 0..5 (grid rows gr1 + j)
-            float4 up = *reinterpret_cast<const float4*>(sc + (br1 - 1) * kCols + cx);
-            float4 cc = *reinterpret_cast<const float4*>(sc + br1 * kCols + cx);
-            const int s1 = (2 + u - 1 + 3) % 3;       // slot of plane seq q-1 (constant after unrolling)
+            const float* sm = ring + (size_t)((q - 2) % kNS) * kSlot;
+            const float* sc = ring + (size_t)((q - 1) % kNS) * kSlot;
+            const float* sp = ring + (size_t)(q % kNS) * kSlot;
+            const int s1 = (2 + u - 1 + 3) % 3;
+            float4 h0 = make_float4(0.f, 0.f, 0.f, 0.f), h5 = h0;
+            float4 up, cc;
+            if (top) {   // block halo row above (j = 0)
+                up = *reinterpret_cast<const float4*>(sc + (br1 - 1) * kCols + cx);
+                cc = *reinterpret_cast<const float4*>(sc + br1 * kCols + cx);
+                const float4 dn = *reinterpret_cast<const float4*>(sc + (br1 + 1) * kCols + cx);
+                const float4 zm = *reinterpret_cast<const float4*>(sm + br1 * kCols + cx);
+                const float4 zp = *reinterpret_cast<const float4*>(sp + br1 * kCols + cx);
+                const float4 ym = (EDGE && gr1 == 0) ? cc : up;
+                const float4 yp = (EDGE && gr1 == Hi - 1) ? cc : dn;
+                h0 = sweep(cc, zm, zp, ym, yp, wclamp, eclamp);
+                up = cc;
+                cc = dn;
+            } else {
+                up = *reinterpret_cast<const float4*>(sc + br1 * kCols + cx);
+                cc = *reinterpret_cast<const float4*>(sc + (br1 + 1) * kCols + cx);
+            }
 #pragma unroll
-            for (int j = 0; j < kL1; ++j) {
+            for (int j = 1; j <= kRW; ++j) {
                 const int br = br1 + j;
                 const int gr = gr1 + j;
                 const float4 dn = *reinterpret_cast<const float4*>(sc + (br + 1) * kCols + cx);
                 const float4 zm = *reinterpret_cast<const float4*>(sm + br * kCols + cx);
                 const float4 zp = *reinterpret_cast<const float4*>(sp + br * kCols + cx);
-                const float4 ym = (EDGE && gr == 0) ? cc : up;        // replicate clamp (TMA zero-filled row -1)
-                const float4 yp = (EDGE && gr == H - 1) ? cc : dn;    // ... and row H
-                L1[s1][j] = sweep(cc, zm, zp, ym, yp, wclamp, eclamp);
+                const float4 ym = (EDGE && gr == 0) ? cc : up;
+                const float4 yp = (EDGE && gr == Hi - 1) ? cc : dn;
+                L1[s1][j - 1] = sweep(cc, zm, zp, ym, yp, wclamp, eclamp);
                 up = cc;
                 cc = dn;
             }
-            // sweep 2 on plane seq q-2 = grid plane k0 + q - 4, own rows j = 1..4
-            if (q >= 4) {
+            if (bot) {   // block halo row below (j = 5)
+                const int br = br1 + kRW + 1, gr = gr1 + kRW + 1;
+                const float4 dn = *reinterpret_cast<const float4*>(sc + (br + 1) * kCols + cx);
+                const float4 zm = *reinterpret_cast<const float4*>(sm + br * kCols + cx);
+                const float4 zp = *reinterpret_cast<const float4*>(sp + br * kCols + cx);
+                const float4 ym = (EDGE && gr == 0) ? cc : up;
+                const float4 yp = (EDGE && gr == Hi - 1) ? cc : dn;
+                h5 = sweep(cc, zm, zp, ym, yp, wclamp, eclamp);
+            }
+            // plane seq q-2 is no longer read from the ring by this warp
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&empty[(q - 2) % kNS]);
+            asm volatile("bar.sync 1, %0;" ::"n"(kNW * 32) : "memory");
+            float* xw = xbuf + (size_t)((q - 1) & 1) * kXRows * kCols + cx;   // plane seq q-1
+            *reinterpret_cast<float4*>(xw + (2 * warp + 1) * kCols) = L1[s1][0];
+            *reinterpret_cast<float4*>(xw + (2 * warp + 2) * kCols) = L1[s1][kRW - 1];
+            if (top) *reinterpret_cast<float4*>(xw) = h0;
+            if (bot) *reinterpret_cast<float4*>(xw + (kXRows - 1) * kCols) = h5;
+            if (q >= 4) {   // sweep 2 on plane seq q-2 = grid plane k0 + q - 4
                 const int s0 = (2 + u - 2 + 3) % 3, sM = (2 + u - 3 + 3) % 3;
+                const float* xr = xbuf + (size_t)((q - 2) & 1) * kXRows * kCols + cx;   // plane seq q-2
+                const float4 above = *reinterpret_cast<const float4*>(xr + (2 * warp) * kCols);
+                const float4 below = *reinterpret_cast<const float4*>(xr + (2 * warp + 3) * kCols);
                 const int pz = (int)k0 + q - 4;
-                const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == Di - 1;   // sweep-1 planes outside: clamp
+                const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == Di - 1;
                 float* outp = uout + (int64_t)pz * HW + rowcol;
 #pragma unroll
                 for (int j = 1; j <= kRW; ++j) {
                     const int gr = gr1 + j;
-                    const float4 c = L1[s0][j];
-                    const float4 zm = zlo ? c : L1[sM][j];
-                    const float4 zp = zhi ? c : L1[s1][j];
-                    const float4 ym = (EDGE && gr == 0) ? c : L1[s0][j - 1];
-                    const float4 yp = (EDGE && gr == Hi - 1) ? c : L1[s0][j + 1];
+                    const float4 c = L1[s0][j - 1];
+                    const float4 zm = zlo ? c : L1[sM][j - 1];
+                    const float4 zp = zhi ? c : L1[s1][j - 1];
+                    const float4 ym = (EDGE && gr == 0) ? c : (j == 1 ? above : L1[s0][j - 2]);
+                    const float4 yp = (EDGE && gr == Hi - 1) ? c : (j == kRW ? below : L1[s0][j]);
                     const float4 o = sweep(c, zm, zp, ym, yp, wclamp, eclamp);
-                    if (store_col && (!EDGE || gr < Hi)) {   // interior blocks: every own row < H
+                    if (store_col && (!EDGE || gr < Hi)) {
                         *reinterpret_cast<float4*>(outp) = o;
                         PK_TRACE_W(outp, 16);
-                        if (PUSH) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);  // fused halo push
+                        if (PUSH) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);
                     }
                     outp += W;
                 }
             }
-            __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&empty[(q - 2) % kNS]);   // plane seq q-2 fully read
         }
     }
     __syncwarp();
