@@ -75,6 +75,9 @@ __device__ __forceinline__ float upd(float c, float zm, float zp, float ym, floa
 
 __device__ __forceinline__ float4 sweep(const float4& c, const float4& zm, const float4& zp, const float4& ym,
                                         const float4& yp, bool wclamp, bool eclamp) {
+#ifdef PK_HEATTB_DIAG   // diagnostic only (power / rate of the data stream without the arithmetic)
+    return c;
+#endif
     float wv = __shfl_up_sync(0xffffffffu, c.w, 1);
     float ev = __shfl_down_sync(0xffffffffu, c.x, 1);
     if (wclamp) wv = c.x;

@@ -4,6 +4,7 @@ the box: torch TF32 matmul (allow_tf32), P2P copy bandwidth and latency, NCCL al
 busbw").  Prints one JSON object.
 
     python scripts/probe_peaks.py                 # TF32 matmul, D2D copy, P2P matrix (>= 2 GPUs)
+    python scripts/probe_peaks.py --sustained 4   # D2D copy back to back for 4 s (power-limited)
     torchrun --nproc-per-node N scripts/probe_peaks.py --nccl   # NCCL all-gather busbw (N >= 2)
 
 Every number is CUDA-event timed on the device after warm-up; nothing here is used by the
@@ -43,6 +44,18 @@ def d2d_copy(nbytes):
     return {"bytes": nbytes, "ms": ms, "gbs_read_plus_write": 2 * nbytes / ms / 1e6}
 
 
+def d2d_copy_sustained(nbytes, seconds):
+    """Back-to-back copies for `seconds` (long enough for the board power limiter to act):
+    the sustained HBM figure next to the best-of-20 burst one."""
+    a = torch.empty(nbytes // 4, device="cuda")
+    b = torch.empty_like(a)
+    one = ev_time(lambda: b.copy_(a), 5)
+    reps = max(1, int(seconds * 1e3 / one))
+    ms = ev_time(lambda: b.copy_(a), reps)
+    return {"bytes": nbytes, "reps": reps, "seconds": reps * ms / 1e3, "ms": ms,
+            "gbs_read_plus_write": 2 * nbytes / ms / 1e6}
+
+
 def p2p(src, dst, nbytes):
     a = torch.empty(nbytes // 4, device=f"cuda:{src}")
     b = torch.empty(nbytes // 4, device=f"cuda:{dst}")
@@ -54,6 +67,8 @@ def p2p(src, dst, nbytes):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--nccl", action="store_true")
+    ap.add_argument("--sustained", type=float, default=0.0,
+                    help="only the sustained D2D copy over this many seconds")
     args = ap.parse_args()
     out = {}
     if args.nccl:
@@ -75,6 +90,10 @@ def main():
         if r == 0:
             print(json.dumps({"nccl_allgather": res, "world": w}))
         dist.destroy_process_group()
+        return
+    if args.sustained:
+        print(json.dumps({"d2d_copy_sustained": d2d_copy_sustained(1 << 30, args.sustained),
+                          "d2d_copy_burst": d2d_copy(1 << 30)}))
         return
     n_dev = torch.cuda.device_count()
     out["device"] = torch.cuda.get_device_name(0)
