@@ -358,13 +358,8 @@ class Workload:
         elif self.name == "heat3d":
             out = K.heat3d_iterate(pr, self.iters, self.t)
         elif self.name == "jacobi2d":
-            h, w = self.shape
-            grid, blk, sc = K.jacobi2d_launch(h, w)
-            b0, b1 = pr.bufs
-            for t in range(self.t, self.t + self.iters):
-                a, b = (b0, b1) if t % 2 == 0 else (b1, b0)
-                pr.launch(grid, blk, [a, b, h, w], sc)
-            out = b1 if (self.t + self.iters) % 2 == 1 else b0
+            # the step's sweeps as one pk_launch_sequence: one graph launch in steady state
+            out = K.jacobi2d_iterate(pr, self.iters, self.t, sequence=True)
         elif self.name == "sgemm":
             for _ in range(self.iters):
                 out = self.step_once()

@@ -274,6 +274,30 @@ const void* pk_builtin_fn(const char* name);
 int pk_launch_partitioned(pk_ctx ctx, pk_kernel k, const int32_t grid[3],
                           const int32_t block[3], size_t smem_bytes,
                           const void* const* args, const int64_t* scalars, int nscalars);
+/* A sequence of partitioned launches (an inner loop of a host program: the C1
+ * Jacobi sweeps, the Hotspot time steps), issued as ONE unit.  The result is
+ * exactly that of n pk_launch_partitioned calls in order -- every launch still
+ * partitions, resolves its stale ranges and updates the trackers (Fig. 4,
+ * P:L616-666) -- but in steady state the whole sequence is memoised as one
+ * multi-stream CUDA graph: the first call with a given (launch list, pre-launch
+ * tracker state) runs eagerly, the second is captured, later ones replay it with
+ * a single graph launch and restore the recorded tracker states.  For launch-bound
+ * loops (microsecond kernels) this removes the per-launch host and launch
+ * latency; it does not change what moves.  Each descriptor is one
+ * pk_launch_partitioned argument list (args / scalars are read during the call).
+ * n <= PK_MAX_SEQUENCE.  Errors: those of pk_launch_partitioned; launches before a
+ * failing one stay issued. */
+#define PK_MAX_SEQUENCE 1024
+typedef struct pk_launch_desc {
+    pk_kernel kernel;
+    int32_t grid[3];
+    int32_t block[3];
+    size_t smem_bytes;
+    const void* const* args;
+    const int64_t* scalars;
+    int nscalars;
+} pk_launch_desc;
+int pk_launch_sequence(pk_ctx ctx, const pk_launch_desc* launches, int n);
 /* The ORIGINAL single-GPU launch, for the paper's E3 measurement (§9.2:
  * "slowdown of the partitioned binary on a single GPU"): the kernel's full grid is
  * launched once on partition 0's stream with partition 0's instances -- no partition
@@ -347,7 +371,8 @@ typedef struct {
     double kernel_ms;            /* sum over partition kernels (PK_MODE_TIME_KERNELS) */
     double kernel_ms_max_launch; /* per launch: max over partitions, summed */
     uint64_t timed_kernels;      /* kernels included in kernel_ms */
-    uint64_t graph_replays;      /* launches served by steady-state graph replay */
+    uint64_t graph_replays;      /* launches served by steady-state graph replay (a replayed sequence counts
+                                    each of its launches) */
     uint64_t graph_captures;     /* launches captured into a replay graph */
     uint64_t strided_copies;     /* of `copies`: equal pieces at a constant pitch (2-D / 3-D) */
     uint64_t copy_kernels;       /* of `strided_copies`: narrow runs moved by the SM halo-copy kernel */
@@ -356,9 +381,9 @@ typedef struct {
     uint64_t graph_fallbacks;    /* a graph capture / instantiation failed: the launch ran eagerly and the
                                     context stays eager (pk_last_error() keeps the reason) */
     double graph_launch_ms;      /* PK_MODE_TIME_KERNELS with graph replay: CUDA events around each replayed
-                                    launch on its stream (copies + partition kernels of that launch) */
-    uint64_t timed_graph_launches;
-    uint64_t host_cpu_ns;        /* thread CPU time spent inside pk_launch_partitioned (excludes time the
+                                    graph on its stream (copies + partition kernels of its launches) */
+    uint64_t timed_graph_launches; /* partitioned launches inside those graphs */
+    uint64_t host_cpu_ns;        /* thread CPU time spent inside pk_launch_partitioned / _sequence (excludes time the
                                     thread is descheduled; a driver spinning on a full launch queue still counts) */
     uint64_t streamed_bytes;     /* of moved_bytes: copied on a side stream while the consuming kernel ran */
     uint64_t timed_eager_launches; /* launches whose partition kernels were timed (kernel_ms_max_launch) */

@@ -133,6 +133,7 @@ def lib():
                                   C.POINTER(C.c_void_p), _I64P, C.c_int],
         "pk_launch_direct": [C.c_void_p, C.c_int64, _I32P, _I32P, C.c_size_t,
                              C.POINTER(C.c_void_p), _I64P, C.c_int],
+        "pk_launch_sequence": [C.c_void_p, C.c_void_p, C.c_int],
         "pk_synchronize": [C.c_void_p],
         "pk_timer_begin": [C.c_void_p],
         "pk_timer_end": [C.c_void_p, C.POINTER(C.c_double)],
@@ -356,6 +357,39 @@ def pk_launch_partitioned(ctx, kernel, grid, block, args, scalars=(), smem=0):
     (int64) value for a scalar; None passes a NULL pointer."""
     m = _launch_args(kernel, grid, block, args, scalars)
     _check(lib().pk_launch_partitioned(ctx, kernel, m[0], m[1], smem, m[2], m[3], m[4]), "pk_launch_partitioned")
+
+
+class pk_launch_desc(C.Structure):
+    _fields_ = [("kernel", C.c_int64), ("grid", C.c_int32 * 3), ("block", C.c_int32 * 3), ("smem_bytes", C.c_size_t),
+                ("args", C.POINTER(C.c_void_p)), ("scalars", _I64P), ("nscalars", C.c_int)]
+
+
+_SEQUENCES = {}
+
+
+def pk_launch_sequence(ctx, launches):
+    """launches: [(kernel, grid, block, args, scalars), ...] -- one pk_launch_partitioned
+    argument list each (args as there), issued as one unit (memoised as one graph)."""
+    key = tuple((k, tuple(g), tuple(b), tuple(a), tuple(sc)) for k, g, b, a, sc in launches)
+    m = _SEQUENCES.get(key)
+    if m is None:
+        descs = (pk_launch_desc * max(1, len(key)))()
+        keep = []
+        for i, (k, g, b, a, sc) in enumerate(key):
+            la = _launch_args(k, g, b, a, sc)
+            keep.append(la)
+            d = descs[i]
+            d.kernel, d.smem_bytes = k, 0
+            d.grid[:] = list(g)
+            d.block[:] = list(b)
+            d.args = la[2]
+            d.scalars = la[3]
+            d.nscalars = la[4]
+        m = (descs, len(key), keep)
+        if len(_SEQUENCES) > 64:
+            _SEQUENCES.clear()
+        _SEQUENCES[key] = m
+    _check(lib().pk_launch_sequence(ctx, C.cast(m[0], C.c_void_p), m[1]), "pk_launch_sequence")
 
 
 def pk_launch_direct(ctx, kernel, grid, block, args, scalars=(), smem=0):

@@ -14,6 +14,8 @@
 // input byte is fetched from HBM about once.  Formulas: DESIGN.md §3 (Q14, Q15).
 #include <cuda_runtime.h>
 
+#include <cstdlib>
+
 #include "../runtime/builtins.h"
 #include "common.cuh"
 
@@ -31,6 +33,11 @@ using dev::st4;
 template <bool PUSH>
 __global__ void __launch_bounds__(256) k_jacobi2d(const float* __restrict__ in, float* __restrict__ out,
                                                   int64_t H, int64_t W, pk_partition part, PushList push) {
+    // programmatic dependent launch (launch_jacobi2d): let the next sweep's grid be scheduled
+    // now, and wait here until the previous sweep's grid has completed and its stores are
+    // visible -- before any load or store, so ping-pong RAW and WAR both stay ordered
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     const int64_t bx = part.min[0] + blockIdx.x, by = part.min[1] + blockIdx.y;  // Eq. 8
     const int64_t i = by * blockDim.y + threadIdx.y, j = bx * blockDim.x + threadIdx.x;
     if (i < 1 || i > H - 2 || j < 1 || j > W - 2) return;
@@ -68,7 +75,21 @@ cudaError_t launch_jacobi2d(const LaunchInfo& li) {
     if (li.push) pl = *li.push;
     void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &H, &W, (void*)&li.part, &pl};
     const void* fn = (li.push && li.push->n > 0) ? (const void*)k_jacobi2d<true> : (const void*)k_jacobi2d<false>;
-    return cudaLaunchKernel(fn, li.grid, li.block, argv, 0, li.stream);
+    // C1 sweeps are microsecond kernels: with programmatic stream serialisation the next
+    // sweep's launch overlaps this one (only a kernel directly after a kernel in the same
+    // stream is affected; copies and event waits keep their full dependencies)
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = li.grid;
+    cfg.blockDim = li.block;
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = li.stream;
+    cfg.attrs = at;
+    static const bool no_pdl = getenv("PK_NO_PDL") != nullptr;   // A/B switch (scripts/r02/gpu_39.sh)
+    cfg.numAttrs = no_pdl ? 0 : 1;
+    return cudaLaunchKernelExC(&cfg, fn, argv);
 }
 
 // ============================================================ C2 hotspot2d

@@ -247,6 +247,7 @@ struct TimedLaunch {
     int part;
     uint64_t launch_id;
     bool graph = false;  // events around a replayed graph launch (whole launch), not one kernel
+    int nlaunch = 1;     // partitioned launches inside that graph (pk_launch_sequence)
 };
 
 }  // namespace
@@ -902,7 +903,7 @@ static int drain_timing(pk_ctx c) {
         PK_CUDA(cudaEventElapsedTime(&ms, t.start, t.stop));
         if (t.graph) {
             c->stats.graph_launch_ms += ms;
-            c->stats.timed_graph_launches += 1;
+            c->stats.timed_graph_launches += t.nlaunch;
         } else {
             c->stats.kernel_ms += ms;
             c->stats.timed_kernels += 1;
@@ -1558,47 +1559,76 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
         for (int j = 0; j < 16; ++j) a.pair_bytes[i][j] += sign * d.pair_bytes[i][j];
 }
 
-int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
-                          const void* const* args, const int64_t* scalars, int ns) {
-    if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
-    struct CpuTime {  // thread CPU time of this call -> pk_stats.host_cpu_ns
-        pk_ctx c;
-        uint64_t t0 = thread_cpu_ns();
-        ~CpuTime() { c->stats.host_cpu_ns += thread_cpu_ns() - t0; }
-    } cpu_time{c};
-    if (ns < 0 || ns > PK_MAX_SCALARS || (ns && !scalars)) return fail(PK_ERR_INVALID, "bad scalars");
-    const Kernel& K = c->kernels[k];
+// One partitioned launch as the memoised launch path sees it.
+struct LaunchReq {
+    pk_kernel k;
+    const int32_t* grid;
+    const int32_t* block;
+    size_t smem;
+    const void* const* args;
+    const int64_t* scalars;
+    int ns;
+};
+
+static int check_launch(pk_ctx c, const LaunchReq& d) {
+    if (!valid_kernel(c, d.k) || !d.grid || !d.block) return fail(PK_ERR_INVALID, "bad argument");
+    if (d.ns < 0 || d.ns > PK_MAX_SCALARS || (d.ns && !d.scalars)) return fail(PK_ERR_INVALID, "bad scalars");
+    return PK_OK;
+}
+
+// n partitioned launches in order, memoised as ONE graph: the key is every launch's
+// identity plus the pre-launch tracker state of every buffer bound by any of them; the
+// first sighting runs eagerly, the second is captured (transfers, kernels and event edges
+// of all n launches), later sightings with the same pre-state replay it and restore the
+// recorded post-states.  n = 1 is pk_launch_partitioned.
+static int launch_memo(pk_ctx c, const LaunchReq* d, int n) {
     const uint32_t mode = c->mode;
+    auto eager_all = [&]() -> int {
+        for (int i = 0; i < n; ++i)
+            if (int r = launch_eager(c, d[i].k, d[i].grid, d[i].block, d[i].smem, d[i].args, d[i].scalars, d[i].ns))
+                return r;
+        return PK_OK;
+    };
     // builtin launchers take every scalar from `scalars`, so the key below captures the launch
-    const bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && K.nargs && args && K.launcher &&
-                           !c->graphs_broken && !(mode & (PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
+    bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && !c->graphs_broken &&
+                     !(mode & (PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
+    for (int i = 0; i < n && can_graph; ++i) {
+        const Kernel& K = c->kernels[d[i].k];
+        can_graph = K.nargs && d[i].args && K.launcher;
+    }
     if (!can_graph) {
         if (!c->host_only)
             if (int r = exit_graph_mode(c)) return r;
-        return launch_eager(c, k, grid, block, smem, args, scalars, ns);
+        return eager_all();
     }
-    // ---- memo key: launch identity + pre-launch tracker state of every bound buffer ----
+    // ---- memo key: launch identities + pre-launch tracker state of every bound buffer ----
     uint64_t t0 = now_ns();
     std::string key;
-    key.reserve(256);
-    auto put = [&key](const void* p, size_t n) { key.append((const char*)p, n); };
-    put(&k, sizeof k);
-    put(&K.version, sizeof K.version);
-    put(grid, 12);
-    put(block, 12);
-    put(&smem, sizeof smem);
+    key.reserve(256 * n);
+    auto put = [&key](const void* p, size_t sz) { key.append((const char*)p, sz); };
+    put(&n, sizeof n);
     const uint32_t kmode = mode & ~(uint32_t)PK_MODE_TIME_KERNELS;  // timing events sit outside the graph
     put(&kmode, sizeof kmode);
-    put(&ns, sizeof ns);
-    if (ns) put(scalars, sizeof(int64_t) * ns);
     std::vector<int64_t> bids;
-    for (int a = 0; a < K.nargs; ++a) {
-        if (K.kinds[a] == PK_ARG_BUFFER) {
-            if (!args[a]) return fail(PK_ERR_INVALID, "null buffer argument");
-            const pk_buf b = *(const pk_buf*)args[a];
-            if (!valid_buf(c, b)) return fail(PK_ERR_INVALID, "argument " + std::to_string(a) + " is not a live buffer");
-            put(&b, sizeof b);
-            if (std::find(bids.begin(), bids.end(), b) == bids.end()) bids.push_back(b);
+    for (int i = 0; i < n; ++i) {
+        const LaunchReq& q = d[i];
+        const Kernel& K = c->kernels[q.k];
+        put(&q.k, sizeof q.k);
+        put(&K.version, sizeof K.version);
+        put(q.grid, 12);
+        put(q.block, 12);
+        put(&q.smem, sizeof q.smem);
+        put(&q.ns, sizeof q.ns);
+        if (q.ns) put(q.scalars, sizeof(int64_t) * q.ns);
+        for (int a = 0; a < K.nargs; ++a) {
+            if (K.kinds[a] == PK_ARG_BUFFER) {
+                if (!q.args[a]) return fail(PK_ERR_INVALID, "null buffer argument");
+                const pk_buf b = *(const pk_buf*)q.args[a];
+                if (!valid_buf(c, b))
+                    return fail(PK_ERR_INVALID, "argument " + std::to_string(a) + " is not a live buffer");
+                put(&b, sizeof b);
+                if (std::find(bids.begin(), bids.end(), b) == bids.end()) bids.push_back(b);
+            }
         }
     }
     for (int64_t b : bids) {
@@ -1635,7 +1665,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
         const int p0 = c->first_local;
         if (int r = c->set_device(c->dev[p0])) return r;
         cudaEvent_t e0 = nullptr, e1 = nullptr;
-        if (mode & PK_MODE_TIME_KERNELS) {  // the whole replayed launch, on the stream it runs on
+        if (mode & PK_MODE_TIME_KERNELS) {  // the whole replayed graph, on the stream it runs on
             auto& pool = c->event_pool[p0];
             for (cudaEvent_t* e : {&e0, &e1}) {
                 if (!pool.empty()) { *e = pool.back(); pool.pop_back(); }
@@ -1648,13 +1678,14 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
             PK_CUDA(cudaEventRecord(e1, c->stream[p0]));
             TimedLaunch tl{e0, e1, p0, c->launch_counter};
             tl.graph = true;
+            tl.nlaunch = n;
             c->pending_timing.push_back(tl);
         }
         for (auto& ps : m.post) c->bufs[ps.buf].tracker.set_state(ps.state, ps.fp);
         c->replay_plan = m.plan;
         add_stats(c->stats, m.delta, 1);
-        c->stats.graph_replays += 1;
-        c->launch_counter++;
+        c->stats.graph_replays += n;
+        c->launch_counter += n;
         c->stats.host_ns_issue += now_ns() - t0;
         return PK_OK;
     }
@@ -1663,10 +1694,10 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
     int rc;
     if (!capture) {
         if (int r = exit_graph_mode(c)) return r;
-        rc = launch_eager(c, k, grid, block, smem, args, scalars, ns);
+        rc = eager_all();
         if (rc) return rc;
     } else {
-        // ---- capture the launch once into a multi-stream graph ----
+        // ---- capture the launches once into a multi-stream graph ----
         // host state the eager path mutates, restored if capture or instantiation fails
         std::vector<std::vector<RangeList>> saved_last_read;
         std::vector<std::vector<uint64_t>> saved_pushers;
@@ -1674,6 +1705,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
             saved_last_read.push_back(c->bufs[b].last_read);
             saved_pushers.push_back(c->bufs[b].pushers);
         }
+        const uint64_t saved_counter = c->launch_counter;
         auto fall_back = [&](const std::string& why) -> int {
             // a failed capture enqueued nothing: undo the bookkeeping and run eagerly, and
             // keep this context on the eager path (no silent retry of a failing capture)
@@ -1684,13 +1716,14 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
                 B.pushers = saved_pushers[i];
             }
             c->stats = before;
+            c->launch_counter = saved_counter;
             c->graphs_broken = true;
             c->stats.graph_fallbacks += 1;
             g_err = why;
             clear_memo(c);
             c->graph_mode = false;  // capture ended; stream[p0] already follows every stream's tail
             if (int r = exit_graph_mode(c)) return r;
-            return launch_eager(c, k, grid, block, smem, args, scalars, ns);
+            return eager_all();
         };
         if (int r = enter_graph_mode(c)) return r;
         const int p0 = c->first_local;
@@ -1703,8 +1736,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
                 ce = cudaStreamWaitEvent(c->stream[p], c->ev_fork, 0);
             }
         c->capturing = true;
-        rc = ce == cudaSuccess ? launch_eager(c, k, grid, block, smem, args, scalars, ns)
-                               : fail(PK_ERR_CUDA, std::string("graph fork: ") + cudaGetErrorName(ce));
+        rc = ce == cudaSuccess ? eager_all() : fail(PK_ERR_CUDA, std::string("graph fork: ") + cudaGetErrorName(ce));
         c->capturing = false;
         if (rc == PK_OK && getenv("PK_DEBUG_FAIL_CAPTURE"))  // test hook: exercise the eager fallback
             rc = fail(PK_ERR_CUDA, "PK_DEBUG_FAIL_CAPTURE");
@@ -1744,7 +1776,7 @@ int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const in
             PK_CUDA(cudaGraphLaunch(ex, c->stream[p0]));
             if (c->memo.size() > 256) clear_memo(c);
             c->memo[key].exec = ex;
-            c->stats.graph_captures += 1;
+            c->stats.graph_captures += n;
         }
     }
 record:
@@ -1762,6 +1794,34 @@ record:
         m.post.push_back({b, T.state(), T.fingerprint()});
     }
     return PK_OK;
+}
+
+struct CpuTime {  // thread CPU time of a launch call -> pk_stats.host_cpu_ns
+    pk_ctx c;
+    uint64_t t0 = thread_cpu_ns();
+    ~CpuTime() { c->stats.host_cpu_ns += thread_cpu_ns() - t0; }
+};
+
+int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
+                          const void* const* args, const int64_t* scalars, int ns) {
+    const LaunchReq d{k, grid, block, smem, args, scalars, ns};
+    if (int r = check_launch(c, d)) return r;
+    CpuTime cpu_time{c};
+    return launch_memo(c, &d, 1);
+}
+
+int pk_launch_sequence(pk_ctx c, const pk_launch_desc* launches, int n) {
+    if (!c || n < 0 || (n && !launches)) return fail(PK_ERR_INVALID, "bad argument");
+    if (n > PK_MAX_SEQUENCE) return fail(PK_ERR_INVALID, "more than PK_MAX_SEQUENCE launches");
+    if (n == 0) return PK_OK;
+    std::vector<LaunchReq> d(n);
+    for (int i = 0; i < n; ++i) {
+        const pk_launch_desc& l = launches[i];
+        d[i] = LaunchReq{l.kernel, l.grid, l.block, l.smem_bytes, l.args, l.scalars, l.nscalars};
+        if (int r = check_launch(c, d[i])) return r;
+    }
+    CpuTime cpu_time{c};
+    return launch_memo(c, d.data(), n);
 }
 
 // Streamed operand (Builtin::stream_arg): the stale ranges of buffer `b` bound for partition

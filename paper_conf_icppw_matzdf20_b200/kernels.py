@@ -136,19 +136,44 @@ class Problem:
         else:
             abi.pk_launch_partitioned(self.ctx, self.k, grid, block, args, scalars)
 
+    def launch_seq(self, launches):
+        """[(grid, block, args, scalars), ...] in order, as one pk_launch_sequence (one graph
+        launch in steady state); one by one on the direct (E3 baseline) path."""
+        if self.direct:
+            for g, b, a, sc in launches:
+                abi.pk_launch_direct(self.ctx, self.k, g, b, a, sc)
+        else:
+            abi.pk_launch_sequence(self.ctx, [(self.k, g, b, a, sc) for g, b, a, sc in launches])
 
-def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None):
+
+def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None, sequence=False):
     """C1: both buffers carry the Dirichlet boundary (uploaded); returns the buffer id
-    that holds the result after `iters` sweeps."""
+    that holds the result after `iters` sweeps (sequence=True: the sweeps go out as one
+    pk_launch_sequence)."""
     h, w = u_host.shape
     pr = Problem(ctx, "jacobi2d", tiles)
-    u0 = pr.buffer((h, w), 4, host=u_host)
-    u1 = pr.buffer((h, w), 4, host=u_host)
-    grid, blk, sc = jacobi2d_launch(h, w, block)
-    for t in range(iters):
+    pr.buffer((h, w), 4, host=u_host)
+    pr.buffer((h, w), 4, host=u_host)
+    pr.geom = jacobi2d_launch(h, w, block)
+    return pr, jacobi2d_iterate(pr, iters, 0, sequence)
+
+
+def jacobi2d_iterate(pr, iters, start=0, sequence=True):
+    """`iters` C1 sweeps from sweep `start` on a jacobi2d_program problem (ping-pong
+    u0 -> u1 -> u0 ...), as one pk_launch_sequence or one launch call per sweep; returns
+    the buffer id of the result."""
+    u0, u1 = pr.bufs[:2]
+    grid, blk, sc = pr.geom
+    launches = []
+    for t in range(start, start + iters):
         a, b = (u0, u1) if t % 2 == 0 else (u1, u0)
-        pr.launch(grid, blk, [a, b, h, w], sc)
-    return pr, (u0 if iters % 2 == 0 else u1)
+        launches.append((grid, blk, [a, b, sc[0], sc[1]], sc))
+    if sequence and launches:
+        pr.launch_seq(launches)
+    else:
+        for g, b, a, s in launches:
+            pr.launch(g, b, a, s)
+    return u1 if (start + iters) % 2 == 1 else u0
 
 
 def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, dev_ptrs=None,

@@ -42,6 +42,30 @@ def test_c1_jacobi_512_p2_oracle_stale_and_bitwise():
     assert s2["kernel_launches"] == 20 and s2["pair_bytes"][0][1] == s2["pair_bytes"][1][0] == 20400
 
 
+@pytest.mark.parametrize("P", [1, 2, 3])
+def test_launch_sequence_graph_replay_equals_single_launches(P):
+    """pk_launch_sequence (the bench's C1 step): 6 sequences of 10 sweeps are captured and
+    then replayed as one graph each, and give bit-for-bit the result of the 60 launches one
+    by one (and the 1-way result), within 1e-5 of the fp64 oracle, with the same stale bytes."""
+    u = synth.jacobi_grid(512, 512)
+    ref, s_single = _jacobi(u, 60, P)
+    one, _ = _jacobi(u, 60, 1)
+    ctx = gpu_ctx(P)
+    pr, out = K.jacobi2d_program(ctx, u, 0)
+    for step in range(6):
+        out = K.jacobi2d_iterate(pr, 10, 10 * step, sequence=True)
+    res = fetch(ctx, out, u.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    assert np.array_equal(res, ref) and np.array_equal(res, one)
+    ok_, err = rel_ok(res, ok.jacobi2d(u, 60), 1e-5)
+    assert ok_, err
+    assert st["launches"] == 60 and st["kernel_launches"] == 60 * P
+    assert st["stale_bytes"] == s_single["stale_bytes"] and st["moved_bytes"] == s_single["moved_bytes"]
+    assert st["graph_fallbacks"] == 0
+    assert st["graph_captures"] >= 10 and st["graph_replays"] >= 10   # captured, then replayed whole
+
+
 @pytest.mark.parametrize("single", [False, True])
 def test_paper_vs_validity_tracker_measured_on_gpu(single):
     """SURVEY NEXT-1 / §8(c) paper-vs-validity pins, measured through the library on the GPU

@@ -281,6 +281,57 @@ def test_c1_sequence_40800_bytes():
     assert st_["launches"] == 10 and st_["kernel_launches"] == 20
 
 
+@pytest.mark.parametrize("P,chunks", [(2, [10]), (3, [3, 3]), (3, [1, 5]), (4, [2, 4])])
+@pytest.mark.parametrize("mode", [0, abi.PK_MODE_SINGLE_OWNER])
+def test_launch_sequence_equals_single_launches(P, chunks, mode):
+    """pk_launch_sequence = the same launches one by one (pk_api.h): after every chunk the
+    trackers equal the shadow oracle's after that many launches, and the stale bytes and
+    launch counts add up (Jacobi 64², misaligned linear upload at P = 3)."""
+    n = 64
+    geom = K.jacobi2d_launch(n, n)
+    iters = sum(chunks)
+    sh = shadow.Shadow(P, single_owner=bool(mode & abi.PK_MODE_SINGLE_OWNER))
+    for name in ("u0", "u1"):
+        sh.register(name, n * n, 4, True)
+    rle_after, stale_after = [], []
+    for t in range(iters):
+        a, b = ("u0", "u1") if t % 2 == 0 else ("u1", "u0")
+        per = []
+        for p in range(P):
+            acc = regions.jacobi2d(og.partition_box(geom[0], P, p), geom[1], n, n)
+            d = {}
+            for (arg, tag), el in acc.items():
+                name = (a, b)[arg]
+                r, w = d.get(name, (np.zeros(0, np.int64), np.zeros(0, np.int64)))
+                d[name] = (np.union1d(r, el), w) if tag == "r" else (r, np.union1d(w, el))
+            per.append(d)
+        res = sh.launch(per)
+        stale_after.append((stale_after[-1] if stale_after else 0) + sum(res["stale"]))
+        rle_after.append({nm: sh.buffers[nm].rle() for nm in ("u0", "u1")})
+    ctx = host_ctx(P, mode)
+    k = abi.pk_builtin_kernel(ctx, "jacobi2d")
+    ids = {nm: abi.pk_register_buffer(ctx, (n, n), 4, host_init=np.zeros(n * n, np.float32)) for nm in ("u0", "u1")}
+    t = 0
+    for c in chunks:
+        seq = []
+        for i in range(t, t + c):
+            a, b = (ids["u0"], ids["u1"]) if i % 2 == 0 else (ids["u1"], ids["u0"])
+            seq.append((k, geom[0], geom[1], [a, b, n, n], geom[2]))
+        abi.pk_launch_sequence(ctx, seq)
+        t += c
+        st_ = abi.pk_get_stats(ctx)
+        assert st_["launches"] == t and st_["kernel_launches"] == t * P
+        assert st_["stale_bytes"] == stale_after[t - 1]
+        for nm, bid in ids.items():
+            assert abi.pk_tracker_dump(ctx, bid) == rle_after[t - 1][nm]
+    abi.pk_launch_sequence(ctx, [])                              # empty: nothing happens
+    assert abi.pk_get_stats(ctx)["launches"] == iters
+    with pytest.raises(abi.PkError) as ei:                       # a bad descriptor: PK_ERR_INVALID
+        abi.pk_launch_sequence(ctx, [(k + 99, geom[0], geom[1], [ids["u0"], ids["u1"], n, n], geom[2])])
+    assert ei.value.name == "PK_ERR_INVALID"
+    abi.pk_finalize(ctx)
+
+
 @pytest.mark.parametrize("mode", [0, abi.PK_MODE_SINGLE_OWNER])
 def test_c1_misaligned_p3_both_tracker_modes(mode):
     _jacobi_case(64, 3, 6, mode)
