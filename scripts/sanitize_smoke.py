@@ -18,6 +18,9 @@ def main():
     ctx = abi.pk_init(P, part_device=[0] * P)
     u = synth.jacobi_grid(70, 90)
     _, jb = K.jacobi2d_program(ctx, u, 3)
+    pj, _ = K.jacobi2d_program(ctx, u, 0)               # launch sequences (graph capture + replay, PDL)
+    for s in range(4):
+        K.jacobi2d_iterate(pj, 4, 4 * s, sequence=True)
     t, p = synth.hotspot_grids(150, 1100)
     pr = K.hotspot2d_setup(ctx, t, p, ty=16)
     hb = K.hotspot2d_iterate(pr, 3)
