@@ -46,6 +46,16 @@ def _sequence(abi, K, ctx, kernel, world):
             K.nbody_iterate(pr, 1, start=s)
             out.append((abi.pk_last_plan(ctx), abi.pk_get_stats(ctx)["stale_bytes"],
                         [abi.pk_tracker_dump(ctx, b) for b in pr.nb]))
+    elif kernel == "jacobi2d_seq":
+        # the same 5 Jacobi launches as below, issued as pk_launch_sequence chunks of 2 + 3
+        n = 64
+        pr, _ = K.jacobi2d_program(ctx, np.zeros((n, n), np.float32), 0)
+        t = 0
+        for c in (2, 3):
+            K.jacobi2d_iterate(pr, c, t, sequence=True)
+            t += c
+            out.append((abi.pk_last_plan(ctx), abi.pk_get_stats(ctx)["stale_bytes"],
+                        [abi.pk_tracker_dump(ctx, x) for x in pr.bufs]))
     else:
         n = 64
         pr = K.Problem(ctx, "jacobi2d")
@@ -122,6 +132,29 @@ def test_spmd_two_ranks_replicated_plan_and_matched_transfers(kernel, transport,
                 assert sends == recvs
                 moved += sum(hi - lo for (_, lo, hi) in sends)
     assert moved == seq0[-1][1] > 0          # all stale bytes cross ranks (one partition per rank)
+
+
+@pytest.mark.parametrize("transport", ["nccl", "ipc"])
+def test_spmd_launch_sequence_replicated(transport, tmp_path):
+    """pk_launch_sequence in SPMD contexts (issued launch by launch there): replicated state
+    identical on both ranks, equal to the single-process sequence, and after the 5 launches
+    equal to the same launches issued one by one."""
+    world = 2
+    mp.spawn(_worker, args=(world, _free_port(), "jacobi2d_seq", str(tmp_path), transport), nprocs=world, join=True)
+    import pickle
+    (seq0, l0, _), (seq1, l1, _) = pickle.load(open(tmp_path / "res.pkl", "rb"))
+    assert seq0 == seq1 and l0 == l1 == 5
+    from paper_conf_icppw_matzdf20_b200 import abi
+    from paper_conf_icppw_matzdf20_b200 import kernels as K
+    ref_ctx = abi.pk_init(world, flags=abi.PK_INIT_HOST_ONLY)
+    ref = _sequence(abi, K, ref_ctx, "jacobi2d_seq", world)
+    abi.pk_finalize(ref_ctx)
+    assert seq0 == ref
+    one_ctx = abi.pk_init(world, flags=abi.PK_INIT_HOST_ONLY)
+    single = _sequence(abi, K, one_ctx, "jacobi2d", world)
+    abi.pk_finalize(one_ctx)
+    assert seq0[-1][1:] == single[-1][1:]           # same stale bytes and trackers after 5 launches
+    assert seq0[0][1:] == single[1][1:]             # ... and after the first chunk of 2
 
 
 def _mismatch_worker(rank, world, port, qdir):
