@@ -352,7 +352,8 @@ typedef void (*pk_segment_cb)(void* user, uint64_t begin_byte, uint64_t end_byte
 int pk_tracker_dump(pk_ctx ctx, pk_buf buf, pk_segment_cb cb, void* user);
 typedef void (*pk_copy_cb)(void* user, pk_buf buf, int src_part, int dst_part,
                            uint64_t begin_byte, uint64_t end_byte);
-/* Copies planned by the most recent pk_launch_partitioned (coalesced, in issue order). */
+/* Copies planned by the most recent pk_launch_partitioned (coalesced, in issue order; after a
+ * pk_launch_sequence: those of its last launch). */
 int pk_last_plan(pk_ctx ctx, pk_copy_cb cb, void* user);
 
 typedef struct {

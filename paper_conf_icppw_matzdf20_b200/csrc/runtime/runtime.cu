@@ -1559,6 +1559,7 @@ static void add_stats(pk_stats& a, const pk_stats& d, int sign) {
         for (int j = 0; j < 16; ++j) a.pair_bytes[i][j] += sign * d.pair_bytes[i][j];
 }
 
+namespace {
 // One partitioned launch as the memoised launch path sees it.
 struct LaunchReq {
     pk_kernel k;
@@ -1569,6 +1570,7 @@ struct LaunchReq {
     const int64_t* scalars;
     int ns;
 };
+}  // namespace
 
 static int check_launch(pk_ctx c, const LaunchReq& d) {
     if (!valid_kernel(c, d.k) || !d.grid || !d.block) return fail(PK_ERR_INVALID, "bad argument");
@@ -1796,11 +1798,13 @@ record:
     return PK_OK;
 }
 
+namespace {
 struct CpuTime {  // thread CPU time of a launch call -> pk_stats.host_cpu_ns
     pk_ctx c;
     uint64_t t0 = thread_cpu_ns();
     ~CpuTime() { c->stats.host_cpu_ns += thread_cpu_ns() - t0; }
 };
+}  // namespace
 
 int pk_launch_partitioned(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
                           const void* const* args, const int64_t* scalars, int ns) {
