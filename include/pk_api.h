@@ -403,8 +403,20 @@ enum {
                                         pk_stats.graph_launch_ms (graph replay stays on) */
     PK_MODE_NO_GRAPHS = 1u << 5,     /* disable steady-state graph replay (see pk_launch_partitioned) */
     PK_MODE_PUSH = 1u << 6,          /* fused halo push, see below */
-    PK_MODE_NO_OVERLAP = 1u << 7     /* streamed operands are copied before the kernel instead (see below) */
+    PK_MODE_NO_OVERLAP = 1u << 7,    /* streamed operands are copied before the kernel instead (see below) */
+    PK_MODE_NO_COLLECTIVES = 1u << 8 /* one process, P distinct GPUs: whole-buffer reads as peer copies
+                                        instead of one ncclAllGather (see below) */
 };
+/* Whole-buffer reads, one process ("copy the data from its most
+ * recently written GPU", P:L999-1004 Matmul's redistribution).  When a launch's plan for a
+ * buffer is exactly "linear slab q -> every partition p != q" (N-body positions every step,
+ * the GEMM's B operand when it is not streamed) and the P partitions sit on P distinct GPUs,
+ * the P(P-1) copies are ONE in-place ncclAllGather over communicators from ncclCommInitAll
+ * (created at the first such launch, destroyed by pk_finalize; NVLS multicast on NVSwitch
+ * where NCCL picks it), issued on the partitions' streams after the launch's hazard waits.
+ * pk_stats.collectives counts them, moved_bytes/copies as the copies they replace.  Not with
+ * partitions sharing a GPU (NCCL refuses two ranks on one device) or without libnccl: peer
+ * copies.  A context that used a collective launches eagerly from then on (no graph replay). */
 /* Streamed operands -- the transfer overlapped with the kernel it feeds (B200 design; the
  * paper synchronises every read before the launch, Fig. 4 l. 2-8).  A builtin may name one
  * input argument it can consume while its copies are in flight (sgemm_tf32x3: B, the

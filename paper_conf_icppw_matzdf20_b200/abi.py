@@ -31,6 +31,7 @@ PK_MODE_TIME_KERNELS = 1 << 4
 PK_MODE_NO_GRAPHS = 1 << 5
 PK_MODE_PUSH = 1 << 6
 PK_MODE_NO_OVERLAP = 1 << 7
+PK_MODE_NO_COLLECTIVES = 1 << 8
 
 
 class PkError(RuntimeError):

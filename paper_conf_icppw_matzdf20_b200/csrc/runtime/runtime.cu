@@ -145,6 +145,7 @@ struct NcclApi {
     bool ok = false;
     int (*GetUniqueId)(NcclId*) = nullptr;
     int (*CommInitRank)(void** comm, int nranks, NcclId id, int rank) = nullptr;
+    int (*CommInitAll)(void** comms, int ndev, const int* devlist) = nullptr;  // optional (one process)
     int (*CommDestroy)(void* comm) = nullptr;
     int (*Send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
     int (*Recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
@@ -171,6 +172,7 @@ NcclApi load_nccl() {
     api.GetUniqueId = (int (*)(NcclId*))dlsym(h, "ncclGetUniqueId");
     api.CommInitRank = (int (*)(void**, int, NcclId, int))dlsym(h, "ncclCommInitRank");
     api.CommDestroy = (int (*)(void*))dlsym(h, "ncclCommDestroy");
+    api.CommInitAll = (int (*)(void**, int, const int*))dlsym(h, "ncclCommInitAll");
     api.Send = (int (*)(const void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclSend");
     api.Recv = (int (*)(void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclRecv");
     api.AllGather = (int (*)(const void*, void*, size_t, int, void*, cudaStream_t))dlsym(h, "ncclAllGather");
@@ -280,6 +282,10 @@ struct pk_ctx_s {
     int first_local = -1;    // lowest partition owned by this rank
     int nlocal = 0;          // partitions owned by this rank
     void* comm = nullptr;    // ncclComm_t (SPMD only)
+    // one process, P partitions on P distinct GPUs: ncclComm_t per partition from ncclCommInitAll
+    // (created at the first whole-buffer read; ag_state -1 = not tried, 0 = unavailable, 1 = ready)
+    std::vector<void*> ag_comm;
+    int ag_state = -1;
     // SPMD over peer memory (pk_init_spmd_ipc)
     bool ipc = false;
     pk_host_allgather_fn allgather = nullptr;
@@ -979,6 +985,8 @@ int pk_finalize(pk_ctx c) {
         }
         if (c->ev_fork) { cudaSetDevice(c->dev[c->first_local]); cudaEventDestroy(c->ev_fork); }
         if (c->comm) nccl().CommDestroy(c->comm);
+        for (void* cm : c->ag_comm)
+            if (cm) nccl().CommDestroy(cm);
         if (c->timer_start) {
             cudaSetDevice(c->dev[c->first_local]);
             cudaEventDestroy(c->timer_start);
@@ -1528,7 +1536,7 @@ int pk_reset_stats(pk_ctx c) {
 
 int pk_set_mode(pk_ctx c, uint32_t flags) {
     if (!c) return fail(PK_ERR_INVALID, "bad argument");
-    if (flags & ~0xFFu) return fail(PK_ERR_INVALID, "unknown mode flag");
+    if (flags & ~0x1FFu) return fail(PK_ERR_INVALID, "unknown mode flag");
     if ((flags & PK_MODE_PUSH) && !c->host_only && !c->ipc)
         for (int p = 0; p < c->P; ++p)
             for (int q = 0; q < c->P; ++q)
@@ -1592,7 +1600,8 @@ static int launch_memo(pk_ctx c, const LaunchReq* d, int n) {
         return PK_OK;
     };
     // builtin launchers take every scalar from `scalars`, so the key below captures the launch
-    bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && !c->graphs_broken &&
+    // (contexts that all-gathered through NCCL launch eagerly: collectives stay out of captures)
+    bool can_graph = !c->host_only && c->world == 1 && c->nlocal >= 1 && !c->graphs_broken && c->ag_comm.empty() &&
                      !(mode & (PK_MODE_GLOBAL_BARRIER | PK_MODE_NO_GRAPHS));
     for (int i = 0; i < n && can_graph; ++i) {
         const Kernel& K = c->kernels[d[i].k];
@@ -1893,6 +1902,52 @@ static int issue_streamed(pk_ctx c, int p, int64_t b, const std::vector<CopyOp>&
     return PK_OK;
 }
 
+// One process, P partitions on P distinct GPUs: one NCCL communicator per
+// partition from ncclCommInitAll, rank p = partition p, created at the first whole-buffer
+// read.  False (peer copies instead) when partitions share a GPU -- NCCL refuses two ranks on
+// one device -- or NCCL is not loadable.
+static bool single_process_comms(pk_ctx c) {
+    if (c->ag_state >= 0) return c->ag_state == 1;
+    c->ag_state = 0;
+    const NcclApi& n = nccl();
+    if (c->P < 2 || c->world != 1 || c->ipc || !n.ok || !n.CommInitAll) return false;
+    for (int p = 0; p < c->P; ++p)
+        for (int q = 0; q < p; ++q)
+            if (c->dev[p] == c->dev[q]) return false;
+    std::vector<void*> comms((size_t)c->P, nullptr);
+    if (n.CommInitAll(comms.data(), c->P, c->dev.data()) != 0) return false;
+    c->ag_comm = std::move(comms);
+    c->ag_state = 1;
+    c->cur_device = -1;  // NCCL initialisation switches devices
+    return true;
+}
+
+// The plan entries of each buffer in `bufs` are exactly "slab q -> every p != q" for P equal
+// linear slabs (allgather_buffers): one in-place ncclAllGather per buffer, all partitions in
+// one group, each on its partition's stream after pass 1's waits.  NVLS multicast on
+// NVSwitch where NCCL selects it.
+static int allgather_single_process(pk_ctx c, const std::vector<int64_t>& bufs) {
+    const NcclApi& n = nccl();
+    const int P = c->P;
+    if (int r = n.GroupStart()) return fail(PK_ERR_NCCL, std::string("ncclGroupStart: ") + n.GetErrorString(r));
+    for (int64_t b : bufs) {
+        const Buffer& B = c->bufs[b];
+        const uint64_t slab = B.bytes / P;
+        for (int p = 0; p < P; ++p) {
+            if (int r = c->set_device(c->dev[p])) { n.GroupEnd(); return r; }
+            int r = n.AllGather((const char*)B.inst[p] + (uint64_t)p * slab, B.inst[p], slab, kNcclUint8,
+                                c->ag_comm[p], c->stream[p]);
+            if (r) { n.GroupEnd(); return fail(PK_ERR_NCCL, std::string("ncclAllGather: ") + n.GetErrorString(r)); }
+            c->stats.copies += P - 1;
+            c->stats.moved_bytes += (uint64_t)(P - 1) * slab;
+            for (int q = 0; q < P && q < 16; ++q)
+                if (q != p && p < 16) c->stats.pair_bytes[q][p] += slab;
+        }
+    }
+    if (int r = n.GroupEnd()) return fail(PK_ERR_NCCL, std::string("ncclGroupEnd: ") + n.GetErrorString(r));
+    return PK_OK;
+}
+
 static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int32_t block[3], size_t smem,
                         const void* const* args, const int64_t* scalars, int ns) {
     if (!valid_kernel(c, k) || !grid || !block) return fail(PK_ERR_INVALID, "bad argument");
@@ -2085,15 +2140,38 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
         if (alone && granule && (SB.bytes + granule - 1) / granule <= (uint64_t)kMaxGranules)
             sbuf = bid[K.stream_arg];
     }
+    // one process driving P distinct GPUs: the same pattern goes to an in-place
+    // ncclAllGather over a communicator of the partitions' devices (ncclCommInitAll)
+    std::vector<int64_t> ag_local;
+    if (c->world == 1 && !c->ipc && !c->host_only && !c->capturing && transfer &&
+        !(mode & PK_MODE_NO_COLLECTIVES) && !c->last_plan.empty()) {
+        ag_local = allgather_buffers(c->last_plan, P, c->bufs);
+        ag_local.erase(std::remove(ag_local.begin(), ag_local.end(), sbuf), ag_local.end());  // streamed instead
+        if (!ag_local.empty() && !single_process_comms(c)) ag_local.clear();  // peer copies instead
+        c->stats.collectives += ag_local.size();
+    }
     if (!c->host_only) {
         if (transfer && !c->last_plan.empty()) {
-            std::vector<size_t> order;
-            size_t i = 0;
-            while (i < c->last_plan.size()) {
+            // the plan's runs of equal destination [i, j) that this process pulls
+            struct Group { size_t i, j; int p; };
+            std::vector<Group> groups;
+            for (size_t i = 0; i < c->last_plan.size();) {
                 const int p = c->last_plan[i].dst;
                 size_t j = i;
                 while (j < c->last_plan.size() && c->last_plan[j].dst == p) ++j;
-                if (!c->local(p)) { i = j; continue; }  // another rank pulls (NCCL / its own IPC pass)
+                if (c->local(p)) groups.push_back(Group{i, j, p});  // else another rank pulls
+                i = j;
+            }
+            // Pass 1: every destination's waits, before ANY copy of this launch is issued.
+            // The plan was made against the pre-launch tracker state (a3), so a copy never
+            // reads bytes another copy of the same launch delivers: its RAW is on the source's
+            // pre-launch writer, and its WAR on readers of earlier launches.  Waiting here, on
+            // events not yet re-recorded by this launch, keeps the destinations' pulls
+            // concurrent (waiting inside the issue loop chained partition p's pulls behind
+            // p-1's, whose ev_copy had just been re-recorded).
+            for (const Group& g : groups) {
+                const size_t i = g.i, j = g.j;
+                const int p = g.p;
                 if (int r = c->set_device(c->dev[p])) return r;
                 if (c->ipc) {
                     // peer memory: RAW on the holder's flag word of its last write of (b,q);
@@ -2111,8 +2189,9 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                     }
                     if (int r = fw.issue(c, c->stream[p])) return r;
                 }
-                // WAR on the destination instances + RAW on each source's last writer
-                uint64_t waited_src = 0;
+                // WAR on the destination instances + RAW on each source's last writer (kernel
+                // or copy, per buffer: two buffers of one source may differ)
+                uint64_t waited_k = 0, waited_c = 0;
                 for (size_t t = i; t < j; ++t) {
                     const CopyOp& o = c->last_plan[t];
                     if (!c->local(o.src)) continue;
@@ -2123,13 +2202,24 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                         PK_CUDA(cudaStreamWaitEvent(c->stream[p], c->ev_kernel[q], 0));
                     }
                     const uint8_t lw = B.last_writer[o.src];
-                    uint64_t bit = 1ull << o.src;
-                    if (lw != W_NONE && !(waited_src & bit)) {
+                    const uint64_t bit = 1ull << o.src;
+                    uint64_t& waited = lw == W_KERNEL ? waited_k : waited_c;
+                    if (lw != W_NONE && !(waited & bit)) {
                         PK_CUDA(cudaStreamWaitEvent(c->stream[p], lw == W_KERNEL ? c->ev_kernel[o.src]
                                                                                  : c->ev_copy[o.src], 0));
-                        waited_src |= bit;
+                        waited |= bit;
                     }
                 }
+            }
+            // one-process multi-GPU: whole-buffer reads as one in-place all-gather per buffer
+            if (!ag_local.empty())
+                if (int r = allgather_single_process(c, ag_local)) return r;
+            // Pass 2: the copies, pulled on the destination stream
+            std::vector<size_t> order;
+            for (const Group& g : groups) {
+                const size_t i = g.i, j = g.j;
+                const int p = g.p;
+                if (int r = c->set_device(c->dev[p])) return r;
                 // group by (buffer, source) in plan order; a run of equal-length pieces at a
                 // constant pitch (a tile partition's halo column, NEXT-2) is ONE 2-D copy
                 order.resize(j - i);
@@ -2159,6 +2249,10 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 for (size_t t = 0; t < order.size();) {
                     const CopyOp& o = c->last_plan[order[t]];
                     if (!c->local(o.src) && !c->ipc) { ++t; continue; }
+                    if (!ag_local.empty() && std::binary_search(ag_local.begin(), ag_local.end(), o.buf)) {
+                        ++t;  // moved by the all-gather above
+                        continue;
+                    }
                     if (o.buf == sbuf && (c->stream_same_dev || c->dev[o.src] != c->dev[p])) {
                         side_ops.push_back(o);  // streamed: copied on the side stream under the kernel
                         ++t;
@@ -2250,15 +2344,17 @@ static int launch_eager(pk_ctx c, pk_kernel k, const int32_t grid[3], const int3
                 }
                 if (c->ipc)
                     if (int r = ipc_signal(c, p, kFlagCopied, E)) return r;
-                for (size_t t = i; t < j; ++t) {
+            }
+            // Pass 3: bookkeeping for the hazards of later work (a copy-in is the instance's
+            // last writer; the source gains a reader that its next writer must wait for)
+            for (const Group& g : groups)
+                for (size_t t = g.i; t < g.j; ++t) {
                     const CopyOp& o = c->last_plan[t];
                     if (!c->local(o.src)) continue;
                     Buffer& B = c->bufs[o.buf];
-                    B.readers[o.src] |= 1ull << p;
-                    B.last_writer[p] = W_COPY;
+                    B.readers[o.src] |= 1ull << g.p;
+                    B.last_writer[g.p] = W_COPY;
                 }
-                i = j;
-            }
             // SPMD: copies between ranks are NCCL send/recv pairs issued in the
             // global plan order on both sides (one partition per rank, so stream
             // order on that partition covers RAW and both WARs).

@@ -731,3 +731,29 @@ def test_degenerate_buffers_and_grids():
                        [["u0", "u1", 4, 4], ["u1", "u0", 4, 4]], geom,
                        lambda box: regions.jacobi2d(box, (32, 8), 4, 4))
     assert st_["kernel_launches"] == 2                      # one partition launched per launch
+
+
+def test_no_collectives_mode_flag_and_allgather_plan_shape():
+    """PK_MODE_NO_COLLECTIVES (one process, distinct GPUs: whole-buffer reads as peer copies
+    instead of one ncclAllGather) is a known flag; the flag after it is not.  The
+    N-body position plan at P = 4 is the all-gather pattern the one-process path detects:
+    every partition pulls every other partition's linear slab, P(P-1) copies of |pos|/P."""
+    ctx = host_ctx(4, abi.PK_MODE_NO_COLLECTIVES)
+    assert abi.pk_get_mode(ctx) == abi.PK_MODE_NO_COLLECTIVES
+    with pytest.raises(RuntimeError):
+        abi.pk_set_mode(ctx, 1 << 9)
+    abi.pk_finalize(ctx)
+    n, P = 1024, 4
+    ctx = host_ctx(P)
+    k = abi.pk_builtin_kernel(ctx, "nbody")
+    p0 = abi.pk_register_buffer(ctx, (n,), 16, host_init=np.zeros((n, 4), np.float32))
+    p1 = abi.pk_register_buffer(ctx, (n,), 16)
+    v = abi.pk_register_buffer(ctx, (n,), 16, host_init=np.zeros((n, 4), np.float32))
+    grid, blk, sc = K.nbody_launch(n, 32)
+    abi.pk_launch_partitioned(ctx, k, grid, blk, [p0, v, p1, n], sc)
+    plan = abi.pk_last_plan(ctx)
+    slab = n * 16 // P
+    assert sorted((s, d, b, e) for buf, s, d, b, e in plan if buf == p0) == sorted(
+        (q, p, q * slab, (q + 1) * slab) for p in range(P) for q in range(P) if q != p)
+    assert abi.pk_get_stats(ctx)["collectives"] == 0     # host-only: plans, no transport
+    abi.pk_finalize(ctx)
