@@ -13,6 +13,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 # PK_TRACE_ACCESS=1 selects the access-recording build libpk_trace.so (tests of the
 # declared descriptors against what the kernels touch; pk_trace_* below)
 LIB_PATH = os.path.join(_HERE, "libpk_trace.so" if os.environ.get("PK_TRACE_ACCESS") == "1" else "libpk.so")
+LIB_PATH = os.environ.get("PK_LIB_OVERRIDE") or LIB_PATH   # A/B measurements of an older build only
 
 PK_OK = 0
 PK_ERR = {-1: "PK_ERR_INVALID", -2: "PK_ERR_CUDA", -3: "PK_ERR_NCCL", -4: "PK_ERR_OOM",
