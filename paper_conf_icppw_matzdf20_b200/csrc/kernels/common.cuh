@@ -48,6 +48,28 @@ namespace dev {
 // (4-byte granularity ranges; `n` is uniform, usually 0 or 2).
 // (static indices only: a runtime-indexed by-value struct would be copied to local
 // memory.  Kernels instantiate a PUSH=false variant without any of this.)
+// The rows [r0, r1) of a row-major array (row = `pitch` bytes: a grid row, or a plane of
+// a 3-D grid) whose bytes a push range may cover: the hull [*a, *b) of the intersecting
+// rows (empty: *a == *b).  Computed once per tile; a store outside it skips push4's
+// per-range checks, which on every store cost as much as the stencil update itself.
+__device__ __forceinline__ void push_rows(const PushList& pl, int64_t r0, int64_t r1, uint64_t pitch, int64_t* a,
+                                          int64_t* b) {
+    int64_t lo = r1, hi = r0;
+    for (int i = 0; i < kMaxPush; ++i) {
+        if (i >= pl.n) break;
+        if (pl.hi[i] <= pl.lo[i]) continue;
+        const int64_t ra = (int64_t)(pl.lo[i] / pitch), rb = (int64_t)((pl.hi[i] - 1) / pitch) + 1;
+        const int64_t x = ra > r0 ? ra : r0, y = rb < r1 ? rb : r1;
+        if (x < y) {
+            lo = x < lo ? x : lo;
+            hi = y > hi ? y : hi;
+        }
+    }
+    *a = lo < hi ? lo : r0;
+    *b = lo < hi ? hi : r0;
+}
+__device__ __forceinline__ bool in_rows(int64_t r, int64_t a, int64_t b) { return (uint64_t)(r - a) < (uint64_t)(b - a); }
+
 __device__ __forceinline__ void push4(const PushList& pl, uint64_t off, const float4& v) {
 #pragma unroll
     for (int i = 0; i < kMaxPush; ++i)

@@ -183,6 +183,8 @@ __device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t
     const int64_t rowcol = (int64_t)(gr1 + 1) * W + col0;
     const bool top = warp == 0, bot = warp == kNW - 1;
     float4 L1[3][kRW];                                // own rows j = 1..4 at index j - 1
+    int64_t pa = 0, pb = 0;                           // planes of this block a push range may cover
+    if (PUSH) dev::push_rows(push, k0, k0 + nq - 4, (uint64_t)HW * 4u, &pa, &pb);
     ptx::mbar_wait(&full[0], 0);
     ptx::mbar_wait(&full[1], 0);
     for (int q0 = 2; q0 < nq; q0 += 3) {
@@ -250,6 +252,7 @@ __device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t
                 const float4 below = *reinterpret_cast<const float4*>(xr + (2 * warp + 3) * kCols);
                 const int pz = (int)k0 + q - 4;
                 const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == Di - 1;
+                const bool pplane = PUSH && dev::in_rows(pz, pa, pb);
                 float* outp = uout + (int64_t)pz * HW + rowcol;
 #pragma unroll
                 for (int j = 1; j <= kRW; ++j) {
@@ -263,7 +266,7 @@ __device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t
                     if (store_col && (!EDGE || gr < Hi)) {
                         *reinterpret_cast<float4*>(outp) = o;
                         PK_TRACE_W(outp, 16);
-                        if (PUSH) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);
+                        if (PUSH && pplane) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);
                     }
                     outp += W;
                 }

@@ -113,9 +113,12 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUt
     // ring slots of planes z-1, z, z+1 and the parity of z+1, advanced incrementally
     int s_m = 0, s_c = 1, s_p = 2 % kNS;
     uint32_t par_p = (2 / kNS) & 1;
+    int64_t pa = 0, pb = 0;  // planes of this block a push range may cover
+    if (PUSH) dev::push_rows(push, k0, k0 + nz, (uint64_t)HW * 4u, &pa, &pb);
     ptx::mbar_wait(&full[0], 0);
     ptx::mbar_wait(&full[1 % kNS], (1 / kNS) & 1);
     for (int q = 1; q <= nz; ++q) {
+        const bool pplane = PUSH && dev::in_rows(k0 + q - 1, pa, pb);
         ptx::mbar_wait(&full[s_p], par_p);
         const float* sm = reinterpret_cast<const float*>(smem + (size_t)s_m * sb);
         const float* sc = reinterpret_cast<const float*>(smem + (size_t)s_c * sb);
@@ -147,7 +150,7 @@ __global__ void __launch_bounds__(1024) k_heat3d_tma(const __grid_constant__ CUt
             o.w = c.w + kAlpha * ((zm.w + zp.w + ym.w + yp.w + c.z + ev) - 6.0f * c.w);
             *reinterpret_cast<float4*>(uout + kout + i * W + j0) = o;
             PK_TRACE_W(uout + kout + i * W + j0, 16);
-            if (PUSH) dev::push4(push, (uint64_t)(kout + i * W + j0) * 4u, o);  // fused halo push
+            if (PUSH && pplane) dev::push4(push, (uint64_t)(kout + i * W + j0) * 4u, o);  // fused halo push
         }
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&empty[s_m]);  // slot z-1 no longer needed by this warp

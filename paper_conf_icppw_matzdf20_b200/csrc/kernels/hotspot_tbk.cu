@@ -127,6 +127,8 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
     in[1] = *reinterpret_cast<const float4*>(stage(1) + scol);
     float* outp = tout + (int64_t)(base + dir * K) * W + col0;
     const int64_t dW = dir * W;
+    int64_t pa = 0, pb = 0;  // rows of this tile a push range may cover
+    if (PUSH) dev::push_rows(push, r0, rend, (uint64_t)W * 4u, &pa, &pb);
     for (int t0 = 2; t0 < nt; t0 += kW3) {
 #pragma unroll
         for (int u = 0; u < kW3; ++u) {
@@ -155,7 +157,8 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
                     if (store) {
                         *reinterpret_cast<float4*>(outp) = o;
                         PK_TRACE_W(outp, 16);
-                        if (PUSH) dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
+                        if (PUSH && dev::in_rows(base + dir * (t - K), pa, pb))
+                            dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
                     }
                     outp += dW;
                 }

@@ -106,6 +106,8 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restr
         const int64_t j0 = c0 + 4 * tc;
         const bool active = j0 < W;
         const bool west_edge = j0 == 0, east_edge = j0 + 4 >= W;
+        int64_t pa = 0, pb = 0;  // rows of this tile a push range may cover
+        if (PUSH) dev::push_rows(push, r0, rend, (uint64_t)W * 4u, &pa, &pb);
         ptx::mbar_wait(&full[g % kNS], (g / kNS) & 1u);
         ptx::mbar_wait(&full[(g + 1) % kNS], ((g + 1) / kNS) & 1u);
         for (int64_t t = 1; t <= nr; ++t) {
@@ -133,7 +135,8 @@ __global__ void __launch_bounds__(kThreads) k_hotspot2d_tma(const float* __restr
                 const int64_t row = down ? r0 - 1 + t : rend - t;
                 *reinterpret_cast<float4*>(tout + row * W + j0) = o;
                 PK_TRACE_W(tout + row * W + j0, 16);
-                if (PUSH) dev::push4(push, (uint64_t)(row * W + j0) * 4u, o);  // fused halo push
+                if (PUSH && dev::in_rows(row, pa, pb))
+                    dev::push4(push, (uint64_t)(row * W + j0) * 4u, o);  // fused halo push
             }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&empty[gp % kNS]);
