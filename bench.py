@@ -518,8 +518,13 @@ def main():
                     help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
                     help="SPMD (torchrun, N > 1) cross-rank transport: CUDA IPC peer memory or NCCL send/recv")
-    ap.add_argument("--push", action="store_true",
-                    help="PK_MODE_PUSH: halo rows stored into the neighbours' instances by the producing kernel")
+    ap.add_argument("--halo", default="auto", choices=["auto", "pull", "push"],
+                    help="stencil halo transport: pull = copies on the reader's stream after the producer's kernel; "
+                         "push = PK_MODE_PUSH, the producing kernel also stores the halo into the readers' instances "
+                         "(peer stores over NVLink, no copy on the critical path); auto = push when the partitions "
+                         "span several GPUs, else pull (on one GPU a pushed halo costs SM time, a pulled one runs on "
+                         "the copy engines: profiles/r02/push_vs_pull.txt)")
+    ap.add_argument("--push", action="store_true", help="same as --halo push")
     ap.add_argument("--abg", action="store_true",
                     help="also run the paper's alpha/beta/gamma overhead decomposition (P:L1164-1181)")
     ap.add_argument("--abg-repeats", type=int, default=3)
@@ -586,6 +591,11 @@ def main():
         ctx = abi.pk_init(P, part_device=[p % ngpu for p in range(P)])
         devices = sorted(set(p % ngpu for p in range(P)))
         process_model = "one host process drives all partitions"
+    if args.push:
+        args.halo = "push"
+    n_gpu_span = world if world > 1 else len(devices)
+    args.push = args.halo == "push" or (args.halo == "auto" and n_gpu_span > 1 and w.name != "sgemm"
+                                        and w.name != "nbody")
     base_mode = (abi.PK_MODE_PUSH if args.push else 0) | (abi.PK_MODE_NO_OVERLAP if args.no_overlap else 0)
     abi.pk_set_mode(ctx, base_mode)
     w.gpus_used = world if world > 1 else len(devices)

@@ -252,7 +252,7 @@ __device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t
                 const float4 below = *reinterpret_cast<const float4*>(xr + (2 * warp + 3) * kCols);
                 const int pz = (int)k0 + q - 4;
                 const bool zlo = EDGE && pz == 0, zhi = EDGE && pz == Di - 1;
-                const bool pplane = PUSH && dev::in_rows(pz, pa, pb);
+
                 float* outp = uout + (int64_t)pz * HW + rowcol;
 #pragma unroll
                 for (int j = 1; j <= kRW; ++j) {
@@ -266,9 +266,20 @@ __device__ __forceinline__ void consume(const float* ring, float* xbuf, uint64_t
                     if (store_col && (!EDGE || gr < Hi)) {
                         *reinterpret_cast<float4*>(outp) = o;
                         PK_TRACE_W(outp, 16);
-                        if (PUSH && pplane) dev::push4(push, (uint64_t)(outp - uout) * 4u, o);
                     }
                     outp += W;
+                }
+                // PUSH: on the (few) planes a push range may cover, re-read the rows this thread
+                // just stored (its own writes) and forward them -- outside the row loop, so the
+                // update loop carries no store branch
+                if (PUSH && dev::in_rows(pz, pa, pb)) {
+                    const float* rp = uout + (int64_t)pz * HW + rowcol;
+#pragma unroll
+                    for (int j = 1; j <= kRW; ++j, rp += W) {
+                        const int gr = gr1 + j;
+                        if (store_col && (!EDGE || gr < Hi))
+                            dev::push4(push, (uint64_t)(rp - uout) * 4u, *reinterpret_cast<const float4*>(rp));
+                    }
                 }
             }
         }

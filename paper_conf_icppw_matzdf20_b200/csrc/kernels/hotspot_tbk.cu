@@ -105,10 +105,10 @@ __device__ __forceinline__ float4 level(const float4& c, const float4& n, const 
 // in registers (4-fold unroll) needs 168 registers -> 2 CTAs/SM, 1764 GLUP/s; a
 // skewed level schedule (level k at row t-2k+1, independent levels) 1476 GLUP/s;
 // this variant at 128 registers, 3 CTAs/SM and a 16-stage ring: 1940 GLUP/s.
-template <int K, bool EDGE, bool COLEDGE, bool PUSH>
+template <int K, bool EDGE, bool COLEDGE>
 __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, uint64_t* empty, float* tout,
                                              int64_t W, int H, int64_t c0, int64_t r0, int64_t rend, bool down,
-                                             uint32_t g, int lane, int warp, const PushList& push) {
+                                             uint32_t g, int lane, int warp) {
     using G = Geo<K>;
     constexpr int kW3 = 3;
     const int scol = G::Own * warp + 4 * lane;
@@ -127,8 +127,6 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
     in[1] = *reinterpret_cast<const float4*>(stage(1) + scol);
     float* outp = tout + (int64_t)(base + dir * K) * W + col0;
     const int64_t dW = dir * W;
-    int64_t pa = 0, pb = 0;  // rows of this tile a push range may cover
-    if (PUSH) dev::push_rows(push, r0, rend, (uint64_t)W * 4u, &pa, &pb);
     for (int t0 = 2; t0 < nt; t0 += kW3) {
 #pragma unroll
         for (int u = 0; u < kW3; ++u) {
@@ -157,8 +155,6 @@ __device__ __forceinline__ void consume_tile(const float* ring, uint64_t* full, 
                     if (store) {
                         *reinterpret_cast<float4*>(outp) = o;
                         PK_TRACE_W(outp, 16);
-                        if (PUSH && dev::in_rows(base + dir * (t - K), pa, pb))
-                            dev::push4(push, (uint64_t)(outp - tout) * 4u, o);  // fused halo push
                     }
                     outp += dW;
                 }
@@ -234,11 +230,22 @@ __global__ void __launch_bounds__(kThreads, K <= 4 ? PK_TBK_MINB : PK_TBK8_MINB)
         const bool redge = r0 < K + 1 || rend + K + 1 > H;
         const bool cedge = c0 == 0 || c0 + G::TC + 4 * G::HL >= W;
         if (redge || cedge)
-            consume_tile<K, true, true, PUSH>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp,
-                                              push);
+            consume_tile<K, true, true>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp);
         else
-            consume_tile<K, false, false, PUSH>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp,
-                                                push);
+            consume_tile<K, false, false>(ring, full, empty, tout, W, (int)H, c0, r0, rend, down, g, lane, warp);
+        if (PUSH) {
+            // fused halo push: the tile's rows a push range may cover (usually the K rows at a
+            // partition edge, else none) are re-read from this thread's own stores and forwarded.
+            // A store branch inside the level loop cost ~19 % per launch even when never taken.
+            int64_t pa = 0, pb = 0;
+            dev::push_rows(push, r0, rend, (uint64_t)W * 4u, &pa, &pb);
+            const int64_t col0 = c0 - 4 * G::HL + G::Own * warp + 4 * lane;
+            if (pb > pa && lane >= G::HL && lane <= 31 - G::HL && col0 < W)
+                for (int64_t R = pa; R < pb; ++R) {
+                    const float* rp = tout + R * W + col0;
+                    dev::push4(push, (uint64_t)(rp - tout) * 4u, *reinterpret_cast<const float4*>(rp));
+                }
+        }
         g += (uint32_t)(rend - r0) + 2 * K;
     }
 }
