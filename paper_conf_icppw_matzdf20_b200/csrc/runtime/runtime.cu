@@ -1944,7 +1944,9 @@ static int allgather_single_process(pk_ctx c, const std::vector<int64_t>& bufs) 
                 if (q != p && p < 16) c->stats.pair_bytes[q][p] += slab;
         }
     }
-    if (int r = n.GroupEnd()) return fail(PK_ERR_NCCL, std::string("ncclGroupEnd: ") + n.GetErrorString(r));
+    const int r = n.GroupEnd();
+    c->cur_device = -1;  // NCCL may have switched the current device
+    if (r) return fail(PK_ERR_NCCL, std::string("ncclGroupEnd: ") + n.GetErrorString(r));
     return PK_OK;
 }
 
