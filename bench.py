@@ -50,6 +50,19 @@ WORKLOADS = {
 }
 
 
+def halo_push(halo, n_gpus, workload):
+    """--halo: pull (copies on the reader's stream), push (PK_MODE_PUSH: the producing kernel stores
+    the halo into the readers' instances) or auto = push when the partitions span several GPUs for
+    the stencils (a pull there puts a copy between the producer's kernel and the reader's next one;
+    on one GPU a pushed halo takes SM time while a pulled one runs on the copy engines).  The GEMM
+    and N-body read whole buffers: streamed operand / all-gather, nothing to push."""
+    if halo == "push":
+        return True
+    if halo == "pull":
+        return False
+    return n_gpus > 1 and workload in ("hotspot2d", "heat3d", "jacobi2d")
+
+
 def env_int(name, default):
     try:
         return int(os.environ.get(name, default))
@@ -593,9 +606,7 @@ def main():
         process_model = "one host process drives all partitions"
     if args.push:
         args.halo = "push"
-    n_gpu_span = world if world > 1 else len(devices)
-    args.push = args.halo == "push" or (args.halo == "auto" and n_gpu_span > 1 and w.name != "sgemm"
-                                        and w.name != "nbody")
+    args.push = halo_push(args.halo, world if world > 1 else len(devices), w.name)
     base_mode = (abi.PK_MODE_PUSH if args.push else 0) | (abi.PK_MODE_NO_OVERLAP if args.no_overlap else 0)
     abi.pk_set_mode(ctx, base_mode)
     w.gpus_used = world if world > 1 else len(devices)

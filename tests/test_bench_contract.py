@@ -62,3 +62,12 @@ def test_reference_arm_under_torchrun_uses_all_host_cores():
     assert len(lines) == 1                     # rank 0 prints the one line
     line = json.loads(lines[0])
     assert line["n_gpus"] == 2 and line["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
+
+
+def test_halo_transport_choice():
+    b = _bench_module()
+    assert b.halo_push("auto", 1, "hotspot2d") is False          # one GPU: pull (copy engines)
+    assert b.halo_push("auto", 8, "hotspot2d") is True           # across GPUs: fused push
+    assert b.halo_push("auto", 2, "heat3d") and b.halo_push("auto", 2, "jacobi2d")
+    assert not b.halo_push("auto", 8, "sgemm") and not b.halo_push("auto", 8, "nbody")
+    assert b.halo_push("push", 1, "hotspot2d") and not b.halo_push("pull", 8, "hotspot2d")
