@@ -108,3 +108,8 @@ def hotspot2d_tbk_power_once(w: int, nparts: int, k: int, elem_bytes: int = 4) -
 def heat3d_tb2_stale_per_launch(h: int, w: int, nparts: int, elem_bytes: int = 4) -> int:
     """Two fused 7-point sweeps per launch: two h x w planes each way per z-cut."""
     return (nparts - 1) * 2 * 2 * h * w * elem_bytes
+
+
+def heat3d_tb3_stale_per_launch(h: int, w: int, nparts: int, elem_bytes: int = 4) -> int:
+    """Three fused 7-point sweeps per launch: three h x w planes each way per z-cut."""
+    return (nparts - 1) * 2 * 3 * h * w * elem_bytes

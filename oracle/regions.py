@@ -152,10 +152,12 @@ def nbody(box, block, n, per_thread=2):
             (2, WRITE): _uniq([i])}
 
 
-def heat3d_tb2(box, d, h, w, zc, cols=120, rows=24):
-    """Two fused sweeps per launch (heat3d_tb2): logical block (bx, by, bz) owns columns
-    [cols*bx, +cols) x rows [rows*by, +rows) x planes [zc*bz, +zc); every owned cell
-    reads the clamped 5x5x5 cube of u_in around it and writes u_out at the cell."""
+def heat3d_tb2(box, d, h, w, zc, cols=120, rows=24, sweeps=2):
+    """`sweeps` fused sweeps per launch (heat3d_tb2: 2, heat3d_tb3: 3): logical block
+    (bx, by, bz) owns columns [cols*bx, +cols) x rows [rows*by, +rows) x planes
+    [zc*bz, +zc); every owned cell reads the clamped (2s+1)^3 cube of u_in around it
+    (s = sweeps: each sweep widens the dependence by one cell per direction) and writes
+    u_out at the cell."""
     bzs, bys, bxs = _block_ranges(box)
     k = (bzs[:, None] * zc + np.arange(zc)[None, :]).ravel()
     i = (bys[:, None] * rows + np.arange(rows)[None, :]).ravel()
@@ -164,7 +166,8 @@ def heat3d_tb2(box, d, h, w, zc, cols=120, rows=24):
     Kk, I, J = np.meshgrid(k, i, j, indexing="ij")
     s = (d, h, w)
     rd = [_ravel(_clamp(Kk + dz, d), _clamp(I + dy, h), _clamp(J + dx, w), s)
-          for dz in range(-2, 3) for dy in range(-2, 3) for dx in range(-2, 3)]
+          for dz in range(-sweeps, sweeps + 1) for dy in range(-sweeps, sweeps + 1)
+          for dx in range(-sweeps, sweeps + 1)]
     return {(0, READ): _uniq(rd), (1, WRITE): _uniq([_ravel(Kk, I, J, s)])}
 
 

@@ -148,7 +148,11 @@ __global__ void __maxnreg__(PK_HEATTB_MAXNREG)
 
     // ---------------- consumers: blocks touching the grid's first/last row or plane apply
     // the replicate clamp of the intermediate sweep; interior blocks skip the selects
+#ifdef PK_HEATTB_ALLEDGE   // diagnostic: every block through the clamping consumer
+    const bool edge = true;
+#else
     const bool edge = y0 < 2 || y0 + kRows + 2 > H || k0 < 2 || k0 + ZC + 2 > D;
+#endif
     if (edge)
         consume<PUSH, true>(ring, xbuf, full, empty, uout, D, H, W, c0, y0, k0, nq, lane, warp, push);
     else

@@ -32,6 +32,17 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "r"(parity)
         : "memory");
 }
+// Wait with a suspend-time hint: the warp sleeps in try_wait (woken when the phase
+// completes or the hint expires) instead of re-issuing the poll loop.
+__device__ __forceinline__ void mbar_wait_hint(uint64_t* bar, uint32_t parity, uint32_t ns) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "LAB_WAITH:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra LAB_WAITH;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity), "r"(ns)
+        : "memory");
+}
 // Wait for a phase with a nanosleep back-off between polls: for a producer thread,
 // whose refill may lag by a fraction of a microsecond without starving anyone, so
 // that its polling does not take issue slots from the consumer warps of the SM.

@@ -90,6 +90,7 @@ extern const Builtin kBuiltinHotspot2dTbk;  // hotspot2d_tbk (K = 2..4 sweeps pe
 extern const Builtin kBuiltinHeat3d;
 extern const Builtin kBuiltinHeat3dTma;      // heat3d (TMA plane ring, default); kBuiltinHeat3d = heat3d_regs
 extern const Builtin kBuiltinHeat3dTb2;      // heat3d_tb2 (two sweeps per launch)
+extern const Builtin kBuiltinHeat3dTb3;      // heat3d_tb3 (three sweeps per launch)
 extern const Builtin kBuiltinNbody;
 extern const Builtin kBuiltinSgemm;          // sgemm_tf32x3 (tcgen05 3xTF32)
 

@@ -84,6 +84,15 @@ def heat3d_tb2_launch(d, h, w, zc=HEAT_TB2_ZC):
     return (_cdiv(w, HEAT_TB2_COLS), _cdiv(h, HEAT_TB2_ROWS), _cdiv(d, zc)), (160, 1, 1), [d, h, w, zc]
 
 
+HEAT_TB3_ZC = 128                         # "heat3d_tb3": planes per logical block (6 halo planes per block)
+
+
+def heat3d_tb3_launch(d, h, w, zc=HEAT_TB3_ZC):
+    """Logical block = 120 columns x 16 rows x zc planes, three sweeps per launch (256 threads:
+    4 row warps, 3 sweep-1 warps, 1 producer warp)."""
+    return (_cdiv(w, HEAT_TB2_COLS), _cdiv(h, HEAT_TB2_ROWS), _cdiv(d, zc)), (256, 1, 1), [d, h, w, zc]
+
+
 def nbody_launch(n, bdx=NBODY_BDX):
     return (_cdiv(n, NBODY_PER_THREAD * bdx), 1, 1), (bdx, 1, 1), [n]
 
@@ -210,26 +219,48 @@ def hotspot2d_iterate(pr, iters, start=0):
 
 
 def heat3d_setup(ctx, u_host, zc=None, bdy=HEAT_BDY, kernel="heat3d", tiles=None):
-    """kernel: heat3d (one sweep per launch, TMA ring), heat3d_regs, heat3d_tb2 (two)."""
+    """kernel: heat3d (one sweep per launch, TMA ring), heat3d_regs, heat3d_tb2 (two), heat3d_tb3 (three)."""
     d, h, w = u_host.shape
     pr = Problem(ctx, kernel, tiles)
     u0 = pr.buffer((d, h, w), 4, host=u_host)
     u1 = pr.buffer((d, h, w), 4)
     if kernel == "heat3d_tb2":
         pr.geom = heat3d_tb2_launch(d, h, w, zc or HEAT_TB2_ZC)
+    elif kernel == "heat3d_tb3":
+        pr.geom = heat3d_tb3_launch(d, h, w, zc or HEAT_TB3_ZC)
     else:
         pr.geom = heat3d_launch(d, h, w, zc or HEAT_ZC, bdy)
     pr.shape = (d, h, w)
     pr.ub = (u0, u1)
-    pr.sweeps = 2 if kernel == "heat3d_tb2" else 1
+    pr.sweeps = {"heat3d_tb2": 2, "heat3d_tb3": 3}.get(kernel, 1)
+    if kernel == "heat3d_tb3":
+        # a remainder of 1 or 2 sweeps (C3's 50 = 16 x 3 + 2) runs on heat3d / heat3d_tb2 over the
+        # same buffers: every cell is the same expression in all three kernels (bit-identical)
+        pr.tail = {1: Problem(ctx, "heat3d", tiles), 2: Problem(ctx, "heat3d_tb2", tiles)}
+        pr.tail_geom = {1: heat3d_launch(d, h, w, HEAT_ZC, bdy), 2: heat3d_tb2_launch(d, h, w, HEAT_TB2_ZC)}
+        pr.cur = 0
     return pr
 
 
 def heat3d_iterate(pr, iters, start=0):
-    """`iters` sweeps from sweep `start` (multiples of pr.sweeps for heat3d_tb2)."""
+    """`iters` sweeps from sweep `start` (multiples of pr.sweeps for heat3d_tb2 / heat3d_tb3)."""
     (u0, u1), (d, h, w) = pr.ub, pr.shape
     grid, blk, sc = pr.geom
     k = pr.sweeps
+    if hasattr(pr, "tail"):
+        # heat3d_tb3: the ping-pong state is the number of launches so far (pr.cur = buffer
+        # holding the current field), since a remainder launch advances fewer sweeps
+        n, rem = divmod(iters, k)
+        for _ in range(n):
+            a, b = pr.ub[pr.cur], pr.ub[1 - pr.cur]
+            pr.launch(grid, blk, [a, b, d, h, w, sc[3]], sc)
+            pr.cur = 1 - pr.cur
+        if rem:
+            a, b = pr.ub[pr.cur], pr.ub[1 - pr.cur]
+            g2, b2, s2 = pr.tail_geom[rem]
+            pr.tail[rem].launch(g2, b2, [a, b, d, h, w, s2[3]], s2)
+            pr.cur = 1 - pr.cur
+        return pr.ub[pr.cur]
     if iters % k or start % k:
         raise ValueError(f"this kernel advances {k} steps per launch")
     for t in range(start // k, (start + iters) // k):

@@ -72,7 +72,8 @@ def _heat(name, ctx, make, d, h, w, zc, bdy=K.HEAT_BDY):
     u = synth.heat_grid(d, h, w)
     kid = abi.pk_builtin_kernel(ctx, name)
     u0, u1 = make((d, h, w), 4, u), make((d, h, w), 4, None)
-    geom = K.heat3d_tb2_launch(d, h, w, zc) if name == "heat3d_tb2" else K.heat3d_launch(d, h, w, zc, bdy)
+    geom = (K.heat3d_tb2_launch(d, h, w, zc) if name == "heat3d_tb2" else
+            K.heat3d_tb3_launch(d, h, w, zc) if name == "heat3d_tb3" else K.heat3d_launch(d, h, w, zc, bdy))
     grid, blk, sc = geom
     launches = [(grid, blk, [u0, u1, d, h, w, sc[3]], sc), (grid, blk, [u1, u0, d, h, w, sc[3]], sc)]
     return kid, launches, {u0: ((d, h, w), 4), u1: ((d, h, w), 4)}
@@ -88,6 +89,10 @@ def heat3d_regs(ctx, make):
 
 def heat3d_tb2(ctx, make):
     return _heat("heat3d_tb2", ctx, make, 21, 40, 252, 4)
+
+
+def heat3d_tb3(ctx, make):
+    return _heat("heat3d_tb3", ctx, make, 21, 40, 252, 4)
 
 
 def nbody(ctx, make, n=3000):
@@ -121,12 +126,13 @@ def tiled(case, tiles):
 
 
 _BASE = (jacobi2d, hotspot2d, hotspot2d_regs, hotspot2d_tb2, hotspot2d_tbk(2), hotspot2d_tbk(3), hotspot2d_tbk(4),
-         hotspot2d_tbk(6), hotspot2d_tbk(8), heat3d, heat3d_regs, heat3d_tb2, nbody, sgemm)
+         hotspot2d_tbk(6), hotspot2d_tbk(8), heat3d, heat3d_regs, heat3d_tb2, heat3d_tb3, nbody, sgemm)
 _B = {f.__name__: f for f in _BASE}
 _TILED = (tiled(_B["jacobi2d"], (2, 2, 1)), tiled(_B["hotspot2d"], (3, 1, 1)), tiled(_B["hotspot2d_regs"], (2, 2, 1)),
           tiled(_B["hotspot2d_tb2"], (3, 1, 1)), tiled(_B["hotspot2d_tbk2"], (3, 1, 1)),
           tiled(_B["hotspot2d_tbk3"], (2, 2, 1)), tiled(_B["hotspot2d_tbk4"], (3, 1, 1)),
           tiled(_B["hotspot2d_tbk8"], (3, 1, 1)), tiled(_B["heat3d"], (2, 1, 2)), tiled(_B["heat3d_tb2"], (2, 1, 2)),
+          tiled(_B["heat3d_tb3"], (2, 1, 2)),
           tiled(_B["sgemm"], (2, 2, 1)))
 CASES = {f.__name__: f for f in _BASE + _TILED}
 
@@ -149,6 +155,7 @@ OVERFETCH = {
     # rows and columns are declared): 136 x (bdy + 2) box = 4 columns / 1 row around the block
     ("heat3d", 0): (0, 1, 4),
     ("heat3d_tb2", 0): (0, 0, 2),                 # 128 x 20 box for 120 x 16 owned: 4 columns, 2 used
+    ("heat3d_tb3", 0): (0, 0, 1),                 # 128 x 22 box for 120 x 16 owned: 4 columns, 3 used
 }
 for _k in (2, 3, 4, 6, 8):
     OVERFETCH[(f"hotspot2d_tbk{_k}", 0)] = (0, 0, _tbk_halo(_k) - _k)

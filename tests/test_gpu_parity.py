@@ -729,6 +729,67 @@ def test_heat3d_tb2_push_bitwise():
     assert np.array_equal(r1, rp) and st["pushed_bytes"] > 0
 
 
+# ------------------------------------------------------------------ three-sweep heat (heat3d_tb3)
+def _heat_tb3(u, iters, P, zc, mode=0):
+    ctx = gpu_ctx(P, mode)
+    pr = K.heat3d_setup(ctx, u, zc, kernel="heat3d_tb3")
+    res = fetch(ctx, K.heat3d_iterate(pr, iters), u.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st
+
+
+@pytest.mark.parametrize("d,h,w,zc", [(40, 36, 132, 8), (17, 9, 256, 4), (9, 70, 260, 3), (30, 50, 124, 128),
+                                      (5, 3, 4, 2), (13, 22, 248, 1)])
+def test_heat3d_tb3_oracle_and_bitwise(d, h, w, zc):
+    """Three sweeps per launch: within 1e-5 of the fp64 oracle, P-way bit-identical to 1-way,
+    moved == stale == three planes each way per z-cut and launch (closed form), and
+    bit-identical to heat3d_tb2 (every cell is the same expression on the same inputs)."""
+    u = synth.heat_grid(d, h, w)
+    iters = 6
+    ref = ok.heat3d(u, iters)
+    g1, s1 = _heat_tb3(u, iters, 1, zc)
+    ok_, err = rel_ok(g1, ref, 1e-5)
+    assert ok_, err
+    assert s1["kernel_launches"] == iters // 3
+    g2, _ = _heat_tb2(u, iters, 1, max(2, zc))
+    assert np.array_equal(g1, g2)
+    for P in (2, 3, 5):
+        gp, st = _heat_tb3(u, iters, P, zc)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+        nz = -(-d // zc)
+        if nz % P == 0 and d % zc == 0 and d // P >= 3:
+            assert st["stale_bytes"] == (iters // 3) * cf.heat3d_tb3_stale_per_launch(h, w, P)
+
+
+@pytest.mark.parametrize("iters", [7, 8])
+def test_heat3d_tb3_remainder_sweeps(iters):
+    """C3's 50 sweeps = 16 three-sweep launches + a 2-sweep heat3d_tb2 launch: a remainder of
+    1 or 2 sweeps runs on heat3d / heat3d_tb2 over the same buffers, bit-identical to
+    heat3d_tb2 alone, and calls continue the ping-pong from the launch count."""
+    u = synth.heat_grid(20, 34, 252)
+    ctx = gpu_ctx(2)
+    pr = K.heat3d_setup(ctx, u, 4, kernel="heat3d_tb3")
+    K.heat3d_iterate(pr, iters)
+    g = fetch(ctx, K.heat3d_iterate(pr, iters), u.shape)
+    abi.pk_finalize(ctx)
+    ok_, err = rel_ok(g, ok.heat3d(u, 2 * iters), 1e-5)
+    assert ok_, err
+    ctx = gpu_ctx(1)
+    pr = K.heat3d_setup(ctx, u, 4, kernel="heat3d")
+    ref = fetch(ctx, K.heat3d_iterate(pr, 2 * iters), u.shape)
+    abi.pk_finalize(ctx)
+    assert np.array_equal(g, ref)
+
+
+def test_heat3d_tb3_push_bitwise():
+    u = synth.heat_grid(40, 36, 132)
+    r1, _ = _heat_tb3(u, 9, 1, 8)
+    rp, st = _heat_tb3(u, 9, 3, 8, abi.PK_MODE_PUSH)
+    assert np.array_equal(r1, rp) and st["pushed_bytes"] > 0
+
+
 # ------------------------------------------------------------------ asynchronous host copies (pipelined steps)
 @pytest.mark.parametrize("P", [1, 3])
 def test_async_host_copies_pipelined_contexts(P):

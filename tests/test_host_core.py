@@ -710,6 +710,22 @@ def test_heat3d_tb2_regions(d, h, w, zc, P):
     abi.pk_finalize(ctx)
 
 
+@pytest.mark.parametrize("d,h,w,zc", [(10, 30, 260, 4), (7, 50, 124, 128), (3, 5, 8, 2)])
+@pytest.mark.parametrize("P", [1, 2, 3, 5])
+def test_heat3d_tb3_regions(d, h, w, zc, P):
+    """Three sweeps per launch: one tap dilated by 3 == brute-force clamped 7x7x7 cubes."""
+    ctx = host_ctx(P)
+    kk = abi.pk_builtin_kernel(ctx, "heat3d_tb3")
+    bufs = [abi.pk_register_buffer(ctx, (d, h, w), 4) for _ in range(2)]
+    grid, blk, sc = K.heat3d_tb3_launch(d, h, w, zc)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, kk, grid, p)
+        lib = _lib_sets(ctx, kk, 6, bufs + [None] * 4, box, blk, sc)
+        ora = _oracle_sets(regions.heat3d_tb2(box, d, h, w, zc, rows=16, sweeps=3), {0: 4, 1: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
 # ------------------------------------------------------------------ degenerate cases
 def test_degenerate_buffers_and_grids():
     """A zero-element buffer holds no segments; an empty grid launches nothing and moves

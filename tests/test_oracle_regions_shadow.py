@@ -264,6 +264,26 @@ def test_heat3d_tb2_stale_matches_closed_form(nparts):
     assert stale == [cf.heat3d_tb2_stale_per_launch(h, w, nparts)] * 3
 
 
+@pytest.mark.parametrize("nparts", [2, 4])
+def test_heat3d_tb3_stale_matches_closed_form(nparts):
+    """Three sweeps: the thread program's 7x7x7 cones cross each z-cut by 3 planes (hand
+    count: 3 planes x h x w x 4 B each way), not 2 (two sweeps) or 4."""
+    d, h, w, zc = 24, 6, 8, 3
+    g = (1, 1, d // zc)
+    sh = shadow.Shadow(nparts)
+    sh.register("u0", d * h * w, 4, True)
+    sh.register("u1", d * h * w, 4, False)
+    stale = []
+    for it in range(3):
+        a, b = ("u0", "u1") if it % 2 == 0 else ("u1", "u0")
+        per = []
+        for p in range(nparts):
+            acc = regions.heat3d_tb2(grid.partition_box(g, nparts, p), d, h, w, zc, sweeps=3)
+            per.append({a: (acc[(0, "r")], None), b: (None, acc[(1, "w")])})
+        stale.append(sum(sh.launch(per)["stale"]))
+    assert stale == [cf.heat3d_tb3_stale_per_launch(h, w, nparts)] * 3 == [(nparts - 1) * 6 * 6 * 8 * 4] * 3
+
+
 @pytest.mark.parametrize("nparts", [2, 3, 4, 8])
 def test_hotspot_steady_state_matches_closed_form(nparts):
     h = w = 64
