@@ -85,9 +85,11 @@ def test_c2_hotspot_fullsize_tbk_sampled():
 
 
 # ------------------------------------------------------------------ C3 Heat 1024^3, 50 it
-@pytest.mark.parametrize("kernel", ["heat3d_tb2", "heat3d"])
+@pytest.mark.parametrize("kernel", ["heat3d_tb2", "heat3d", "heat3d_tb3"])
 def test_c3_heat_fullsize_sampled(kernel):
-    """heat3d_tb2 (bench default: 25 launches of two sweeps, ZC = 64) and heat3d (one sweep)."""
+    """heat3d_tb2 (bench default: 25 launches of two sweeps, ZC = 64), heat3d (one sweep) and
+    heat3d_tb3 (16 launches of three sweeps + one two-sweep launch, ZC = 128); stale bytes are
+    two planes per sweep and cut whatever the blocking."""
     d = h = w = 1024
     iters = 50
     u = synth.heat_grid(d, h, w)
