@@ -357,7 +357,18 @@ class Workload:
             for _ in range(4):
                 self.step_once()
         elif self.name == "jacobi2d":
-            self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0, tiles=self.tiles)
+            if (getattr(self, "variant", None) or "jacobi2d_tb") == "jacobi2d_tb":
+                # default C1 kernel: K sweeps per launch (ghost zones), K = --sweeps or half a
+                # step's iterations (two launches per step: an even count replays one graph per
+                # step; odd counts alternate two graphs and measured 2x slower, scripts/r02/gpu_70.sh)
+                k = getattr(self, "sweeps_jacobi", None) or (self.iters // 2 if self.iters % 2 == 0 and
+                                                              self.iters <= 32 else min(self.iters, 16))
+                self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0, tiles=self.tiles, kernel="jacobi2d_tb",
+                                                sweeps=k)
+                self.sweeps = k
+                self.bytes_per_unit = 8 / k
+            else:
+                self.pr, _ = K.jacobi2d_program(ctx, self.host[0], 0, tiles=self.tiles)
             self.upload_bufs = [(b, self.host[0]) for b in self.pr.bufs]
         elif self.name == "nbody":
             self.pr = K.nbody_setup(ctx, *self.host)
@@ -525,7 +536,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--variant", default=None, help="kernel variant (hotspot2d_regs: register-window Hotspot)")
-    ap.add_argument("--sweeps", type=int, default=4, help="time steps per launch of hotspot2d_tbk (2..8; iterations must be a multiple)")
+    ap.add_argument("--sweeps", type=int, default=None,
+                    help="time steps per launch: hotspot2d_tbk 2..8 (default 4; iterations must be a multiple), "
+                         "jacobi2d_tb 1..16 (default: a step's iterations)")
     ap.add_argument("--tile", type=int, default=0, help="rows per block (hotspot2d TY) / planes per block (heat3d ZC)")
     ap.add_argument("--tiles", default=None,
                     help="tile partitions TXxTY[xTZ] (NEXT-2) instead of 1-D slabs; product = partitions")
@@ -555,7 +568,8 @@ def main():
         dist.init_process_group("gloo")
     w = Workload(args.workload, args.iters or WORKLOADS[args.workload][1])
     w.variant = args.variant
-    w.sweeps_arg = args.sweeps
+    w.sweeps_arg = args.sweeps or 4
+    w.sweeps_jacobi = args.sweeps
     w.tile = args.tile
     w.tiles = None
     if args.tiles:
@@ -678,7 +692,8 @@ def main():
     units = w.units_per_iter * w.iters * args.steps
     value = units / (elapsed_ms / 1e3) / w.scale
     peaks = load_peaks()
-    kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk", "heat3d": "heat3d_tb2"}.get(w.name, w.name)
+    kname = getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk", "heat3d": "heat3d_tb2",
+                                            "jacobi2d": "jacobi2d_tb"}.get(w.name, w.name)
     # duration of one timed launch: a replayed graph (single process: every partition's
     # copies + kernels of the launch) or, launched eagerly, the slowest partition kernel
     # (a launch captured into a graph inside the timed region carries no events: not counted)
@@ -731,8 +746,8 @@ def main():
                    "process_model": process_model,
                    "halo_push": bool(args.push),
                    "overlap": not args.no_overlap,
-                   "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk",
-                                                             "heat3d": "heat3d_tb2"}.get(w.name, w.name),
+                   "kernel": getattr(w, "variant", None) or {"hotspot2d": "hotspot2d_tbk", "heat3d": "heat3d_tb2",
+                                                             "jacobi2d": "jacobi2d_tb"}.get(w.name, w.name),
                    "sweeps_per_launch": getattr(w, "sweeps", 1),
                    **({"rows_per_tile": w.block_depth()} if w.name == "hotspot2d" and not w.variant else {}),
                    **({"planes_per_block": w.block_depth()} if w.name == "heat3d" and not w.variant else {}),

@@ -60,6 +60,27 @@ def jacobi2d(box, block, h, w):
     return {(0, READ): _uniq(reads), (1, WRITE): _uniq([_ravel(I, J, (h, w))])}
 
 
+def jacobi2d_tb(box, h, w, k, t=32):
+    """K fused C1 sweeps per launch (jacobi2d_tb): logical block (bx, by) owns the t x t
+    cells rows [t*by, +t) x cols [t*bx, +t); it loads every grid cell within K of its
+    tile (the square window, corners included) and writes its interior cells."""
+    _, bys, bxs = _block_ranges(box)
+    reads, writes = [], []
+    for by in bys:
+        for bx in bxs:
+            r = np.arange(by * t - k, by * t + t + k)
+            c = np.arange(bx * t - k, bx * t + t + k)
+            r, c = r[(r >= 0) & (r < h)], c[(c >= 0) & (c < w)]
+            R, C = np.meshgrid(r, c, indexing="ij")
+            reads.append(_ravel(R, C, (h, w)))
+            ro = np.arange(by * t, by * t + t)
+            co = np.arange(bx * t, bx * t + t)
+            ro, co = ro[(ro >= 1) & (ro <= h - 2)], co[(co >= 1) & (co <= w - 2)]
+            R, C = np.meshgrid(ro, co, indexing="ij")
+            writes.append(_ravel(R, C, (h, w)))
+    return {(0, READ): _uniq(reads), (1, WRITE): _uniq(writes)}
+
+
 # ---------------------------------------------------------------------------
 # C2 hotspot2d(temp_in, power, temp_out; H, W, TY): block (bdx) threads, each
 #   thread owns VEC=4 consecutive columns j = bx*4*bdx + 4*tx + v and marches the

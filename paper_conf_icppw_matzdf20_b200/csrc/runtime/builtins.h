@@ -83,6 +83,7 @@ int32_t find_builtin_push_arg(const void* fn);
 
 // Per-kernel-file registration (defined in kernels/*.cu)
 extern const Builtin kBuiltinJacobi2d;
+extern const Builtin kBuiltinJacobi2dTb;     // jacobi2d_tb (K sweeps per launch, ghost zones)
 extern const Builtin kBuiltinHotspot2d;     // hotspot2d_regs (register window)
 extern const Builtin kBuiltinHotspot2dTma;  // hotspot2d (TMA bulk ring, default)
 extern const Builtin kBuiltinHotspot2dTb2;  // hotspot2d_tb2 (two sweeps per launch)

@@ -2743,7 +2743,7 @@ void* context_scratch(const LaunchInfo& li, int slot, size_t bytes, cudaError_t*
 
 // the one registry of builtin kernels (kernels/*.cu)
 static const Builtin* const kAllBuiltins[] = {
-    &kBuiltinJacobi2d,     &kBuiltinHotspot2dTma, &kBuiltinHotspot2d, &kBuiltinHotspot2dTb2, &kBuiltinHotspot2dTbk,
+    &kBuiltinJacobi2d,     &kBuiltinJacobi2dTb,   &kBuiltinHotspot2dTma, &kBuiltinHotspot2d, &kBuiltinHotspot2dTb2, &kBuiltinHotspot2dTbk,
     &kBuiltinHeat3dTma,    &kBuiltinHeat3d,       &kBuiltinHeat3dTb2, &kBuiltinHeat3dTb3,    &kBuiltinNbody,
     &kBuiltinSgemm};
 

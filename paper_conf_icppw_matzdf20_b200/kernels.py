@@ -155,25 +155,51 @@ class Problem:
             abi.pk_launch_sequence(self.ctx, [(self.k, g, b, a, sc) for g, b, a, sc in launches])
 
 
-def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None, sequence=False):
+JACOBI_TB_T = 32                          # "jacobi2d_tb": owned rows x columns per logical block
+
+
+def jacobi2d_tb_launch(h, w, k):
+    """Logical block = 32 x 32 cells, k sweeps per launch (256 threads, ghost zones)."""
+    return (_cdiv(w, JACOBI_TB_T), _cdiv(h, JACOBI_TB_T), 1), (256, 1, 1), [h, w, k]
+
+
+def jacobi2d_program(ctx, u_host, iters, block=JACOBI_BLOCK, tiles=None, sequence=False, kernel="jacobi2d",
+                     sweeps=1):
     """C1: both buffers carry the Dirichlet boundary (uploaded); returns the buffer id
     that holds the result after `iters` sweeps (sequence=True: the sweeps go out as one
-    pk_launch_sequence)."""
+    pk_launch_sequence).  kernel="jacobi2d_tb": `sweeps` (1..16) sweeps per launch."""
     h, w = u_host.shape
-    pr = Problem(ctx, "jacobi2d", tiles)
+    pr = Problem(ctx, kernel, tiles)
     pr.buffer((h, w), 4, host=u_host)
     pr.buffer((h, w), 4, host=u_host)
-    pr.geom = jacobi2d_launch(h, w, block)
+    pr.sweeps = sweeps if kernel == "jacobi2d_tb" else 1
+    pr.geom = jacobi2d_tb_launch(h, w, sweeps) if kernel == "jacobi2d_tb" else jacobi2d_launch(h, w, block)
+    pr.cur = 0
     return pr, jacobi2d_iterate(pr, iters, 0, sequence)
 
 
 def jacobi2d_iterate(pr, iters, start=0, sequence=True):
     """`iters` C1 sweeps from sweep `start` on a jacobi2d_program problem (ping-pong
     u0 -> u1 -> u0 ...), as one pk_launch_sequence or one launch call per sweep; returns
-    the buffer id of the result."""
+    the buffer id of the result.  jacobi2d_tb: launches of pr.sweeps sweeps, a remainder
+    as one shorter launch; the ping-pong state is the launch count (pr.cur)."""
     u0, u1 = pr.bufs[:2]
     grid, blk, sc = pr.geom
     launches = []
+    if getattr(pr, "sweeps", 1) > 1:
+        k = pr.sweeps
+        n, rem = divmod(iters, k)
+        for kk in [k] * n + ([rem] if rem else []):
+            a, b = pr.bufs[pr.cur], pr.bufs[1 - pr.cur]
+            s2 = [sc[0], sc[1], kk]
+            launches.append((grid, blk, [a, b, *s2], s2))
+            pr.cur = 1 - pr.cur
+        if sequence and launches:
+            pr.launch_seq(launches)
+        else:
+            for g, b, a, s in launches:
+                pr.launch(g, b, a, s)
+        return pr.bufs[pr.cur]
     for t in range(start, start + iters):
         a, b = (u0, u1) if t % 2 == 0 else (u1, u0)
         launches.append((grid, blk, [a, b, sc[0], sc[1]], sc))

@@ -39,6 +39,14 @@ def jacobi2d(ctx, make, h=72, w=100):
     return kid, _pingpong(geom, u0, u1, ([], [h, w]), 2), {u0: ((h, w), 4), u1: ((h, w), 4)}
 
 
+def jacobi2d_tb(ctx, make, h=72, w=100, k=3):
+    u = synth.jacobi_grid(h, w)
+    kid = abi.pk_builtin_kernel(ctx, "jacobi2d_tb")
+    u0, u1 = make((h, w), 4, u), make((h, w), 4, u)
+    geom = K.jacobi2d_tb_launch(h, w, k)
+    return kid, _pingpong(geom, u0, u1, ([], [h, w, k]), 2), {u0: ((h, w), 4), u1: ((h, w), 4)}
+
+
 def _hotspot(name, ctx, make, h, w, ty, k=4, bdx=K.HOTSPOT_BDX):
     t, p = synth.hotspot_grids(h, w)
     kid = abi.pk_builtin_kernel(ctx, name)
@@ -125,10 +133,10 @@ def tiled(case, tiles):
     return fn
 
 
-_BASE = (jacobi2d, hotspot2d, hotspot2d_regs, hotspot2d_tb2, hotspot2d_tbk(2), hotspot2d_tbk(3), hotspot2d_tbk(4),
+_BASE = (jacobi2d, jacobi2d_tb, hotspot2d, hotspot2d_regs, hotspot2d_tb2, hotspot2d_tbk(2), hotspot2d_tbk(3), hotspot2d_tbk(4),
          hotspot2d_tbk(6), hotspot2d_tbk(8), heat3d, heat3d_regs, heat3d_tb2, heat3d_tb3, nbody, sgemm)
 _B = {f.__name__: f for f in _BASE}
-_TILED = (tiled(_B["jacobi2d"], (2, 2, 1)), tiled(_B["hotspot2d"], (3, 1, 1)), tiled(_B["hotspot2d_regs"], (2, 2, 1)),
+_TILED = (tiled(_B["jacobi2d"], (2, 2, 1)), tiled(_B["jacobi2d_tb"], (2, 2, 1)), tiled(_B["hotspot2d"], (3, 1, 1)), tiled(_B["hotspot2d_regs"], (2, 2, 1)),
           tiled(_B["hotspot2d_tb2"], (3, 1, 1)), tiled(_B["hotspot2d_tbk2"], (3, 1, 1)),
           tiled(_B["hotspot2d_tbk3"], (2, 2, 1)), tiled(_B["hotspot2d_tbk4"], (3, 1, 1)),
           tiled(_B["hotspot2d_tbk8"], (3, 1, 1)), tiled(_B["heat3d"], (2, 1, 2)), tiled(_B["heat3d_tb2"], (2, 1, 2)),

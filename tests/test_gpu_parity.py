@@ -729,6 +729,55 @@ def test_heat3d_tb2_push_bitwise():
     assert np.array_equal(r1, rp) and st["pushed_bytes"] > 0
 
 
+# ------------------------------------------------------------------ K-sweep Jacobi (jacobi2d_tb)
+def _jacobi_tb(u, iters, P, k, sequence=True, per_launch=False):
+    ctx = gpu_ctx(P)
+    pr, _ = K.jacobi2d_program(ctx, u, 0, kernel="jacobi2d_tb", sweeps=k)
+    stale = []
+    if per_launch:
+        for _ in range(iters // k):
+            abi.pk_reset_stats(ctx)
+            out = K.jacobi2d_iterate(pr, k, sequence=False)
+            stale.append(abi.pk_get_stats(ctx)["stale_bytes"])
+    else:
+        out = K.jacobi2d_iterate(pr, iters, sequence=sequence)
+    res = fetch(ctx, out, u.shape)
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return res, st, stale
+
+
+@pytest.mark.parametrize("k", [1, 3, 10, 16])
+@pytest.mark.parametrize("h,w", [(100, 130), (512, 512), (33, 7)])
+def test_jacobi2d_tb_oracle_and_bitwise(h, w, k):
+    """K sweeps per launch (ghost zones): within 1e-5 of the fp64 oracle, bit-identical to
+    the one-sweep jacobi2d run, P-way bit-identical to 1-way with moved == stale, a
+    remainder sweep count as one shorter launch."""
+    u = synth.jacobi_grid(h, w)
+    iters = 20
+    g1, s1, _ = _jacobi_tb(u, iters, 1, k)
+    ok_, err = rel_ok(g1, ok.jacobi2d(u, iters), 1e-5)
+    assert ok_, err
+    ref, _ = _jacobi(u, iters, 1)
+    assert np.array_equal(g1, ref)
+    assert s1["kernel_launches"] == -(-iters // k)
+    for P in (2, 3):
+        gp, st, _ = _jacobi_tb(u, iters, P, k)
+        assert np.array_equal(g1, gp), P
+        assert st["moved_bytes"] == st["stale_bytes"]
+
+
+def test_jacobi2d_tb_stale_hand_derived_on_gpu():
+    """tests/test_oracle_regions_shadow.py's hand count measured through the library: 64^2,
+    P = 2, K = 3: 2 K 64 4 B for the first two launches (uploaded buffers, full rows), then
+    2 K 62 4 B (the boundary columns are co-held after one copy)."""
+    u = synth.jacobi_grid(64, 64)
+    g, _, stale = _jacobi_tb(u, 15, 2, 3, per_launch=True)
+    assert stale == [1536, 1536, 1488, 1488, 1488]
+    ok_, err = rel_ok(g, ok.jacobi2d(u, 15), 1e-5)
+    assert ok_, err
+
+
 # ------------------------------------------------------------------ three-sweep heat (heat3d_tb3)
 def _heat_tb3(u, iters, P, zc, mode=0):
     ctx = gpu_ctx(P, mode)

@@ -726,6 +726,22 @@ def test_heat3d_tb3_regions(d, h, w, zc, P):
     abi.pk_finalize(ctx)
 
 
+@pytest.mark.parametrize("h,w,k", [(64, 64, 1), (64, 64, 5), (70, 100, 10), (33, 31, 16), (3, 3, 2)])
+@pytest.mark.parametrize("P", [1, 2, 3])
+def test_jacobi2d_tb_regions(h, w, k, P):
+    """K sweeps per launch: the dilated, clamped window and the interior writes == brute force."""
+    ctx = host_ctx(P)
+    kk = abi.pk_builtin_kernel(ctx, "jacobi2d_tb")
+    bufs = [abi.pk_register_buffer(ctx, (h, w), 4) for _ in range(2)]
+    grid, blk, sc = K.jacobi2d_tb_launch(h, w, k)
+    for p in range(P):
+        box = abi.pk_partition_grid(ctx, kk, grid, p)
+        lib = _lib_sets(ctx, kk, 5, bufs + [None] * 3, box, blk, sc)
+        ora = _oracle_sets(regions.jacobi2d_tb(box, h, w, k), {0: 4, 1: 4})
+        assert lib == ora
+    abi.pk_finalize(ctx)
+
+
 # ------------------------------------------------------------------ degenerate cases
 def test_degenerate_buffers_and_grids():
     """A zero-element buffer holds no segments; an empty grid launches nothing and moves

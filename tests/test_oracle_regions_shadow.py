@@ -124,6 +124,32 @@ def test_c1_stale_bytes_40800():
     assert sh.stale_bytes == 40800
 
 
+@pytest.mark.parametrize("k", [1, 3, 5])
+def test_jacobi2d_tb_stale_hand_derived(k):
+    """K sweeps per launch (jacobi2d_tb), 64^2, P = 2 (row slabs [0, 32), [32, 64), aligned
+    with the linear H2D split).  Hand count: each partition's window reaches K full rows
+    into the other (all 64 columns, boundary columns included).  Launch 1 reads u0 and
+    launch 2 reads u1 as uploaded: both directions lack K full rows, 2 K 64 4 B.  From
+    launch 3 on, the boundary columns of those rows were copied once (validity mode: the
+    reader became a co-holder, and they are never rewritten), so only the K interior row
+    segments rewritten by the owner move: 2 K 62 4 B."""
+    n, P = 64, 2
+    sh = shadow.Shadow(P)
+    sh.register("u0", n * n, 4, True)
+    sh.register("u1", n * n, 4, True)
+    g = (2, 2, 1)                       # 32 x 32 logical blocks
+    per_launch = []
+    for t in range(5):
+        a, b = ("u0", "u1") if t % 2 == 0 else ("u1", "u0")
+        per = []
+        for p in range(P):
+            acc = regions.jacobi2d_tb(grid.partition_box(g, P, p), n, n, k)
+            per.append({a: (acc[(0, "r")], None), b: (None, acc[(1, "w")])})
+        per_launch.append(sum(sh.launch(per)["stale"]))
+    full, inner = 2 * k * 64 * 4, 2 * k * 62 * 4
+    assert per_launch == [full, full, inner, inner, inner]
+
+
 def test_misaligned_h2d_redistribution_and_paper_mode_redundancy():
     """Jacobi 64^2, P = 3 (SURVEY §8(c) Q2 / paper-vs-validity pin).
 
