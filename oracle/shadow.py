@@ -24,7 +24,7 @@ Readings:
   Q25 halo push (PK_MODE_PUSH, not in the paper, which only pulls): after the update,
       for a push-capable output buffer that this launch does not read, the elements
       writer q wrote that partition p read in the last launch that read the buffer
-      become valid on p as well -- unless q's pushes would need more than 4 contiguous
+      become valid on p as well -- unless q's pushes would need more than 16 contiguous
       byte runs in total (then q pushes nothing; those bytes are pulled later).
 """
 from __future__ import annotations
@@ -87,7 +87,7 @@ def choose_source(mask: int, p: int, nparts: int) -> int:
     return best[1]
 
 
-MAX_PUSH_RUNS = 4
+MAX_PUSH_RUNS = 16
 
 
 def _runs(el):

@@ -34,9 +34,10 @@ constexpr int kThreads = 512;   // 32 columns x 16 rows of threads
 // One CTA per logical block; KS = K is a template parameter so that the window side, the
 // loop trip counts and the shared-memory offsets are compile-time constants (the loops
 // unroll and the cells a thread handles in one sweep are independent instructions).
-template <int KS>
+template <int KS, bool PUSH>
 __global__ void __launch_bounds__(kThreads) k_jacobi2d_tb(const float* __restrict__ in, float* __restrict__ out,
-                                                          int64_t H, int64_t W, int64_t K, pk_partition part) {
+                                                          int64_t H, int64_t W, int64_t K, pk_partition part,
+                                                          PushList push) {
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     asm volatile("griddepcontrol.wait;" ::: "memory");
     constexpr int S = kT + 2 * KS;                 // window side
@@ -100,16 +101,32 @@ __global__ void __launch_bounds__(kThreads) k_jacobi2d_tb(const float* __restric
         const int i = i0 + ty, r = (int)r0 + i, c = (int)c0 + tx;
         if (r < 1 || r > Hi - 2 || c < 1 || c > Wi - 2) continue;
         float* o = out + (int64_t)r * W + c;
-        *o = a[(KS + i) * S + KS + tx];
+        const float v = a[(KS + i) * S + KS + tx];
+        *o = v;
         PK_TRACE_W(o, 4);
+        // fused halo push (PK_MODE_PUSH): only the rows a push range may cover (the K edge rows
+        // of a partition) take the per-range check
+        if (PUSH) {
+            int64_t pa = 0, pb = 0;
+            dev::push_rows(push, r0, r0 + kT, (uint64_t)W * 4u, &pa, &pb);
+            if (dev::in_rows(r, pa, pb)) dev::push1(push, (uint64_t)((int64_t)r * W + c) * 4u, v);
+        }
     }
 }
 
-template <int KS>
-constexpr const void* tb_fn() { return (const void*)k_jacobi2d_tb<KS>; }
-const void* const kTbFns[kMaxK + 1] = {nullptr,     tb_fn<1>(),  tb_fn<2>(),  tb_fn<3>(),  tb_fn<4>(),  tb_fn<5>(),
-                                       tb_fn<6>(),  tb_fn<7>(),  tb_fn<8>(),  tb_fn<9>(),  tb_fn<10>(), tb_fn<11>(),
-                                       tb_fn<12>(), tb_fn<13>(), tb_fn<14>(), tb_fn<15>(), tb_fn<16>()};
+template <int KS, bool P>
+const void* tb_fn() { return (const void*)k_jacobi2d_tb<KS, P>; }
+template <bool P>
+const void* tb_fn_k(int64_t k) {
+    switch (k) {
+        case 1: return tb_fn<1, P>();   case 2: return tb_fn<2, P>();   case 3: return tb_fn<3, P>();
+        case 4: return tb_fn<4, P>();   case 5: return tb_fn<5, P>();   case 6: return tb_fn<6, P>();
+        case 7: return tb_fn<7, P>();   case 8: return tb_fn<8, P>();   case 9: return tb_fn<9, P>();
+        case 10: return tb_fn<10, P>(); case 11: return tb_fn<11, P>(); case 12: return tb_fn<12, P>();
+        case 13: return tb_fn<13, P>(); case 14: return tb_fn<14, P>(); case 15: return tb_fn<15, P>();
+        case 16: return tb_fn<16, P>(); default: return nullptr;
+    }
+}
 
 int describe_jacobi2d_tb(pk_ctx c, pk_kernel k) {
     // scalars: 0 = H, 1 = W, 2 = K.  Logical block (bx, by) = rows [32 by, +32) x columns
@@ -136,11 +153,14 @@ cudaError_t launch_jacobi2d_tb(const LaunchInfo& li) {
     int64_t H = li.scalars[0], W = li.scalars[1], K = li.scalars[2];
     if (K < 1 || K > kMaxK || H < 1 || W < 1 || H >= (int64_t)1 << 30 || W >= (int64_t)1 << 30)
         return cudaErrorInvalidValue;
-    const void* fn = kTbFns[K];
+    const bool push = li.push && li.push->n > 0;
+    const void* fn = push ? tb_fn_k<true>(K) : tb_fn_k<false>(K);
+    PushList pl{};
+    if (li.push) pl = *li.push;
     const size_t smem = (size_t)2 * (kT + 2 * K) * (kT + 2 * K) * sizeof(float);
     KernelDevInfo kd;
     if (cudaError_t e = prepare_kernel(fn, li.device, smem, kThreads, &kd)) return e;
-    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &H, &W, &K, (void*)&li.part};
+    void* argv[] = {(void*)&li.inst[0], (void*)&li.inst[1], &H, &W, &K, (void*)&li.part, &pl};
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     at[0].val.programmaticStreamSerializationAllowed = 1;
@@ -157,8 +177,8 @@ cudaError_t launch_jacobi2d_tb(const LaunchInfo& li) {
 }  // namespace
 
 const Builtin kBuiltinJacobi2dTb = {
-    "jacobi2d_tb", (const void*)k_jacobi2d_tb<1>, 5,
+    "jacobi2d_tb", (const void*)k_jacobi2d_tb<1, false>, 5,
     {PK_ARG_BUFFER, PK_ARG_BUFFER, PK_ARG_SCALAR, PK_ARG_SCALAR, PK_ARG_SCALAR}, -1,
-    describe_jacobi2d_tb, launch_jacobi2d_tb, /*push_arg=*/-1};
+    describe_jacobi2d_tb, launch_jacobi2d_tb, /*push_arg=*/1};
 
 }  // namespace pk

@@ -11,7 +11,7 @@ namespace pk {
 // instance are ALSO stored at dst[i] + offset (another partition's instance of the same
 // buffer, same layout; a peer GPU's memory over NVLink or an IPC mapping) by the kernel
 // that produces them.  Passed to the kernel by value.
-constexpr int kMaxPush = 4;
+constexpr int kMaxPush = 16;
 struct PushList {
     int32_t n;
     int32_t pad;

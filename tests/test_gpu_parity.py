@@ -730,8 +730,8 @@ def test_heat3d_tb2_push_bitwise():
 
 
 # ------------------------------------------------------------------ K-sweep Jacobi (jacobi2d_tb)
-def _jacobi_tb(u, iters, P, k, sequence=True, per_launch=False):
-    ctx = gpu_ctx(P)
+def _jacobi_tb(u, iters, P, k, sequence=True, per_launch=False, mode=0):
+    ctx = gpu_ctx(P, mode)
     pr, _ = K.jacobi2d_program(ctx, u, 0, kernel="jacobi2d_tb", sweeps=k)
     stale = []
     if per_launch:
@@ -765,6 +765,18 @@ def test_jacobi2d_tb_oracle_and_bitwise(h, w, k):
         gp, st, _ = _jacobi_tb(u, iters, P, k)
         assert np.array_equal(g1, gp), P
         assert st["moved_bytes"] == st["stale_bytes"]
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_jacobi2d_tb_push_bitwise(P):
+    """The halo pushed by the producing jacobi2d_tb kernel (PK_MODE_PUSH) instead of pulled:
+    bit-identical to 1-way, the pushed interior rows make later launches move nothing but
+    the boundary columns' first copies."""
+    u = synth.jacobi_grid(100, 130)
+    g1, _, _ = _jacobi_tb(u, 20, 1, 5)
+    gp, st, _ = _jacobi_tb(u, 20, P, 5, mode=abi.PK_MODE_PUSH)
+    assert np.array_equal(g1, gp)
+    assert st["pushed_bytes"] > 0 and st["moved_bytes"] == st["stale_bytes"]
 
 
 def test_jacobi2d_tb_stale_hand_derived_on_gpu():
