@@ -252,8 +252,11 @@ int pk_register_kernel(pk_ctx ctx, const char* name, const void* fn, int nargs,
  * injective; read taps may over-approximate. */
 int pk_declare_affine_access(pk_ctx ctx, pk_kernel k, int arg_index, int mode,
                              const pk_affine_access* tap);
-/* Register one of the library's sm_100a kernels ("jacobi2d", "hotspot2d",
- * "heat3d", "nbody", "sgemm_tf32x3") with its descriptors already declared. */
+/* Register one of the library's sm_100a kernels with its descriptors already declared:
+ * "jacobi2d", "jacobi2d_tb" (K sweeps per launch, scalar 2), "hotspot2d",
+ * "hotspot2d_regs", "hotspot2d_tb2", "hotspot2d_tbk" (K sweeps, scalar 3), "heat3d",
+ * "heat3d_regs", "heat3d_tb2", "heat3d_tb3" (two / three sweeps per launch), "nbody",
+ * "sgemm_tf32x3".  Launch geometry per kernel: DESIGN.md §4 and kernels.py. */
 int pk_builtin_kernel(pk_ctx ctx, const char* name, pk_kernel* out);
 /* __global__ entry of a builtin kernel, for pk_register_kernel + user-declared
  * descriptors.  NULL if unknown. */
@@ -433,9 +436,10 @@ enum {
  * streams virtual partitions' copies too (functional tests on one GPU). */
 /* PK_MODE_PUSH -- the transfer fused into the producing kernel (B200 design; the paper
  * only pulls).  For a kernel whose builtin can push its output (jacobi2d,
- * hotspot2d, hotspot2d_tbk, heat3d), the library predicts that the next reader of the
- * written buffer reads what its last reader read: the bytes partition q writes that
- * partition p read last time (W_q n R_p, at most 4 ranges per writer, 4-byte aligned)
+ * jacobi2d_tb, hotspot2d, hotspot2d_tbk, heat3d, heat3d_tb2, heat3d_tb3), the library
+ * predicts that the next reader of the written buffer reads what its last reader read:
+ * the bytes partition q writes that partition p read last time (W_q n R_p, at most 16
+ * ranges per writer, 4-byte aligned)
  * are stored by q's kernel ALSO into p's instance (peer stores over NVLink/NVSwitch, or
  * an IPC mapping in peer-memory SPMD), and the tracker marks p as a holder, so the next
  * launch finds nothing stale and issues no copy.  A wrong prediction only costs bytes:
