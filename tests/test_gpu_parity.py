@@ -882,3 +882,49 @@ def test_async_host_copies_pipelined_contexts(P):
     for s in range(5):
         assert np.array_equal(outs[s].numpy(), ref), s
     assert st["moved_bytes"] == st["stale_bytes"]
+
+
+# ------------------------------------------------------------------ randomised launch programs
+def _random_program(P, mode, seed, h=200, w=1028):
+    """One context, two kernels (one-sweep hotspot2d and four-sweep hotspot2d_tbk) on the same
+    ping-pong buffers, and a seeded random mix of launches, re-uploads of the current field and
+    mid-program reads -- the hazards of the event DAG (RAW on copies' sources, WAR on both sides,
+    pushed halos, graph replay vs eager) in orders no hand-written test has."""
+    rng = np.random.default_rng(seed)
+    t, p = synth.hotspot_grids(h, w)
+    t2 = (t + np.float32(1.5)).astype(np.float32)
+    ctx = gpu_ctx(P, mode)
+    k1 = abi.pk_builtin_kernel(ctx, "hotspot2d")
+    k4 = abi.pk_builtin_kernel(ctx, "hotspot2d_tbk")
+    b = [abi.pk_register_buffer(ctx, (h, w), 4, host_init=t), abi.pk_register_buffer(ctx, (h, w), 4)]
+    pw = abi.pk_register_buffer(ctx, (h, w), 4, host_init=p)
+    g1, bl1, s1 = K.hotspot2d_launch(h, w, 16, K.HOTSPOT_BDX)
+    g4, bl4, s4 = K.hotspot2d_tbk_launch(h, w, 16, 4)
+    cur, reads = 0, []
+    for op in rng.choice(["s1", "s1", "s4", "s4", "s4", "up", "rd"], size=40):
+        if op == "s1":
+            abi.pk_launch_partitioned(ctx, k1, g1, bl1, [b[cur], pw, b[1 - cur], h, w, s1[2]], s1)
+            cur = 1 - cur
+        elif op == "s4":
+            abi.pk_launch_partitioned(ctx, k4, g4, bl4, [b[cur], pw, b[1 - cur], h, w, s4[2]], s4)
+            cur = 1 - cur
+        elif op == "up":
+            abi.pk_copy_from_host(ctx, b[cur], t2 if len(reads) % 2 else t)
+        else:
+            reads.append(fetch(ctx, b[cur], (h, w)))
+    reads.append(fetch(ctx, b[cur], (h, w)))
+    st = abi.pk_get_stats(ctx)
+    abi.pk_finalize(ctx)
+    return reads, st
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("P,mode", [(3, 0), (5, 0), (5, abi.PK_MODE_PUSH), (4, abi.PK_MODE_NO_GRAPHS),
+                                    (3, abi.PK_MODE_GLOBAL_BARRIER), (5, abi.PK_MODE_SINGLE_OWNER)])
+def test_random_launch_programs_bitwise(seed, P, mode):
+    ref, _ = _random_program(1, 0, seed)
+    got, st = _random_program(P, mode, seed)
+    assert len(got) == len(ref)
+    for r, g in zip(ref, got):
+        assert np.array_equal(r, g)
+    assert st["moved_bytes"] == st["stale_bytes"] or mode == abi.PK_MODE_PUSH
