@@ -885,7 +885,7 @@ def test_async_host_copies_pipelined_contexts(P):
 
 
 # ------------------------------------------------------------------ randomised launch programs
-def _random_program(P, mode, seed, h=200, w=1028):
+def _random_program(P, mode, seed, h=200, w=1028, tiles=None):
     """One context, two kernels (one-sweep hotspot2d and four-sweep hotspot2d_tbk) on the same
     ping-pong buffers, and a seeded random mix of launches, re-uploads of the current field and
     mid-program reads -- the hazards of the event DAG (RAW on copies' sources, WAR on both sides,
@@ -896,6 +896,9 @@ def _random_program(P, mode, seed, h=200, w=1028):
     ctx = gpu_ctx(P, mode)
     k1 = abi.pk_builtin_kernel(ctx, "hotspot2d")
     k4 = abi.pk_builtin_kernel(ctx, "hotspot2d_tbk")
+    if tiles:   # NEXT-2 tile partitions: column cuts make strided halo copies
+        abi.pk_set_partition_shape(ctx, k1, tiles)
+        abi.pk_set_partition_shape(ctx, k4, tiles)
     b = [abi.pk_register_buffer(ctx, (h, w), 4, host_init=t), abi.pk_register_buffer(ctx, (h, w), 4)]
     pw = abi.pk_register_buffer(ctx, (h, w), 4, host_init=p)
     g1, bl1, s1 = K.hotspot2d_launch(h, w, 16, K.HOTSPOT_BDX)
@@ -928,3 +931,16 @@ def test_random_launch_programs_bitwise(seed, P, mode):
     for r, g in zip(ref, got):
         assert np.array_equal(r, g)
     assert st["moved_bytes"] == st["stale_bytes"] or mode == abi.PK_MODE_PUSH
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+@pytest.mark.parametrize("tiles,mode", [((2, 2, 1), 0), ((3, 2, 1), 0), ((2, 3, 1), abi.PK_MODE_NO_GRAPHS),
+                                        ((3, 1, 1), abi.PK_MODE_SINGLE_OWNER)])
+def test_random_launch_programs_tiles_bitwise(seed, tiles, mode):
+    """The random programs on tile partitions (2-D and 3-D strided halo copies, the SM
+    strided-copy kernel for narrow column halos)."""
+    ref, _ = _random_program(1, 0, seed)
+    got, st = _random_program(tiles[0] * tiles[1] * tiles[2], mode, seed, tiles=tiles)
+    for r, g in zip(ref, got):
+        assert np.array_equal(r, g)
+    assert st["moved_bytes"] == st["stale_bytes"] and st["strided_copies"] + st["copy_kernels"] > 0
