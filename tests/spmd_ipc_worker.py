@@ -195,12 +195,54 @@ def main():
         record("lifecycle", np.array_equal(g, one_way(f6)))
     dist.barrier()
 
+    # --- seeded random launch programs (two kernels on shared ping-pong buffers, collective
+    # re-uploads and mid-program gathers), pulled and pushed halos: every read bit-identical
+    for seed in (0, 1):
+        for mode in (0, abi.PK_MODE_PUSH):
+            ctx = new_ctx(mode)
+            reads = _random_program(ctx, seed, lambda c, bb, sh: gather(c, bb, sh))
+            s = summed(ctx)
+            abi.pk_finalize(ctx)
+            if rank == 0:
+                ref = one_way(lambda c: _random_program(c, seed, _fetch))
+                ok = len(reads) == len(ref) and all(np.array_equal(x, y) for x, y in zip(reads, ref))
+                record(f"random/{seed}/mode{mode}", ok and s["stale"] == s["moved"], reads=len(reads), **s)
+            dist.barrier()
+
     if rank == 0:
         with open(out_path, "w") as f:
             json.dump(report, f, indent=1)
         print("SPMD-IPC ALL OK", json.dumps({k: v["ok"] for k, v in report["cases"].items()}), flush=True)
     dist.barrier()
     dist.destroy_process_group()
+
+
+def _random_program(ctx, seed, read, h=200, w=1028):
+    """tests/test_gpu_parity.py's random launch program through any context; `read(ctx, buf,
+    shape)` returns the host copy (a collective gather in SPMD)."""
+    rng = np.random.default_rng(seed)
+    t, p = synth.hotspot_grids(h, w)
+    t2 = (t + np.float32(1.5)).astype(np.float32)
+    k1 = abi.pk_builtin_kernel(ctx, "hotspot2d")
+    k4 = abi.pk_builtin_kernel(ctx, "hotspot2d_tbk")
+    b = [abi.pk_register_buffer(ctx, (h, w), 4, host_init=t), abi.pk_register_buffer(ctx, (h, w), 4)]
+    pw = abi.pk_register_buffer(ctx, (h, w), 4, host_init=p)
+    g1, bl1, s1 = K.hotspot2d_launch(h, w, 16, K.HOTSPOT_BDX)
+    g4, bl4, s4 = K.hotspot2d_tbk_launch(h, w, 16, 4)
+    cur, reads = 0, []
+    for op in rng.choice(["s1", "s1", "s4", "s4", "s4", "up", "rd"], size=30):
+        if op == "s1":
+            abi.pk_launch_partitioned(ctx, k1, g1, bl1, [b[cur], pw, b[1 - cur], h, w, s1[2]], s1)
+            cur = 1 - cur
+        elif op == "s4":
+            abi.pk_launch_partitioned(ctx, k4, g4, bl4, [b[cur], pw, b[1 - cur], h, w, s4[2]], s4)
+            cur = 1 - cur
+        elif op == "up":
+            abi.pk_copy_from_host(ctx, b[cur], t2 if len(reads) % 2 else t)
+        else:
+            reads.append(read(ctx, b[cur], (h, w)))
+    reads.append(read(ctx, b[cur], (h, w)))
+    return reads
 
 
 def _fetch(ctx, buf, shape):

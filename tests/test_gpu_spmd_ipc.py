@@ -45,7 +45,7 @@ def test_spmd_ipc_processes_match_one_way(world, flags_on_sm, tmp_path):
     assert rep["world"] == world
     names = set(rep["cases"])
     assert {"hotspot2d/mode0", "hotspot2d_tb2/mode0", "hotspot2d_tbk/mode0", "hotspot2d/oracle", "jacobi2d/C1", "heat3d", "nbody",
-            "sgemm", "lifecycle"} <= names
+            "sgemm", "lifecycle", "random/0/mode0", "random/1/mode64"} <= names
     assert all(c["ok"] for c in rep["cases"].values()), rep
     if world == 2:
         assert rep["cases"]["jacobi2d/C1"]["stale"] == 40800
