@@ -230,17 +230,24 @@ def hotspot2d_setup(ctx, temp_host, power_host, ty=HOTSPOT_TY, bdx=HOTSPOT_BDX, 
     return pr
 
 
-def hotspot2d_iterate(pr, iters, start=0):
+def hotspot2d_iterate(pr, iters, start=0, sequence=False):
     """`iters` Hotspot time steps starting at step `start` (the tb2/tbk kernels advance
-    pr.sweeps steps per launch: iters and start must then be multiples of it)."""
+    pr.sweeps steps per launch: iters and start must then be multiples of it);
+    sequence=True issues them as one pk_launch_sequence."""
     (t0, t1, pw), (h, w) = pr.tb, pr.hw
     grid, blk, sc = pr.geom
     k = pr.sweeps
     if iters % k or start % k:
         raise ValueError(f"this kernel advances {k} steps per launch")
+    launches = []
     for t in range(start // k, (start + iters) // k):
         a, b = (t0, t1) if t % 2 == 0 else (t1, t0)
-        pr.launch(grid, blk, [a, pw, b, h, w, sc[2]], sc)
+        launches.append((grid, blk, [a, pw, b, h, w, sc[2]], sc))
+    if sequence and launches:
+        pr.launch_seq(launches)
+    else:
+        for g, bl, a, s in launches:
+            pr.launch(g, bl, a, s)
     return t1 if ((start + iters) // k) % 2 == 1 else t0
 
 
