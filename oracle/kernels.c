@@ -56,6 +56,23 @@ void oracle_jacobi2d(double* u0, double* u1, int64_t h, int64_t w, int iters) {
     }
 }
 
+/* The same sweeps in fp32 storage AND arithmetic, each operation rounded to nearest as
+ * written (-ffp-contract=off: no fused multiply-add; x86-64 SSE: no extended precision).
+ * Not the reference for tolerances (that is the fp64 definition above): SURVEY.md §8(c)'s
+ * optional strong pin -- a kernel that evaluates the same expression in the same order in
+ * fp32 (jacobi2d, jacobi2d_tb use __fadd_rn / __fmul_rn) must match it bit for bit. */
+void oracle_jacobi2d_f32(float* u0, float* u1, int64_t h, int64_t w, int iters) {
+    for (int t = 0; t < iters; ++t) {
+        const float* in = t % 2 == 0 ? u0 : u1;
+        float* out = t % 2 == 0 ? u1 : u0;
+        #pragma omp parallel for schedule(static)
+        for (int64_t i = 1; i < h - 1; ++i)
+            for (int64_t j = 1; j < w - 1; ++j)
+                out[i * w + j] = 0.25f * (((in[(i - 1) * w + j] + in[(i + 1) * w + j])
+                                           + in[i * w + j - 1]) + in[i * w + j + 1]);
+    }
+}
+
 /* ---------------- C2: Hotspot (Rodinia form), clamped borders ---------------- */
 /* For every cell (i, j), with N/S/E/W neighbours clamped to the grid:
  *   out = C + cap * (P + (S + N - 2C) * ry1 + (E + W - 2C) * rx1 + (amb - C) * rz1)

@@ -39,6 +39,7 @@ def lib():
         _lib = ctypes.CDLL(path)
         L = _lib
         L.oracle_jacobi2d.argtypes = [_D, _D, _i64, _i64, ctypes.c_int]
+        L.oracle_jacobi2d_f32.argtypes = [_F, _F, _i64, _i64, ctypes.c_int]
         L.oracle_hotspot2d.argtypes = [_D, _D, _D, _i64, _i64, ctypes.c_int] + [ctypes.c_double] * 5
         L.oracle_heat3d.argtypes = [_D, _D, _i64, _i64, _i64, ctypes.c_int, ctypes.c_double]
         L.oracle_gemm.argtypes = [_D, _D, _D, _i64, _i64, _i64]
@@ -63,6 +64,16 @@ def jacobi2d(u: np.ndarray, iters: int) -> np.ndarray:
     u1 = u0.copy()
     h, w = u0.shape
     lib().oracle_jacobi2d(_dp(u0), _dp(u1), h, w, iters)
+    return u0 if iters % 2 == 0 else u1
+
+
+def jacobi2d_f32(u: np.ndarray, iters: int) -> np.ndarray:
+    """C1 in fp32 storage and arithmetic, each operation rounded as written (no FMA): the
+    bit-exact mirror of a kernel that evaluates the same expression in the same order."""
+    u0 = np.ascontiguousarray(u, dtype=np.float32).copy()
+    u1 = u0.copy()
+    h, w = u0.shape
+    lib().oracle_jacobi2d_f32(u0.ctypes.data_as(_F), u1.ctypes.data_as(_F), h, w, iters)
     return u0 if iters % 2 == 0 else u1
 
 

@@ -779,6 +779,20 @@ def test_jacobi2d_tb_push_bitwise(P):
     assert st["pushed_bytes"] > 0 and st["moved_bytes"] == st["stale_bytes"]
 
 
+@pytest.mark.parametrize("h,w", [(512, 512), (100, 130)])
+def test_jacobi_bit_exact_vs_fp32_cpu_mirror(h, w):
+    """SURVEY §8(c)'s optional strong pin: jacobi2d and jacobi2d_tb evaluate the C1 update with
+    __fadd_rn / __fmul_rn in the oracle's order, so after 20 sweeps they equal the fp32 CPU
+    mirror (oracle/kernels.c, -ffp-contract=off) bit for bit, at P = 1 and 2."""
+    u = synth.jacobi_grid(h, w)
+    ref = ok.jacobi2d_f32(u, 20)
+    for P in (1, 2):
+        g1, _ = _jacobi(u, 20, P)
+        assert np.array_equal(g1, ref), P
+        g5, _, _ = _jacobi_tb(u, 20, P, 5)
+        assert np.array_equal(g5, ref), P
+
+
 def test_jacobi2d_tb_stale_hand_derived_on_gpu():
     """tests/test_oracle_regions_shadow.py's hand count measured through the library: 64^2,
     P = 2, K = 3: 2 K 64 4 B for the first two launches (uploaded buffers, full rows), then

@@ -90,6 +90,28 @@ def test_jacobi_boundary_untouched_and_asymmetric_input():
     assert np.array_equal(out[0], u[0]) and np.array_equal(out[:, -1], u[:, -1])
 
 
+def test_jacobi_f32_mirror_brute_force_and_fp64():
+    """The fp32 mirror (SURVEY §8(c) optional strong pin): equal bit for bit to a per-cell
+    numpy float32 evaluation of the same expression in the same order (each operation rounded
+    to fp32, no FMA) on a tiny ragged input over three ping-pong sweeps; within 1e-6 of the fp64
+    definition after 10 sweeps on 64^2; the harmonic field i*j stays an exact fixed point."""
+    rng = np.random.default_rng(8)
+    u = rng.uniform(size=(9, 13)).astype(np.float32)
+    a, b = u.copy(), u.copy()
+    q = np.float32(0.25)
+    for _ in range(3):
+        for r in range(1, 8):
+            for c in range(1, 12):
+                b[r, c] = q * (((a[r - 1, c] + a[r + 1, c]) + a[r, c - 1]) + a[r, c + 1])
+        a, b = b, a
+    assert np.array_equal(ok.jacobi2d_f32(u, 3), a)
+    v = np.random.default_rng(9).uniform(size=(64, 64)).astype(np.float32)
+    np.testing.assert_allclose(ok.jacobi2d_f32(v, 10), ok.jacobi2d(v, 10), rtol=1e-6, atol=0)
+    i = np.arange(64)[:, None].astype(np.float32)
+    j = np.arange(64)[None, :].astype(np.float32)
+    assert np.array_equal(ok.jacobi2d_f32(i * j, 10), i * j)
+
+
 # --------------------------- C2 Hotspot (reading Q14) ---------------------------
 def test_hotspot_uniform_recurrence():
     h, w, it = 17, 24, 9
